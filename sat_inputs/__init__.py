@@ -1,0 +1,141 @@
+"""Seeded synthetic inputs shared by the oracle side and the CUDA side.
+
+This module holds NO SAT arithmetic: only a counter-based generator
+(splitmix64 of (seed, global element index)), implemented twice -- numpy for
+host/oracle use and torch (CPU or CUDA) for device-resident bench inputs --
+producing identical values.  Element (b, i, j) of a batch x rows x cols tensor
+has global counter ``(b*rows + i)*cols + j``; a row strip starting at global row
+``row0`` reproduces the same elements as the full matrix (used by the sharded
+and streaming paths).
+
+Distributions:
+  int32 "u32"  : low 32 bits of the hash (uniform 32-bit, wraps at once)
+  int32 "u8"   : hash & 255 (8-bit image-like pixels)
+  int32 "ones" : all ones (closed form (i+1)(j+1))
+  float32 "unit": (hash >> 40) * 2^-24, dyadic uniform in [0, 1)
+  float32 "ones": all ones (exact in float32 while the SAT stays <= 2^24)
+"""
+from __future__ import annotations
+
+import numpy as np
+
+_GOLDEN = np.uint64(0x9E3779B97F4A7C15)
+_M1 = np.uint64(0xBF58476D1CE4E5B9)
+_M2 = np.uint64(0x94D049BB133111EB)
+
+INT_DISTS = ("u32", "u8", "ones")
+FLOAT_DISTS = ("unit", "ones")
+
+
+def _splitmix_np(ctr: np.ndarray, seed: int) -> np.ndarray:
+    with np.errstate(over="ignore"):
+        z = np.uint64(seed & 0xFFFFFFFFFFFFFFFF) + (ctr + np.uint64(1)) * _GOLDEN
+        z = (z ^ (z >> np.uint64(30))) * _M1
+        z = (z ^ (z >> np.uint64(27))) * _M2
+        return z ^ (z >> np.uint64(31))
+
+
+def _counters_np(shape, row0: int, cols: int, batch_rows: int | None = None):
+    if len(shape) == 2:
+        r, c = shape
+        i = np.arange(row0, row0 + r, dtype=np.uint64)[:, None]
+        j = np.arange(c, dtype=np.uint64)[None, :]
+        return i * np.uint64(cols) + j
+    b, r, c = shape
+    bi = np.arange(b, dtype=np.uint64)[:, None, None]
+    i = np.arange(r, dtype=np.uint64)[None, :, None]
+    j = np.arange(c, dtype=np.uint64)[None, None, :]
+    return (bi * np.uint64(r) + i) * np.uint64(c) + j
+
+
+def _finish_np(h: np.ndarray, dtype: str, dist: str) -> np.ndarray:
+    if dtype == "int32":
+        if dist == "u32":
+            return (h & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32)
+        if dist == "u8":
+            return (h & np.uint64(0xFF)).astype(np.int32)
+        if dist == "ones":
+            return np.ones(h.shape, dtype=np.int32)
+    elif dtype == "float32":
+        if dist == "unit":
+            return ((h >> np.uint64(40)).astype(np.float64) * 2.0 ** -24).astype(np.float32)
+        if dist == "ones":
+            return np.ones(h.shape, dtype=np.float32)
+    raise ValueError(f"unknown dtype/dist {dtype}/{dist}")
+
+
+def make_np(rows: int, cols: int, dtype: str = "int32", dist: str | None = None,
+            seed: int = 0, row0: int = 0, batch: int | None = None) -> np.ndarray:
+    """Host (numpy) input: (rows, cols) or (batch, rows, cols)."""
+    dist = dist or ("u32" if dtype == "int32" else "unit")
+    shape = (rows, cols) if batch is None else (batch, rows, cols)
+    if dist == "ones":
+        return _finish_np(np.zeros(shape, dtype=np.uint64), dtype, dist)
+    ctr = _counters_np(shape, row0, cols)
+    return _finish_np(_splitmix_np(ctr, seed), dtype, dist)
+
+
+# ------------------------------ torch twin ---------------------------------
+def _i64(u: int) -> int:
+    u &= 0xFFFFFFFFFFFFFFFF
+    return u - (1 << 64) if u >= (1 << 63) else u
+
+
+def _lsr(z, k: int):
+    """Logical right shift of an int64 tensor holding uint64 bits."""
+    import torch
+    return torch.bitwise_and(torch.bitwise_right_shift(z, k), (1 << (64 - k)) - 1)
+
+
+def _splitmix_torch(ctr, seed: int):
+    z = (ctr + 1) * _i64(0x9E3779B97F4A7C15) + _i64(seed)
+    z = torch_xor(z, _lsr(z, 30)) * _i64(0xBF58476D1CE4E5B9)
+    z = torch_xor(z, _lsr(z, 27)) * _i64(0x94D049BB133111EB)
+    return torch_xor(z, _lsr(z, 31))
+
+
+def torch_xor(a, b):
+    import torch
+    return torch.bitwise_xor(a, b)
+
+
+def make_torch(rows: int, cols: int, dtype: str = "int32", dist: str | None = None,
+               seed: int = 0, row0: int = 0, batch: int | None = None,
+               device="cpu", out=None, chunk_rows: int = 2048):
+    """Same values as :func:`make_np`, generated with torch ops on ``device``.
+
+    Generates ``chunk_rows`` rows at a time (int64 temporaries) so that very
+    large matrices fit; writes into ``out`` if given.
+    """
+    import torch
+    dist = dist or ("u32" if dtype == "int32" else "unit")
+    tdt = torch.int32 if dtype == "int32" else torch.float32
+    shape = (rows, cols) if batch is None else (batch, rows, cols)
+    if out is None:
+        out = torch.empty(shape, dtype=tdt, device=device)
+    if dist == "ones":
+        out.fill_(1)
+        return out
+    flat = out.view(-1, cols)            # (batch*rows, cols)
+    total_rows = flat.shape[0]
+    j = torch.arange(cols, dtype=torch.int64, device=out.device)
+    for s in range(0, total_rows, chunk_rows):
+        e = min(total_rows, s + chunk_rows)
+        i = torch.arange(s, e, dtype=torch.int64, device=out.device) + row0
+        ctr = i[:, None] * cols + j[None, :]
+        h = _splitmix_torch(ctr, seed)
+        if dtype == "int32":
+            if dist == "u32":
+                v = torch.bitwise_and(h, 0xFFFFFFFF)
+                v = torch.where(v >= (1 << 31), v - (1 << 32), v).to(torch.int32)
+            elif dist == "u8":
+                v = torch.bitwise_and(h, 0xFF).to(torch.int32)
+            else:
+                raise ValueError(dist)
+        else:
+            if dist != "unit":
+                raise ValueError(dist)
+            v = (_lsr(h, 40).to(torch.float64) * 2.0 ** -24).to(torch.float32)
+        flat[s:e].copy_(v)
+        del ctr, h, v
+    return out
