@@ -1,0 +1,473 @@
+#!/usr/bin/env python
+"""bench.py -- libsat throughput on B200 (driver contract).
+
+Default workload (BASELINE.json config 4, the one the metric "... at
+1/2/4/8 B200" is quoted on; it fits one GPU): the SAT of one 65536 x 65536
+int32 matrix (uint32 wrapping arithmetic), 1R1W.  At N=1 one GPU computes it
+with one kernel launch per step; at N>1 the matrix is split into N row strips
+(one per rank) and each step is: column totals -> NCCL all-gather -> rank
+exclusive scan -> seeded 1R1W (strong scaling: total work fixed).
+
+Timing: W untimed warm-up steps, then exactly K steps bracketed by barrier +
+cuda synchronize, CUDA events on the launching stream, max over ranks.  Inputs
+(16 GiB) are far larger than L2 (126 MB), so no flush is needed.
+`--impl reference` times the CPU oracle (the reference arm of this tier).
+Other BASELINE configs: `--config cfg1|cfg2|cfg3|cfg3b|cfg4|cfg5`.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BASELINE_METRIC = "SAT elements/sec and % of HBM roofline (1R1W bytes) at 1/2/4/8 B200"
+
+CONFIGS = {
+    # name: (rows, cols, batch, dtype, variant, description)
+    "cfg1": (1024, 1024, None, "int32", "1r1w", "cfg1: 1024x1024 int32 SAT, 1R1W"),
+    "cfg2": (4096, 4096, None, "float32", "1r1w", "cfg2: 4096x4096 float32 SAT"),
+    "cfg3": (18432, 18432, None, "int32", "1r1w", "cfg3: 18432x18432 int32 SAT, 1R1W"),
+    "cfg3b": (16384, 16384, None, "int32", "1r1w", "cfg3': 16384x16384 int32 SAT, 1R1W (north-star gate)"),
+    "cfg4": (65536, 65536, None, "int32", "1r1w",
+             "cfg4: 65536x65536 int32 SAT, row strips over N GPUs, 1R1W"),
+    "cfg5": (1080, 1920, 32, "float32", "1r1w",
+             "cfg5: 32 images/GPU x 1080x1920 float32 SATs (data parallel)"),
+}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ------------------------------------------------------------------ clocks
+REASON_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clocks_setting"}
+
+
+class ClockSampler:
+    """nvidia-smi sampled every 100 ms during the timed region."""
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 3:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+                bits = int(parts[2], 16)
+            except ValueError:
+                continue
+            for b, name in REASON_BITS.items():
+                if bits & b:
+                    reasons.add(name)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx),
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ helpers
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def ncu_traffic(workload_key: str, kernel_regex: str = "sat_band_kernel"):
+    """Per-launch DRAM bytes of the dominant kernel from the committed ncu
+    summary (profiles/ncu_summary.json), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    e = d.get(workload_key)
+    if not e:
+        return None
+    return e.get("dram_bytes_per_launch")
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_sample_rate(rows: int, cols: int, dtype: str, seed: int, sample_rows: int,
+                       batch=None):
+    """Time the CPU oracle (single-threaded C, as it stands) on the first
+    `sample_rows` rows of the workload; returns (elements/s, elements, seconds)."""
+    import numpy as np
+    import oracle
+    from sat_inputs import make_torch
+    import torch
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    sr = min(rows, sample_rows)
+    x = make_torch(sr, cols, dtype, "u32" if dtype == "int32" else "unit", seed=seed,
+                   device=dev).cpu().numpy()
+    oracle.build()
+    t0 = time.perf_counter()
+    st = oracle.Stream(cols, dtype == "int32")
+    step = max(1, (1 << 24) // cols)
+    for r0 in range(0, sr, step):
+        st.feed(x[r0:r0 + step])
+    dt = time.perf_counter() - t0
+    return sr * cols / dt, sr * cols, dt
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args, cfg_key):
+    rows, cols, batch, dtype, variant, desc = CONFIGS[cfg_key]
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import numpy as np
+    import oracle
+    from sat_inputs import make_np
+    oracle.build()
+    # each step: the oracle on a bounded sample (full width, `srows` rows)
+    srows = max(1, min(rows, (1 << 24) // cols))
+    x = make_np(srows, cols, dtype, "u32" if dtype == "int32" else "unit", seed=1)
+    for _ in range(args.warmup):
+        oracle.sat(x)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.sat(x)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    elems = srows * cols
+    value = elems * args.steps / tot
+    line = {
+        "impl": "reference", "metric": BASELINE_METRIC, "value": value, "unit": "elem/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1000 * tot / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32" if dtype == "int32" else "f64",
+        "data": "synthetic", "config": {"workload": desc + " [oracle sample]"},
+        "cpu_baseline": {"value": value, "unit": "elem/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{srows} rows x {cols} cols per step (first rows of the workload)",
+                         "cpu": cpu_model()},
+        "e2e": {"value": value, "unit": "elem/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=None)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="cfg4", choices=sorted(CONFIGS))
+    ap.add_argument("--variant", default=None)
+    ap.add_argument("--tile-rows", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-sample-rows", type=int, default=None)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        ap.error("--warmup must be >= 3")
+    cfg_key = args.config
+    rows, cols, batch, dtype, variant, desc = CONFIGS[cfg_key]
+    if args.variant:
+        variant = args.variant
+    if args.steps is None:
+        args.steps = {"cfg1": 2000, "cfg2": 1000, "cfg3": 300, "cfg3b": 400, "cfg4": 200,
+                      "cfg5": 500}[cfg_key]
+    if args.impl == "reference":
+        return run_reference(args, cfg_key)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_kasagini14_b200 as libsat
+    from paper_conf_icpp_kasagini14_b200.dist import partition_rows
+    from sat_inputs import make_torch
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    tdt = torch.int32 if dtype == "int32" else torch.float32
+    dist_name = "u32" if dtype == "int32" else "unit"
+    eb = 4
+
+    # ---------------- per-rank work unit
+    if batch is None:
+        if world > 1:
+            r0, r1 = partition_rows(rows, world, rank)
+        else:
+            r0, r1 = 0, rows
+        x = make_torch(r1 - r0, cols, dtype, dist_name, seed=4001, row0=r0, device=dev)
+        y = torch.empty_like(x)
+        my_elems = (r1 - r0) * cols
+        total_elems = rows * cols
+        scaling = "strong"
+    else:
+        # data parallel images: `batch` images per GPU (weak scaling)
+        x = make_torch(rows, cols, dtype, dist_name, seed=5001 + rank, batch=batch, device=dev)
+        y = torch.empty_like(x)
+        my_elems = batch * rows * cols
+        total_elems = my_elems * world
+        scaling = "weak"
+    sharded = world > 1 and batch is None
+    opts = dict(tile_rows=args.tile_rows) if args.tile_rows else {}
+
+    launches = [0]
+
+    if sharded:
+        P = world
+        gathered = torch.empty(P * cols, dtype=tdt, device=dev)
+        send = torch.empty(cols, dtype=tdt, device=dev)
+
+        def step(ev=None):
+            n = 0
+            if rank < P - 1:
+                libsat.column_totals(x, out=send)
+                n += libsat.last_launch_count()
+            else:
+                send.zero_()
+            dist.all_gather_into_tensor(gathered, send)
+            carry = None
+            if rank > 0:
+                carry = libsat.rank_exscan(gathered.view(P, cols), rank)
+                n += libsat.last_launch_count()
+            if ev:
+                ev[0].record(stream)
+            libsat.sat_seeded(x, carry_row=carry, out=y)
+            if ev:
+                ev[1].record(stream)
+            n += libsat.last_launch_count()
+            launches[0] += n
+    else:
+        def step(ev=None):
+            if ev:
+                ev[0].record(stream)
+            if batch is None:
+                libsat.sat(x, variant=variant, out=y, **opts)
+            else:
+                libsat.sat_batched(x, variant=variant, out=y, **opts)
+            if ev:
+                ev[1].record(stream)
+            launches[0] += libsat.last_launch_count()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---------------- warm-up + quick parity re-check of the timed path
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    parity = None
+    if rank == 0 and batch is None and not sharded:
+        import numpy as np
+        import oracle
+        srow = min(r1 - r0, 256)
+        a = x[:srow].cpu().numpy()
+        ref = oracle.sat(a)
+        got = y[:srow].cpu().numpy()
+        parity = bool(np.array_equal(got, ref)) if dtype == "int32" else \
+            bool(oracle.max_rel_err(got, ref) <= 1e-5)
+
+    # ---------------- timed region
+    launches[0] = 0
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    barrier()
+    with ClockSampler(local) as clk:
+        time.sleep(0.3)                     # let the sampler start
+        barrier()
+        ev0.record(stream)
+        for i in range(args.steps):
+            step(kev[i])
+        ev1.record(stream)
+        barrier()
+    kern_ms = [a.elapsed_time(b) for a, b in kev]
+    ms_local = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms_local, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_total, kern_avg_ms = float(t[0]), float(t[1])
+    ms_per_step = ms_total / args.steps
+    value = total_elems * args.steps / (ms_total / 1e3)
+    clocks = clk.summary()
+
+    # ---------------- roofline of the dominant kernel (the band kernel)
+    peak, peak_kind = measured_peaks()
+    alg_bytes = 2 * eb * my_elems                      # 1R1W: one read + one write
+    if variant == "2r2w":
+        alg_bytes = 4 * eb * my_elems
+    elif variant == "2r1w":
+        alg_bytes = 3 * eb * my_elems
+    achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9
+    traffic = ncu_traffic(f"{cfg_key}:{variant}:n{world}")
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "peak_kind": peak_kind, "kernel": "sat_band_kernel",
+                "alg_bytes_per_launch": alg_bytes, "kernel_ms": round(kern_avg_ms, 4),
+                "frac_of_8TBs": round(achieved / 8000.0, 4)}
+
+    # ---------------- end to end through the public API from pinned host memory
+    e2e = None
+    if not args.no_e2e:
+        e2e = run_e2e(args, libsat, x, rows, cols, batch, dtype, world, rank, dev, sharded,
+                      total_elems, barrier)
+
+    # ---------------- CPU oracle baseline (rank 0, N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        sr = args.cpu_sample_rows or max(1, min(rows, (1 << 30) // cols))
+        rate, n_el, secs = oracle_sample_rate(rows, cols, dtype, 4001, sr, batch)
+        cpu = {"value": rate, "unit": "elem/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {min(rows, sr)} rows x {cols} cols of the workload "
+                         f"({n_el} elements, {secs:.1f} s, single-threaded C)",
+               "cpu": cpu_model(), "host_cores": os.cpu_count()}
+
+    if rank == 0:
+        line = {
+            "metric": BASELINE_METRIC, "value": value, "unit": "elem/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
+            "dtype": "u32" if dtype == "int32" else "f32",
+            "data": "synthetic (splitmix64 counter hash: uniform 32-bit int / dyadic [0,1) float)",
+            "config": {"workload": desc + (f" [{variant}]" if variant != "1r1w" else ""),
+                       "rows": rows, "cols": cols, "batch": batch,
+                       "parallelism": (f"row-strips x{world}" if sharded else
+                                       (f"dp{world}" if world > 1 else "1 GPU")),
+                       "l2": "inputs > L2, no flush" if my_elems * eb > 4 * 126e6 else
+                             "inputs near L2 size: hot-L2 number",
+                       "tile_rows": libsat.last_tile_rows()},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches[0],
+            "clocks": clocks,
+            "parity_recheck": parity,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def run_e2e(args, libsat, x, rows, cols, batch, dtype, world, rank, dev, sharded,
+            total_elems, barrier):
+    """Same metric through the public API with host buffers: H2D of the step's
+    input from pinned memory, the SAT, D2H of the result, all timed."""
+    import torch
+    import torch.distributed as dist
+    steps = max(1, args.e2e_steps)
+    try:
+        hin = torch.empty(x.shape, dtype=x.dtype, pin_memory=True)
+        hout = torch.empty(x.shape, dtype=x.dtype, pin_memory=True)
+    except RuntimeError as e:
+        return {"value": None, "unit": "elem/s", "error": f"pinned alloc failed: {e}"}
+    hin.copy_(x.cpu() if x.numel() * 4 < (1 << 31) else x.to("cpu"))
+    nbytes = x.numel() * x.element_size()
+    if not sharded and batch is None:
+        def step():
+            libsat.sat_host(hin, hout)
+    elif batch is not None:
+        dx = torch.empty_like(x)
+        dy = torch.empty_like(x)
+
+        def step():
+            dx.copy_(hin, non_blocking=True)
+            libsat.sat_batched(dx, out=dy)
+            hout.copy_(dy, non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+    else:
+        from paper_conf_icpp_kasagini14_b200.dist import sharded_sat
+        dx = torch.empty_like(x)
+        dy = torch.empty_like(x)
+
+        def step():
+            dx.copy_(hin, non_blocking=True)
+            sharded_sat(dx, out=dy)
+            hout.copy_(dy, non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+    step()                                           # warm
+    barrier()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    for _ in range(steps):
+        step()
+    ev1.record()
+    barrier()
+    ms = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms = float(ms[0])
+    return {"value": total_elems * steps / (ms / 1e3), "unit": "elem/s",
+            "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "steps": steps,
+            "ms_per_step": ms / steps, "api": "sat_host (pinned)" if (not sharded and batch is None)
+            else "copy + public API + copy"}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,180 @@
+/*
+ * sat.h -- libsat: B200 (sm_100a) summed area tables.  C ABI.
+ *
+ * The operation (Kasagi, Nakano, Ito, "Parallel Algorithms for the Summed Area
+ * Table on the Asynchronous Hierarchical Memory Machine, with GPU
+ * implementations", ICPP 2014; /root/reference/PAPER.md):
+ *
+ *   P:L187-L193 (Sec. I, Fig. 3): for an n x m matrix a the summed area table
+ *   is the n x m matrix b with  b[i][j] = sum_{0<=k<=i, 0<=l<=j} a[k][l]
+ *   (inclusive, 0-indexed), i.e. column-wise prefix-sums followed by row-wise
+ *   prefix-sums.
+ *
+ * Conventions shared by every entry point:
+ *   - Matrices are row-major and contiguous: element (i, j) of image b lives at
+ *     index (b*rows + i)*cols + j.  Input and output have the same dtype.
+ *   - All data pointers are DEVICE pointers owned by the caller (e.g. a torch
+ *     tensor's data_ptr()), except sat_compute_host() which takes host pointers.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     Every call is asynchronous on `stream` unless stated otherwise.
+ *   - SAT_INT32 is computed in uint32 arithmetic, i.e. the result is exact
+ *     modulo 2^32 (two's-complement wrap), bit-identical for every variant,
+ *     tile shape and sharding.  SAT_FLOAT32 uses IEEE fp32 adds (round to
+ *     nearest, no FTZ); its summation order differs between variants and may
+ *     differ between runs (the look-back takes whichever predecessor state it
+ *     finds first); every order stays within the documented 1e-5 max relative
+ *     error for inputs in [0, 1).
+ *   - in == out (exact aliasing) is allowed for every entry point that takes
+ *     both; a partial overlap returns SAT_ERR_INVALID.
+ *   - rows == 0 or cols == 0 (or batch == 0) is a no-op returning SAT_OK.
+ *   - Validation errors are returned synchronously and nothing is launched.
+ *     Faults inside kernels surface as SAT_ERR_CUDA at this or a later call or
+ *     at the caller's next synchronisation.  No C++ exception crosses the ABI.
+ *     sat_last_error() returns a thread-local description of the last error.
+ *   - The library keeps a per-(device, stream) workspace (look-back
+ *     descriptors, a ticket counter, 2R1W carry buffers), grown on demand and
+ *     never memset per call (descriptors carry per-launch tags).  Calls that
+ *     share a stream are serialised by the stream; do not issue calls on two
+ *     threads with the same stream concurrently.
+ */
+#ifndef LIBSAT_SAT_H
+#define LIBSAT_SAT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SAT_ABI_VERSION 1
+
+typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1 } sat_dtype;
+
+/* Variants (Table I / Secs. IV-VII):
+ *   SAT_2R2W        column-wise prefix pass then row-wise prefix pass, each a
+ *                   full read+write of the matrix (Sec. IV, P:L847-L945,
+ *                   Lemma 2).  The paper's row pass is strided; ours is
+ *                   coalesced with the same byte count (R6).
+ *   SAT_2R1W        Step 1 tile reductions (1R), Step 2 carry scans (small),
+ *                   Step 3 re-read + carries + tile SAT (1R+1W) (Sec. V,
+ *                   P:L1059-L1137, Lemma 4).
+ *   SAT_1R1W        the hot path: one read and one write per element (Sec. VI,
+ *                   P:L2151-L2163, Theorem 6), as one launch with a decoupled
+ *                   look-back instead of 2n/w-1 stage launches.
+ *   SAT_1PLUSR_R1W  2R1W on the top-left tile triangle A, 1R1W on the middle
+ *                   band C, 2R1W on the bottom-right triangle B (Sec. VII,
+ *                   P:L2289-L2355, Theorem 7); r from sat_options (0.25 =
+ *                   the paper's 1.25R1W).
+ */
+typedef enum { SAT_2R2W = 0, SAT_2R1W = 1, SAT_1R1W = 2, SAT_1PLUSR_R1W = 3 } sat_variant;
+
+typedef enum {
+    SAT_OK = 0,
+    SAT_ERR_INVALID = -1,      /* bad pointer / size / enum / overlap */
+    SAT_ERR_UNSUPPORTED = -2,  /* valid but not implemented (e.g. seeded batch) */
+    SAT_ERR_NOMEM = -3,        /* workspace allocation failed */
+    SAT_ERR_CUDA = -4,         /* a CUDA runtime/driver call failed */
+    SAT_ERR_COMM = -5          /* the all-gather callback returned nonzero */
+} sat_status;
+
+typedef struct sat_options {
+    double r;            /* SAT_1PLUSR_R1W: target fraction of tiles done by 2R1W
+                            (0..1, default 0.25); the realised value is the tile
+                            count ratio, see sat_last_r_effective() */
+    int tile_rows;       /* band height TH in {16, 32, 64}; 0 = automatic */
+    int force_generic;   /* 1 = use the non-TMA load/store path (tests) */
+    int jitter;          /* debug: random delay (ns) before descriptor
+                            publication, to stress the look-back; 0 = off */
+    int reserved[4];     /* must be 0 */
+} sat_options;
+
+/* Fill *opt with defaults (r = 0.25, automatic tile, TMA when eligible). */
+void sat_options_init(sat_options *opt);
+
+/* out = SAT(in) for one rows x cols matrix.  variant: sat_variant. */
+int sat_compute(const void *in, void *out, int64_t rows, int64_t cols,
+                int dtype, int variant, void *stream);
+
+/* As sat_compute with options (NULL = defaults). */
+int sat_compute_ex(const void *in, void *out, int64_t rows, int64_t cols,
+                   int dtype, int variant, const sat_options *opt, void *stream);
+
+/* `batch` independent rows x cols matrices stored back to back (the
+ * data-parallel image workload, BASELINE.json config 5).  One launch for the
+ * whole batch. */
+int sat_compute_batched(const void *in, void *out, int64_t batch, int64_t rows,
+                        int64_t cols, int dtype, int variant, const sat_options *opt,
+                        void *stream);
+
+/* Seeded 1R1W: the rows x cols matrix is a strip of a taller matrix and
+ * carry_row[j] (device, cols entries, same dtype) is the column sum of
+ * everything above the strip in column j.  Result: the strip's rows of the
+ * full matrix's SAT.  carry_row == NULL is the unseeded case. */
+int sat_compute_seeded(const void *in, void *out, int64_t rows, int64_t cols,
+                       int dtype, const void *carry_row, void *stream);
+
+/* As sat_compute_seeded, but sat_row[j] is the SAT row just above the strip
+ * (the last SAT row of the strip above), not the column sums. */
+int sat_compute_seeded_satrow(const void *in, void *out, int64_t rows, int64_t cols,
+                              int dtype, const void *sat_row, void *stream);
+
+/* totals[j] = sum_i in[i][j] (device, cols entries).  Deterministic order. */
+int sat_column_totals(const void *in, void *totals, int64_t rows, int64_t cols,
+                      int dtype, void *stream);
+
+/* carry_row[j] = sum_{q < rank} gathered[q][j]; gathered is nranks x cols
+ * (device), q ascending. */
+int sat_rank_exscan(const void *gathered, void *carry_row, int64_t nranks,
+                    int64_t cols, int rank, int dtype, void *stream);
+
+/* All-gather callback for the sharded mode: gather `bytes` from every rank's
+ * `send` into `recv` (rank-major, nranks * bytes), enqueued on or completed
+ * before work on `stream`.  Return 0 on success. */
+typedef int (*sat_allgather_fn)(void *ctx, const void *send, void *recv,
+                                size_t bytes, void *stream);
+
+typedef struct sat_shard_stats {
+    int64_t strip_bytes_read;     /* SAT pass: rows*cols*eb */
+    int64_t strip_bytes_written;  /* SAT pass: rows*cols*eb */
+    int64_t extra_bytes_read;     /* column-totals pass (0 on the last rank) */
+    int64_t allgather_bytes;      /* bytes received by this rank */
+} sat_shard_stats;
+
+/* Row-strip sharded SAT (north star (3)): this rank holds strip `rank` of
+ * `nranks` consecutive row strips of one matrix (strips may have different
+ * heights; every rank passes the same cols).  Steps: column totals of the
+ * strip (skipped on the last rank, whose totals nobody needs -- it sends
+ * zeros), all-gather through `allgather`, exclusive scan over ranks, seeded
+ * 1R1W.  `workspace` is a caller-owned device buffer of at least
+ * sat_sharded_workspace_bytes(cols, nranks, dtype) bytes (NULL = library
+ * allocated).  stats may be NULL. */
+int sat_compute_sharded(const void *in_strip, void *out_strip, int64_t strip_rows,
+                        int64_t cols, int dtype, int rank, int nranks,
+                        sat_allgather_fn allgather, void *comm_ctx, void *workspace,
+                        void *stream, sat_shard_stats *stats);
+size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype);
+
+/* End to end from HOST memory: copies in_host (rows*cols elements) to the
+ * device, computes the SAT with `variant`, copies it back to out_host, and
+ * synchronises `stream` before returning.  Pinned host buffers overlap the
+ * copies with compute (the matrix is streamed in row strips, each seeded with
+ * the SAT row above it); pageable buffers work but are slower. */
+int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t cols,
+                     int dtype, int variant, void *stream);
+
+/* Number of kernels launched by the last successful call on this thread. */
+int sat_last_launch_count(void);
+/* Band height used by the last 1R1W-family call on this thread. */
+int sat_last_tile_rows(void);
+/* Realised r of the last SAT_1PLUSR_R1W call on this thread. */
+double sat_last_r_effective(void);
+
+const char *sat_strerror(int status);
+const char *sat_last_error(void);
+int sat_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIBSAT_SAT_H */

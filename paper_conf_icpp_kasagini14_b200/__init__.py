@@ -1,0 +1,267 @@
+"""libsat Python binding: summed area tables on B200 (sm_100a).
+
+Thin ctypes marshalling over the C ABI in ``include/sat.h`` -- every step of
+every variant runs in the CUDA kernels of ``libsat.so``; there is no CPU or
+PyTorch fallback.  If the shared library is missing this module raises on
+import.  Torch is used only for device memory and streams.
+
+The operation: ``b[i][j] = sum_{k<=i, l<=j} a[k][l]``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from ._build import LIB as _LIB_PATH
+
+if not os.path.exists(_LIB_PATH):
+    raise ImportError(
+        f"libsat.so not found at {_LIB_PATH}; run __graft_entry__.build() "
+        "(or python -m paper_conf_icpp_kasagini14_b200._build)")
+
+_lib = ctypes.CDLL(_LIB_PATH)
+
+SAT_INT32, SAT_FLOAT32 = 0, 1
+VARIANTS = {"2r2w": 0, "2r1w": 1, "1r1w": 2, "1+rr1w": 3}
+SAT_OK = 0
+
+
+class SatOptions(ctypes.Structure):
+    _fields_ = [("r", ctypes.c_double), ("tile_rows", ctypes.c_int),
+                ("force_generic", ctypes.c_int), ("jitter", ctypes.c_int),
+                ("reserved", ctypes.c_int * 4)]
+
+
+class SatShardStats(ctypes.Structure):
+    _fields_ = [("strip_bytes_read", ctypes.c_int64), ("strip_bytes_written", ctypes.c_int64),
+                ("extra_bytes_read", ctypes.c_int64), ("allgather_bytes", ctypes.c_int64)]
+
+
+ALLGATHER_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+
+_P, _I64, _I = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+_SIGS = {
+    "sat_options_init": ([ctypes.POINTER(SatOptions)], None),
+    "sat_compute": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
+    "sat_compute_ex": ([_P, _P, _I64, _I64, _I, _I, ctypes.POINTER(SatOptions), _P], _I),
+    "sat_compute_batched": ([_P, _P, _I64, _I64, _I64, _I, _I, ctypes.POINTER(SatOptions), _P], _I),
+    "sat_compute_seeded": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
+    "sat_compute_seeded_satrow": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
+    "sat_column_totals": ([_P, _P, _I64, _I64, _I, _P], _I),
+    "sat_rank_exscan": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
+    "sat_compute_sharded": ([_P, _P, _I64, _I64, _I, _I, _I, ALLGATHER_FN, _P, _P, _P,
+                             ctypes.POINTER(SatShardStats)], _I),
+    "sat_sharded_workspace_bytes": ([_I64, _I, _I], ctypes.c_size_t),
+    "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
+    "sat_last_launch_count": ([], _I),
+    "sat_last_tile_rows": ([], _I),
+    "sat_last_r_effective": ([], ctypes.c_double),
+    "sat_strerror": ([_I], ctypes.c_char_p),
+    "sat_last_error": ([], ctypes.c_char_p),
+    "sat_abi_version": ([], _I),
+}
+for _name, (_args, _res) in _SIGS.items():
+    _f = getattr(_lib, _name)
+    _f.argtypes = _args
+    _f.restype = _res
+
+# every symbol include/sat.h declares (checked by tests/test_abi.py)
+EXPORTED = tuple(_SIGS)
+
+
+class SatError(RuntimeError):
+    pass
+
+
+def _check(status: int):
+    if status != SAT_OK:
+        msg = f"{_lib.sat_strerror(status).decode()}: {_lib.sat_last_error().decode()}"
+        if status == -1:
+            raise ValueError(msg)
+        raise SatError(msg)
+
+
+def _dtype_code(t) -> int:
+    import torch
+    if t.dtype == torch.int32:
+        return SAT_INT32
+    if t.dtype == torch.float32:
+        return SAT_FLOAT32
+    raise TypeError(f"libsat supports int32 and float32, got {t.dtype}")
+
+
+def _stream(stream) -> int:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+def _check_dev(*ts):
+    for t in ts:
+        if t is None:
+            continue
+        if not t.is_cuda:
+            raise ValueError("libsat takes CUDA tensors (use sat_host for host memory)")
+        if not t.is_contiguous():
+            raise ValueError("libsat takes contiguous row-major tensors")
+
+
+def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
+            jitter: int = 0) -> SatOptions:
+    o = SatOptions()
+    _lib.sat_options_init(ctypes.byref(o))
+    o.r = float(r)
+    o.tile_rows = int(tile_rows)
+    o.force_generic = int(bool(force_generic))
+    o.jitter = int(jitter)
+    return o
+
+
+def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
+        force_generic: bool = False, jitter: int = 0, stream=None):
+    """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32 IEEE).
+
+    ``out`` may be ``x`` itself (in place).  ``variant`` in
+    {"1r1w", "2r2w", "2r1w", "1+rr1w"}.
+    """
+    import torch
+    if x.dim() != 2:
+        raise ValueError("sat expects a 2-D tensor (use sat_batched for 3-D)")
+    if out is None:
+        out = torch.empty_like(x)
+    _check_dev(x, out)
+    if out.shape != x.shape or out.dtype != x.dtype:
+        raise ValueError("out must match x in shape and dtype")
+    o = options(r, tile_rows, force_generic, jitter)
+    _check(_lib.sat_compute_ex(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                               _dtype_code(x), VARIANTS[variant], ctypes.byref(o), _stream(stream)))
+    return out
+
+
+def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
+                force_generic: bool = False, stream=None):
+    """SATs of a (batch, rows, cols) CUDA tensor, one launch for the batch."""
+    import torch
+    if x.dim() != 3:
+        raise ValueError("sat_batched expects (batch, rows, cols)")
+    if out is None:
+        out = torch.empty_like(x)
+    _check_dev(x, out)
+    o = options(r, tile_rows, force_generic)
+    _check(_lib.sat_compute_batched(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                                    x.shape[2], _dtype_code(x), VARIANTS[variant],
+                                    ctypes.byref(o), _stream(stream)))
+    return out
+
+
+def sat_seeded(x, carry_row=None, out=None, sat_row=None, stream=None):
+    """Rows of the SAT of a taller matrix: ``carry_row`` = column sums of
+    everything above ``x`` (or ``sat_row`` = the SAT row just above)."""
+    import torch
+    if out is None:
+        out = torch.empty_like(x)
+    _check_dev(x, out, carry_row, sat_row)
+    if sat_row is not None:
+        _check(_lib.sat_compute_seeded_satrow(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                                              _dtype_code(x), sat_row.data_ptr(), _stream(stream)))
+    else:
+        _check(_lib.sat_compute_seeded(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                                       _dtype_code(x),
+                                       carry_row.data_ptr() if carry_row is not None else None,
+                                       _stream(stream)))
+    return out
+
+
+def column_totals(x, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.empty(x.shape[1], dtype=x.dtype, device=x.device)
+    _check_dev(x, out)
+    _check(_lib.sat_column_totals(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                                  _dtype_code(x), _stream(stream)))
+    return out
+
+
+def rank_exscan(gathered, rank: int, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.empty(gathered.shape[1], dtype=gathered.dtype, device=gathered.device)
+    _check_dev(gathered, out)
+    _check(_lib.sat_rank_exscan(gathered.data_ptr(), out.data_ptr(), gathered.shape[0],
+                                gathered.shape[1], int(rank), _dtype_code(gathered),
+                                _stream(stream)))
+    return out
+
+
+def sat_host(x_host, out_host=None, variant: str = "1r1w", stream=None):
+    """End to end from host memory (pinned tensors overlap copies and compute)."""
+    import torch
+    if x_host.is_cuda:
+        raise ValueError("sat_host takes CPU tensors")
+    if not x_host.is_contiguous():
+        raise ValueError("sat_host takes contiguous tensors")
+    if out_host is None:
+        out_host = torch.empty_like(x_host, pin_memory=x_host.is_pinned())
+    _check(_lib.sat_compute_host(x_host.data_ptr(), out_host.data_ptr(), x_host.shape[0],
+                                 x_host.shape[1], _dtype_code(x_host), VARIANTS[variant],
+                                 _stream(stream)))
+    return out_host
+
+
+def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=None):
+    """Row-strip sharded SAT through the single C-ABI call.
+
+    ``allgather(send, recv)`` receives torch views of the library's send
+    (cols) and receive (nranks x cols) buffers and must fill ``recv``.
+    Returns (out, stats dict).
+    """
+    import torch
+    if out is None:
+        out = torch.empty_like(strip)
+    _check_dev(strip, out)
+    cols = strip.shape[1]
+    nbytes = _lib.sat_sharded_workspace_bytes(cols, nranks, _dtype_code(strip))
+    ws = torch.empty(max(nbytes, 1), dtype=torch.uint8, device=strip.device)
+    row = ((cols * 4) + 255) // 256 * 256
+    send = ws[:cols * 4].view(strip.dtype)
+    recv = ws[2 * row:2 * row + nranks * cols * 4].view(strip.dtype).view(nranks, cols)
+    err = []
+
+    def cb(ctx, send_p, recv_p, nb, st):
+        try:
+            assert send_p == send.data_ptr() and recv_p == recv.data_ptr() and nb == cols * 4
+            allgather(send, recv)
+            return 0
+        except Exception as e:  # reported through SAT_ERR_COMM
+            err.append(e)
+            return 1
+    cfun = ALLGATHER_FN(cb)
+    stats = SatShardStats()
+    st = _lib.sat_compute_sharded(strip.data_ptr(), out.data_ptr(), strip.shape[0], cols,
+                                  _dtype_code(strip), int(rank), int(nranks), cfun, None,
+                                  ws.data_ptr(), _stream(stream), ctypes.byref(stats))
+    if err:
+        raise err[0]
+    _check(st)
+    return out, {f: getattr(stats, f) for f, _ in SatShardStats._fields_}
+
+
+def last_launch_count() -> int:
+    return _lib.sat_last_launch_count()
+
+
+def last_tile_rows() -> int:
+    return _lib.sat_last_tile_rows()
+
+
+def last_r_effective() -> float:
+    return _lib.sat_last_r_effective()
+
+
+def abi_version() -> int:
+    return _lib.sat_abi_version()
+
+
+lib = _lib

@@ -1,0 +1,762 @@
+// sat_api.cu -- the libsat C ABI (include/sat.h): validation, per-stream
+// workspace, tensor maps, variant drivers and kernel dispatch.
+//
+// Variant drivers follow PAPER.md: 2R2W Sec. IV, 2R1W Sec. V
+// (P:L1059-L1137), 1R1W Sec. VI, (1+r)R1W Sec. VII
+// (P:L2289-L2355).  The sharded and host (end-to-end) entry points are the
+// north star's (1)/(3) additions (BASELINE.json).
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+
+#include "../../include/sat.h"
+#include "sat_aux.cuh"
+#include "sat_band.cuh"
+
+using namespace sat;
+
+namespace {
+
+thread_local std::string t_err;
+thread_local int t_launches = 0;
+thread_local int t_th = 0;
+thread_local double t_r = 0.0;
+
+int fail(int code, const std::string& msg) {
+    t_err = msg;
+    return code;
+}
+
+#define CUDA_TRY(expr)                                                                  \
+    do {                                                                                \
+        cudaError_t _e = (expr);                                                        \
+        if (_e != cudaSuccess)                                                          \
+            return fail(SAT_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(_e)); \
+    } while (0)
+
+#define SAT_TRY(expr)                  \
+    do {                               \
+        int _s = (expr);               \
+        if (_s != SAT_OK) return _s;   \
+    } while (0)
+
+// ------------------------------------------------------------------ devices
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+struct DevInfo {
+    int sms = 0;
+    int smem_optin = 0;
+    bool ok = false;
+};
+
+std::mutex g_mu;
+std::map<int, DevInfo> g_dev;
+EncodeTiledFn g_encode = nullptr;
+
+int get_dev(int& dev, DevInfo& info) {
+    CUDA_TRY(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    DevInfo& d = g_dev[dev];
+    if (!d.ok) {
+        CUDA_TRY(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
+        CUDA_TRY(cudaDeviceGetAttribute(&d.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+        d.ok = true;
+    }
+    if (!g_encode) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        CUDA_TRY(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+        if (q != cudaDriverEntryPointSuccess || !fn)
+            return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled entry point not found");
+        g_encode = reinterpret_cast<EncodeTiledFn>(fn);
+    }
+    info = d;
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ workspace
+struct Buf {
+    void* p = nullptr;
+    size_t bytes = 0;
+};
+
+int ensure(Buf& b, size_t bytes, bool zero) {
+    if (b.bytes >= bytes && b.p) return SAT_OK;
+    if (b.p) { cudaFree(b.p); b.p = nullptr; b.bytes = 0; }
+    size_t want = std::max<size_t>(bytes, 256);
+    if (cudaMalloc(&b.p, want) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(SAT_ERR_NOMEM, "cudaMalloc of " + std::to_string(want) + " bytes failed");
+    }
+    b.bytes = want;
+    if (zero) CUDA_TRY(cudaMemset(b.p, 0, want));
+    return SAT_OK;
+}
+
+constexpr unsigned long long kTagSpace = 1ull << 30;
+
+struct Workspace {
+    Buf desc;                 // look-back descriptors (zeroed when (re)allocated)
+    Buf ticket;               // unsigned long long counter
+    unsigned long long next_base = 0;
+    Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
+    Buf part;                 // column totals partials
+    Buf shard;                // sharded default workspace
+    Buf din, dout;            // host e2e device copies
+    cudaStream_t cstream_in = nullptr, cstream_out = nullptr;
+};
+
+std::map<std::pair<int, void*>, Workspace*> g_ws;
+
+int get_ws(int dev, cudaStream_t st, Workspace*& ws) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    Workspace*& w = g_ws[{dev, reinterpret_cast<void*>(st)}];
+    if (!w) w = new Workspace();
+    ws = w;
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ helpers
+
+int validate(const void* in, const void* out, int64_t batch, int64_t rows, int64_t cols,
+             int dtype, bool need_in = true) {
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32)
+        return fail(SAT_ERR_INVALID, "dtype must be SAT_INT32 or SAT_FLOAT32");
+    if (rows < 0 || cols < 0 || batch < 0) return fail(SAT_ERR_INVALID, "negative size");
+    if (rows > INT32_MAX || cols > INT32_MAX || batch > INT32_MAX)
+        return fail(SAT_ERR_INVALID, "rows, cols and batch must each be < 2^31");
+    if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
+    const double n = double(rows) * double(cols) * double(batch);
+    if (n * 4.0 > 9.0e18) return fail(SAT_ERR_INVALID, "matrix byte size overflows");
+    if ((need_in && !in) || !out) return fail(SAT_ERR_INVALID, "null pointer with nonzero size");
+    if (need_in && in != out) {
+        const uintptr_t a0 = reinterpret_cast<uintptr_t>(in), b0 = reinterpret_cast<uintptr_t>(out);
+        const uintptr_t len = uintptr_t(rows) * uintptr_t(cols) * uintptr_t(batch) * 4u;
+        if (a0 < b0 + len && b0 < a0 + len)
+            return fail(SAT_ERR_INVALID, "in and out partially overlap");
+    }
+    if ((reinterpret_cast<uintptr_t>(out) & 3) || (need_in && (reinterpret_cast<uintptr_t>(in) & 3)))
+        return fail(SAT_ERR_INVALID, "pointers must be 4-byte aligned");
+    return SAT_OK;
+}
+
+bool tma_ok(const void* in, const void* out, int64_t cols) {
+    return (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) &&
+           ((reinterpret_cast<uintptr_t>(out) & 15) == 0);
+}
+
+int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_t rows,
+              int64_t cols, int th) {
+    cuuint64_t dims[3] = {cuuint64_t(cols), cuuint64_t(rows), cuuint64_t(batch)};
+    cuuint64_t strides[2] = {cuuint64_t(cols) * 4, cuuint64_t(cols) * cuuint64_t(rows) * 4};
+    cuuint32_t box[3] = {cuuint32_t(TW), cuuint32_t(th), 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    CUresult r = g_encode(m, dtype == SAT_INT32 ? CU_TENSOR_MAP_DATA_TYPE_UINT32
+                                                : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+                          3, const_cast<void*>(base), dims, strides, box, es,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS)
+        return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string(int(r)) + ")");
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ band kernel dispatch
+struct BandCfg {
+    int R, W, S, MINB;
+};
+// TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
+// S*W*512 (warp bottom rows) + S*512 (SAT row above) + barriers.
+constexpr BandCfg kCfg16{2, 8, 4, 4};
+constexpr BandCfg kCfg32{4, 8, 4, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 2};
+
+template <typename T, int R, int W, int S, int MODE, bool TMA, int MINB>
+int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
+                  const DevInfo& di, cudaStream_t st, int& grid_out) {
+    auto kern = sat_band_kernel<T, R, W, S, MODE, TMA, MINB>;
+    const size_t smem = BandSmem<T, R, W, S>::total;
+    const int threads = (W + 2) * 32;
+    static int configured = 0;   // per instantiation (per process; devices share the attribute)
+    if (!configured) {
+        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+        configured = 1;
+    }
+    int occ = 0;
+    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, smem));
+    if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
+    long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
+    if (grid < 1) grid = 1;
+    grid_out = int(grid);
+    kern<<<int(grid), threads, smem, st>>>(ti, to, p);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    return SAT_OK;
+}
+
+template <typename T, int MODE, bool TMA>
+int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
+                   const DevInfo& di, cudaStream_t st, int& grid) {
+    switch (th) {
+        case 16: return launch_band_t<T, kCfg16.R, kCfg16.W, kCfg16.S, MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
+        case 32: return launch_band_t<T, kCfg32.R, kCfg32.W, kCfg32.S, MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
+        case 64: return launch_band_t<T, kCfg64.R, kCfg64.W, kCfg64.S, MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
+    }
+    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32 or 64");
+}
+
+template <typename T, int MODE>
+int launch_band_m(bool tma, int th, const BandParams& p, const CUtensorMap& ti,
+                  const CUtensorMap& to, const DevInfo& di, cudaStream_t st, int& grid) {
+    return tma ? launch_band_th<T, MODE, true>(th, p, ti, to, di, st, grid)
+               : launch_band_th<T, MODE, false>(th, p, ti, to, di, st, grid);
+}
+
+template <typename T>
+int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtensorMap& ti,
+                  const CUtensorMap& to, const DevInfo& di, cudaStream_t st, int& grid) {
+    switch (mode) {
+        case MODE_SAT: return launch_band_m<T, MODE_SAT>(tma, th, p, ti, to, di, st, grid);
+        case MODE_COL: return launch_band_m<T, MODE_COL>(tma, th, p, ti, to, di, st, grid);
+        case MODE_ROW: return launch_band_m<T, MODE_ROW>(tma, th, p, ti, to, di, st, grid);
+    }
+    return fail(SAT_ERR_INVALID, "bad mode");
+}
+
+// Automatic band height: the tallest band that still gives roughly one band
+// per resident CTA slot (the look-back chain is per band; more, shorter bands
+// raise parallelism, taller bands cut descriptor traffic).
+int auto_th(int64_t rows, int64_t batch, const DevInfo& di) {
+    const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
+    for (int th : {64, 32}) {
+        const long long bands = batch * ((rows + th - 1) / th);
+        if (bands * 5 >= slots * 4) return th;
+    }
+    return 16;
+}
+
+struct Job {
+    const void* in;
+    void* out;
+    int64_t batch, rows, cols;
+    int dtype;
+    int th;
+    bool tma;
+    int jitter;
+    const DevInfo* di;
+    Workspace* ws;
+    cudaStream_t st;
+};
+
+// One band-kernel launch with ticket/tag bookkeeping.
+int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
+    p.in = in;
+    p.out = out;
+    p.rows = j.rows;
+    p.cols = j.cols;
+    p.batch = int(j.batch);
+    p.nb = int((j.rows + j.th - 1) / j.th);
+    p.nc = int((j.cols + TW - 1) / TW);
+    p.total_bands = int(j.batch * p.nb);
+    p.total_units = p.tile_units ? (long long)p.total_bands * p.nc : p.total_bands;
+    p.jitter = j.jitter;
+    Workspace& ws = *j.ws;
+    if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
+        const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t);
+        SAT_TRY(ensure(ws.desc, need, true));
+    }
+    SAT_TRY(ensure(ws.ticket, sizeof(unsigned long long), true));
+    const unsigned long long units = (unsigned long long)p.total_units;
+    const unsigned long long worst = units + 4096ull * 64ull;   // units + max grid
+    if (ws.next_base + worst >= kTagSpace) {
+        // tag space exhausted: clear descriptors and the counter (rare)
+        if (ws.desc.p) CUDA_TRY(cudaMemsetAsync(ws.desc.p, 0, ws.desc.bytes, j.st));
+        CUDA_TRY(cudaMemsetAsync(ws.ticket.p, 0, sizeof(unsigned long long), j.st));
+        ws.next_base = 0;
+    }
+    p.desc = static_cast<uint64_t*>(ws.desc.p);
+    p.ticket = static_cast<unsigned long long*>(ws.ticket.p);
+    p.base = ws.next_base;
+    CUtensorMap ti, to;
+    std::memset(&ti, 0, sizeof(ti));
+    std::memset(&to, 0, sizeof(to));
+    if (j.tma) {
+        SAT_TRY(make_tmap(&ti, in, j.dtype, j.batch, j.rows, j.cols, j.th));
+        SAT_TRY(make_tmap(&to, out, j.dtype, j.batch, j.rows, j.cols, j.th));
+    }
+    int grid = 0;
+    int s = (j.dtype == SAT_INT32)
+                ? launch_band_d<uint32_t>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid)
+                : launch_band_d<float>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid);
+    if (s != SAT_OK) return s;
+    ws.next_base += units + (unsigned long long)grid;
+    return SAT_OK;
+}
+
+BandParams base_params() {
+    BandParams p;
+    std::memset(&p, 0, sizeof(p));
+    p.top_src = TOP_LOOKBACK;
+    p.region = REG_ALL;
+    p.seed_kind = SEED_NONE;
+    return p;
+}
+
+// ------------------------------------------------------------------ 2R1W family
+struct Carry2r1w {
+    int nb, nc, total_bands;
+};
+
+int prep_2r1w(const Job& j, Carry2r1w& c) {
+    c.nb = int((j.rows + j.th - 1) / j.th);
+    c.nc = int((j.cols + TW - 1) / TW);
+    c.total_bands = int(j.batch * c.nb);
+    Workspace& ws = *j.ws;
+    const size_t eb = 4;
+    const size_t wide = size_t(c.total_bands) * c.nc * TW * eb;
+    const size_t rowsp = size_t(c.total_bands) * j.th * eb;
+    SAT_TRY(ensure(ws.bt, wide, false));
+    SAT_TRY(ensure(ws.topx, wide, false));
+    SAT_TRY(ensure(ws.rs, rowsp * c.nc, false));
+    SAT_TRY(ensure(ws.lx, rowsp * (c.nc + 1), false));
+    SAT_TRY(ensure(ws.lsum, size_t(c.total_bands) * (c.nc + 1) * eb, false));
+    SAT_TRY(ensure(ws.lb, rowsp, false));
+    return SAT_OK;
+}
+
+template <typename T>
+int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, const void* in,
+                      void* out, const void* Lb) {
+    Workspace& ws = *j.ws;
+    TileParams tp;
+    tp.in = in; tp.rows = j.rows; tp.cols = j.cols; tp.batch = int(j.batch);
+    tp.nb = c.nb; tp.nc = c.nc; tp.total_bands = c.total_bands; tp.th = j.th;
+    tp.region = region; tp.tA = tA; tp.Bt = ws.bt.p; tp.RS = ws.rs.p;
+    // Step 1: tile reductions
+    sat_reduce_kernel<T><<<dim3(c.nc, c.total_bands), 256, 0, j.st>>>(tp);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    // Step 2: row carries, then SAT row above every tile
+    CarryParams cp;
+    cp.rows = j.rows; cp.cols = j.cols; cp.batch = int(j.batch); cp.nb = c.nb; cp.nc = c.nc;
+    cp.total_bands = c.total_bands; cp.th = j.th; cp.region = region; cp.tA = tA;
+    cp.RS = ws.rs.p; cp.Bt = ws.bt.p; cp.Lb = Lb; cp.Lx = ws.lx.p; cp.Lsum = ws.lsum.p;
+    cp.TopX = ws.topx.p; cp.out = out;
+    const int rthreads = ((j.th + 31) / 32) * 32;
+    sat_carry_rows_kernel<T><<<c.total_bands, rthreads, 0, j.st>>>(cp);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    const int W = c.nc * TW;
+    sat_carry_top_kernel<T><<<dim3((W + 255) / 256, unsigned(j.batch)), 256, 0, j.st>>>(cp);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    // Step 3: re-read, add carries, tile SAT, write (tile tickets, external carries)
+    BandParams p = base_params();
+    p.top_src = TOP_EXTERNAL;
+    p.tile_units = 1;
+    p.region = region;
+    p.tA = tA;
+    p.Lx = ws.lx.p;
+    p.TopX = ws.topx.p;
+    return run_band(j, MODE_SAT, in, out, p);
+}
+
+int run_2r1w_region(const Job& j, const Carry2r1w& c, int region, int tA, const void* in,
+                    void* out, const void* Lb) {
+    return j.dtype == SAT_INT32 ? run_2r1w_region_t<uint32_t>(j, c, region, tA, in, out, Lb)
+                                : run_2r1w_region_t<float>(j, c, region, tA, in, out, Lb);
+}
+
+// Choose the triangle threshold tA whose tile fraction (|A|+|B|)/(nb*nc) is
+// closest to r (reading R10), keeping A and B disjoint.
+int choose_tA(int nb, int nc, double r, double& r_eff) {
+    const int last = nb + nc - 2;
+    const int tmax = (last + 1) / 2;
+    int best = 0;
+    double bestd = 1e30;
+    r_eff = 0;
+    for (int tA = 0; tA <= tmax; ++tA) {
+        long long cnt = 0;
+        for (int I = 0; I < nb; ++I) {
+            int a0, a1, b0, b1;
+            region_range(REG_A, tA, nb, nc, I, a0, a1);
+            region_range(REG_B, tA, nb, nc, I, b0, b1);
+            cnt += (a1 - a0) + (b1 - b0);
+        }
+        const double re = double(cnt) / (double(nb) * nc);
+        if (std::fabs(re - r) < bestd) { bestd = std::fabs(re - r); best = tA; r_eff = re; }
+    }
+    return best;
+}
+
+// ------------------------------------------------------------------ core driver
+int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
+                 int dtype, int variant, const sat_options* opt, const void* seed,
+                 int seed_kind, cudaStream_t st) {
+    t_launches = 0;
+    SAT_TRY(validate(in, out, batch, rows, cols, dtype));
+    if (variant < SAT_2R2W || variant > SAT_1PLUSR_R1W) return fail(SAT_ERR_INVALID, "bad variant");
+    sat_options o;
+    sat_options_init(&o);
+    if (opt) o = *opt;
+    if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 64)
+        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32 or 64");
+    if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
+    if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    Workspace* ws;
+    SAT_TRY(get_ws(dev, st, ws));
+    Job j;
+    j.in = in; j.out = out; j.batch = batch; j.rows = rows; j.cols = cols; j.dtype = dtype;
+    j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di);
+    j.tma = !o.force_generic && tma_ok(in, out, cols);
+    j.jitter = o.jitter;
+    j.di = &di;
+    j.ws = ws;
+    j.st = st;
+    t_th = j.th;
+    switch (variant) {
+        case SAT_1R1W: {
+            BandParams p = base_params();
+            p.seed = seed;
+            p.seed_kind = seed ? seed_kind : SEED_NONE;
+            return run_band(j, MODE_SAT, in, out, p);
+        }
+        case SAT_2R2W: {
+            // column-wise prefix-sums (look-back down the columns), then
+            // row-wise prefix-sums (rows independent)
+            BandParams p = base_params();
+            SAT_TRY(run_band(j, MODE_COL, in, out, p));
+            Job j2 = j;
+            j2.tma = !o.force_generic && tma_ok(out, out, cols);
+            return run_band(j2, MODE_ROW, out, out, base_params());
+        }
+        case SAT_2R1W: {
+            Carry2r1w c;
+            SAT_TRY(prep_2r1w(j, c));
+            return run_2r1w_region(j, c, REG_ALL, 0, in, out, nullptr);
+        }
+        case SAT_1PLUSR_R1W: {
+            Carry2r1w c;
+            SAT_TRY(prep_2r1w(j, c));
+            double r_eff = 0;
+            const int tA = choose_tA(c.nb, c.nc, o.r, r_eff);
+            t_r = r_eff;
+            // (A) 2R1W on the top-left triangle; its Step 2 also leaves the
+            // row carry into (C) in Lx.
+            SAT_TRY(run_2r1w_region(j, c, REG_A, tA, in, out, nullptr));
+            // (C) 1R1W over the middle band, seeded from (A)'s final SAT rows
+            // and row carries; leaves the row carry into (B) in Lb.
+            BandParams p = base_params();
+            p.region = REG_C;
+            p.tA = tA;
+            p.Lx = ws->lx.p;
+            p.Lb = ws->lb.p;
+            SAT_TRY(run_band(j, MODE_SAT, in, out, p));
+            // (B) 2R1W on the bottom-right triangle, seeded from (C).
+            return run_2r1w_region(j, c, REG_B, tA, in, out, ws->lb.p);
+        }
+    }
+    return fail(SAT_ERR_INVALID, "bad variant");
+}
+
+template <typename T>
+int column_totals_t(const void* in, void* totals, int64_t rows, int64_t cols, const DevInfo& di,
+                    Workspace& ws, cudaStream_t st) {
+    const int nc = int((cols + TW - 1) / TW);
+    long long splits = std::max<long long>(1, (4LL * di.sms + nc - 1) / nc);
+    splits = std::min<long long>(splits, (rows + 63) / 64);
+    if (splits < 1) splits = 1;
+    const int64_t seg = (rows + splits - 1) / splits;
+    splits = (rows + seg - 1) / seg;
+    SAT_TRY(ensure(ws.part, size_t(splits) * nc * TW * sizeof(T), false));
+    sat_colsum_partial_kernel<T><<<dim3(nc, unsigned(splits)), 256, 0, st>>>(
+        static_cast<const T*>(in), static_cast<T*>(ws.part.p), rows, cols, seg);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    sat_colsum_final_kernel<T><<<unsigned((cols + 255) / 256), 256, 0, st>>>(
+        static_cast<const T*>(ws.part.p), static_cast<T*>(totals), cols, int(splits), nc * TW);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    return SAT_OK;
+}
+
+int column_totals_core(const void* in, void* totals, int64_t rows, int64_t cols, int dtype,
+                       cudaStream_t st) {
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    Workspace* ws;
+    SAT_TRY(get_ws(dev, st, ws));
+    return dtype == SAT_INT32 ? column_totals_t<uint32_t>(in, totals, rows, cols, di, *ws, st)
+                              : column_totals_t<float>(in, totals, rows, cols, di, *ws, st);
+}
+
+int exscan_core(const void* gathered, void* carry, int64_t nranks, int64_t cols, int rank,
+                int dtype, cudaStream_t st) {
+    const unsigned blocks = unsigned((cols + 255) / 256);
+    if (dtype == SAT_INT32)
+        sat_rank_exscan_kernel<uint32_t><<<blocks, 256, 0, st>>>(
+            static_cast<const uint32_t*>(gathered), static_cast<uint32_t*>(carry), cols, rank);
+    else
+        sat_rank_exscan_kernel<float><<<blocks, 256, 0, st>>>(
+            static_cast<const float*>(gathered), static_cast<float*>(carry), cols, rank);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    return SAT_OK;
+}
+
+size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+void sat_options_init(sat_options* opt) {
+    if (!opt) return;
+    std::memset(opt, 0, sizeof(*opt));
+    opt->r = 0.25;
+}
+
+int sat_compute(const void* in, void* out, int64_t rows, int64_t cols, int dtype, int variant,
+                void* stream) {
+    return compute_core(in, out, 1, rows, cols, dtype, variant, nullptr, nullptr, SEED_NONE,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int sat_compute_ex(const void* in, void* out, int64_t rows, int64_t cols, int dtype, int variant,
+                   const sat_options* opt, void* stream) {
+    return compute_core(in, out, 1, rows, cols, dtype, variant, opt, nullptr, SEED_NONE,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int sat_compute_batched(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
+                        int dtype, int variant, const sat_options* opt, void* stream) {
+    return compute_core(in, out, batch, rows, cols, dtype, variant, opt, nullptr, SEED_NONE,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int sat_compute_seeded(const void* in, void* out, int64_t rows, int64_t cols, int dtype,
+                       const void* carry_row, void* stream) {
+    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, carry_row, SEED_COLSUM,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int sat_compute_seeded_satrow(const void* in, void* out, int64_t rows, int64_t cols, int dtype,
+                              const void* sat_row, void* stream) {
+    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, sat_row, SEED_SATROW,
+                        static_cast<cudaStream_t>(stream));
+}
+
+int sat_column_totals(const void* in, void* totals, int64_t rows, int64_t cols, int dtype,
+                      void* stream) {
+    t_launches = 0;
+    SAT_TRY(validate(in, totals, 1, rows, cols, dtype, true));
+    if (rows == 0 || cols == 0) {
+        if (cols > 0 && totals)
+            CUDA_TRY(cudaMemsetAsync(totals, 0, size_t(cols) * 4, static_cast<cudaStream_t>(stream)));
+        return SAT_OK;
+    }
+    return column_totals_core(in, totals, rows, cols, dtype, static_cast<cudaStream_t>(stream));
+}
+
+int sat_rank_exscan(const void* gathered, void* carry_row, int64_t nranks, int64_t cols, int rank,
+                    int dtype, void* stream) {
+    t_launches = 0;
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (nranks < 1 || rank < 0 || rank >= nranks || cols < 0)
+        return fail(SAT_ERR_INVALID, "bad rank / nranks / cols");
+    if (cols == 0) return SAT_OK;
+    if (!carry_row || (rank > 0 && !gathered)) return fail(SAT_ERR_INVALID, "null pointer");
+    return exscan_core(gathered, carry_row, nranks, cols, rank, dtype,
+                       static_cast<cudaStream_t>(stream));
+}
+
+size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype) {
+    (void)dtype;
+    if (cols <= 0 || nranks <= 0) return 0;
+    const size_t row = align256(size_t(cols) * 4);
+    return row * size_t(nranks + 2);
+}
+
+int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_rows, int64_t cols,
+                        int dtype, int rank, int nranks, sat_allgather_fn allgather,
+                        void* comm_ctx, void* workspace, void* stream, sat_shard_stats* stats) {
+    t_launches = 0;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAT_ERR_INVALID, "bad rank / nranks");
+    SAT_TRY(validate(in_strip, out_strip, 1, strip_rows, cols, dtype));
+    if (nranks > 1 && !allgather) return fail(SAT_ERR_INVALID, "allgather callback required");
+    if (stats) std::memset(stats, 0, sizeof(*stats));
+    if (cols == 0) return SAT_OK;
+    const size_t row = align256(size_t(cols) * 4);
+    uint8_t* wsp = static_cast<uint8_t*>(workspace);
+    if (!wsp) {
+        int dev;
+        DevInfo di;
+        SAT_TRY(get_dev(dev, di));
+        Workspace* ws;
+        SAT_TRY(get_ws(dev, st, ws));
+        SAT_TRY(ensure(ws->shard, sat_sharded_workspace_bytes(cols, nranks, dtype), false));
+        wsp = static_cast<uint8_t*>(ws->shard.p);
+    }
+    void* send = wsp;
+    void* carry = wsp + row;
+    void* recv = wsp + 2 * row;
+    int launches = 0;
+    const void* seed = nullptr;
+    if (nranks > 1) {
+        // 1. column totals of the strip (the extra read); the last rank's
+        //    totals are never consumed, so it sends zeros instead
+        if (rank < nranks - 1 && strip_rows > 0) {
+            SAT_TRY(column_totals_core(in_strip, send, strip_rows, cols, dtype, st));
+            launches += t_launches;
+        } else {
+            CUDA_TRY(cudaMemsetAsync(send, 0, size_t(cols) * 4, st));
+        }
+        // 2. all-gather of the m-vectors (NCCL over NVLink in the Python binding)
+        if (allgather(comm_ctx, send, recv, size_t(cols) * 4, stream) != 0)
+            return fail(SAT_ERR_COMM, "allgather callback failed");
+        // 3. exclusive scan over ranks
+        if (rank > 0) {
+            t_launches = 0;
+            SAT_TRY(exscan_core(recv, carry, nranks, cols, rank, dtype, st));
+            launches += t_launches;
+            seed = carry;
+        }
+    }
+    // 4. seeded local 1R1W
+    if (strip_rows > 0) {
+        SAT_TRY(compute_core(in_strip, out_strip, 1, strip_rows, cols, dtype, SAT_1R1W, nullptr,
+                             seed, SEED_COLSUM, st));
+        launches += t_launches;
+    }
+    t_launches = launches;
+    if (stats) {
+        const int64_t b = strip_rows * cols * 4;
+        stats->strip_bytes_read = b;
+        stats->strip_bytes_written = b;
+        stats->extra_bytes_read = (nranks > 1 && rank < nranks - 1) ? b : 0;
+        stats->allgather_bytes = nranks > 1 ? int64_t(nranks) * cols * 4 : 0;
+    }
+    return SAT_OK;
+}
+
+int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t cols, int dtype,
+                     int variant, void* stream) {
+    t_launches = 0;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (rows < 0 || cols < 0) return fail(SAT_ERR_INVALID, "negative size");
+    if (rows == 0 || cols == 0) return SAT_OK;
+    if (!in_host || !out_host) return fail(SAT_ERR_INVALID, "null pointer");
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    Workspace* ws;
+    SAT_TRY(get_ws(dev, st, ws));
+    const size_t bytes = size_t(rows) * size_t(cols) * 4;
+    SAT_TRY(ensure(ws->din, bytes, false));
+    SAT_TRY(ensure(ws->dout, bytes, false));
+    cudaPointerAttributes ai, ao;
+    bool pinned = cudaPointerGetAttributes(&ai, in_host) == cudaSuccess &&
+                  cudaPointerGetAttributes(&ao, out_host) == cudaSuccess &&
+                  ai.type == cudaMemoryTypeHost && ao.type == cudaMemoryTypeHost;
+    cudaGetLastError();
+    int launches = 0;
+    if (!pinned || variant != SAT_1R1W || rows < 512) {
+        CUDA_TRY(cudaMemcpyAsync(ws->din.p, in_host, bytes, cudaMemcpyHostToDevice, st));
+        SAT_TRY(compute_core(ws->din.p, ws->dout.p, 1, rows, cols, dtype, variant, nullptr,
+                             nullptr, SEED_NONE, st));
+        launches = t_launches;
+        CUDA_TRY(cudaMemcpyAsync(out_host, ws->dout.p, bytes, cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(cudaStreamSynchronize(st));
+        t_launches = launches;
+        return SAT_OK;
+    }
+    // Pinned 1R1W: stream row strips; strip k is seeded with the last SAT row
+    // of strip k-1, so H2D of strip k+1 and D2H of strip k-1 overlap the SAT
+    // of strip k.
+    if (!ws->cstream_in) {
+        CUDA_TRY(cudaStreamCreateWithFlags(&ws->cstream_in, cudaStreamNonBlocking));
+        CUDA_TRY(cudaStreamCreateWithFlags(&ws->cstream_out, cudaStreamNonBlocking));
+    }
+    const int nstrips = int(std::min<int64_t>(8, rows / 256));
+    const int64_t srows = (rows + nstrips - 1) / nstrips;
+    cudaEvent_t ev_start, ev_in[8], ev_done[8];
+    CUDA_TRY(cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming));
+    for (int k = 0; k < nstrips; ++k) {
+        CUDA_TRY(cudaEventCreateWithFlags(&ev_in[k], cudaEventDisableTiming));
+        CUDA_TRY(cudaEventCreateWithFlags(&ev_done[k], cudaEventDisableTiming));
+    }
+    CUDA_TRY(cudaEventRecord(ev_start, st));
+    CUDA_TRY(cudaStreamWaitEvent(ws->cstream_in, ev_start, 0));
+    const uint8_t* hin = static_cast<const uint8_t*>(in_host);
+    uint8_t* hout = static_cast<uint8_t*>(out_host);
+    uint8_t* din = static_cast<uint8_t*>(ws->din.p);
+    uint8_t* dout = static_cast<uint8_t*>(ws->dout.p);
+    const size_t rowb = size_t(cols) * 4;
+    for (int k = 0; k < nstrips; ++k) {
+        const int64_t r0 = k * srows, r1 = std::min<int64_t>(rows, r0 + srows);
+        if (r1 <= r0) { CUDA_TRY(cudaEventRecord(ev_in[k], ws->cstream_in)); continue; }
+        CUDA_TRY(cudaMemcpyAsync(din + r0 * rowb, hin + r0 * rowb, (r1 - r0) * rowb,
+                                 cudaMemcpyHostToDevice, ws->cstream_in));
+        CUDA_TRY(cudaEventRecord(ev_in[k], ws->cstream_in));
+    }
+    for (int k = 0; k < nstrips; ++k) {
+        const int64_t r0 = k * srows, r1 = std::min<int64_t>(rows, r0 + srows);
+        CUDA_TRY(cudaStreamWaitEvent(st, ev_in[k], 0));
+        if (r1 > r0) {
+            SAT_TRY(compute_core(din + r0 * rowb, dout + r0 * rowb, 1, r1 - r0, cols, dtype,
+                                 SAT_1R1W, nullptr, k > 0 ? dout + (r0 - 1) * rowb : nullptr,
+                                 SEED_SATROW, st));
+            launches += t_launches;
+        }
+        CUDA_TRY(cudaEventRecord(ev_done[k], st));
+        CUDA_TRY(cudaStreamWaitEvent(ws->cstream_out, ev_done[k], 0));
+        if (r1 > r0)
+            CUDA_TRY(cudaMemcpyAsync(hout + r0 * rowb, dout + r0 * rowb, (r1 - r0) * rowb,
+                                     cudaMemcpyDeviceToHost, ws->cstream_out));
+    }
+    CUDA_TRY(cudaStreamSynchronize(ws->cstream_out));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    cudaEventDestroy(ev_start);
+    for (int k = 0; k < nstrips; ++k) { cudaEventDestroy(ev_in[k]); cudaEventDestroy(ev_done[k]); }
+    t_launches = launches;
+    return SAT_OK;
+}
+
+int sat_last_launch_count(void) { return t_launches; }
+int sat_last_tile_rows(void) { return t_th; }
+double sat_last_r_effective(void) { return t_r; }
+
+const char* sat_strerror(int status) {
+    switch (status) {
+        case SAT_OK: return "ok";
+        case SAT_ERR_INVALID: return "invalid argument";
+        case SAT_ERR_UNSUPPORTED: return "unsupported";
+        case SAT_ERR_NOMEM: return "out of device memory";
+        case SAT_ERR_CUDA: return "CUDA error";
+        case SAT_ERR_COMM: return "communication error";
+    }
+    return "unknown status";
+}
+
+const char* sat_last_error(void) { return t_err.c_str(); }
+int sat_abi_version(void) { return SAT_ABI_VERSION; }
+
+}  // extern "C"

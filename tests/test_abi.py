@@ -1,0 +1,74 @@
+"""The C-ABI library loads and exports every symbol include/sat.h declares;
+host-side validation works without a GPU (no compute calls here)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_icpp_kasagini14_b200 as libsat
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "sat.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = set(re.findall(r"\b(sat_[a-z0-9_]+)\s*\(", src))
+    return sorted(n for n in names if n != "sat_allgather_fn")
+
+
+def test_every_declared_symbol_is_exported():
+    decl = declared_symbols()
+    assert len(decl) >= 15
+    for name in decl:
+        assert hasattr(libsat.lib, name), name
+        assert name in libsat.EXPORTED, name
+
+
+def test_abi_version_and_strings():
+    assert libsat.abi_version() == 1
+    assert libsat.lib.sat_strerror(0) == b"ok"
+    assert libsat.lib.sat_strerror(-1) == b"invalid argument"
+
+
+L = libsat.lib
+
+
+def test_validation_without_gpu():
+    # bad dtype
+    assert L.sat_compute(8, 8, 4, 4, 7, 2, None) == -1
+    assert b"dtype" in L.sat_last_error()
+    # negative sizes
+    assert L.sat_compute(8, 8, -1, 4, 0, 2, None) == -1
+    # null pointers with nonzero size
+    assert L.sat_compute(None, 64, 4, 4, 0, 2, None) == -1
+    # partial overlap
+    assert L.sat_compute(4096, 4100, 4, 4, 0, 2, None) == -1
+    assert b"overlap" in L.sat_last_error()
+    # misaligned
+    assert L.sat_compute(4097, 4097 + 1 << 20, 4, 4, 0, 2, None) == -1
+    # bad variant (valid pointers, validated before any CUDA call)
+    assert L.sat_compute(4096, 1 << 20, 4, 4, 0, 9, None) == -1
+    # empty is a no-op, no device needed
+    assert L.sat_compute(None, None, 0, 5, 0, 2, None) == 0
+    assert L.sat_compute(None, None, 5, 0, 1, 2, None) == 0
+    # bad options
+    o = libsat.options(tile_rows=48)
+    assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 2, ctypes.byref(o), None) == -1
+    o = libsat.options(r=1.5)
+    assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 3, ctypes.byref(o), None) == -1
+    # sharded argument checks
+    assert L.sat_compute_sharded(4096, 1 << 20, 4, 4, 0, 2, 2, libsat.ALLGATHER_FN(0),
+                                 None, None, None, None) == -1
+    assert L.sat_rank_exscan(None, 64, 2, 4, 3, 0, None) == -1
+    assert L.sat_sharded_workspace_bytes(1000, 4, 0) == 256 * 16 * 6
+    assert L.sat_compute_host(None, None, 0, 3, 0, 2, None) == 0
+
+
+def test_python_wrapper_rejects_cpu_tensors():
+    import torch
+    with pytest.raises(ValueError):
+        libsat.sat(torch.zeros(4, 4, dtype=torch.int32))
+    with pytest.raises(ValueError):
+        libsat.sat(torch.zeros(4, 4, 4, dtype=torch.int32))

@@ -1,0 +1,310 @@
+"""GPU parity: libsat (through the C ABI) vs the CPU oracle, element by element.
+
+int32: bit-exact (mod 2^32).  float32: max relative error <= 1e-5 against the
+float64 oracle with inputs in [0, 1) (north star (5)).
+Inputs are seeded and synthetic (sat_inputs); expected values come only from
+``oracle``.  Run on a B200 via gpurun: ``pytest -m gpu``.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from sat_inputs import make_np, make_torch
+
+pytestmark = pytest.mark.gpu
+
+VARIANTS = ["1r1w", "2r2w", "2r1w", "1+rr1w"]
+FTOL = 1e-5
+
+
+@pytest.fixture(scope="module")
+def libsat():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_icpp_kasagini14_b200 as m
+    return m
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def check(got, ref, dtype):
+    got = got.cpu().numpy() if isinstance(got, torch.Tensor) else got
+    if dtype == "int32":
+        if not np.array_equal(got, ref):
+            bad = np.argwhere(got != ref)
+            raise AssertionError(f"{len(bad)} mismatches, first at {bad[:5].tolist()}")
+    else:
+        err = oracle.max_rel_err(got, ref)
+        assert err <= FTOL, f"max rel err {err}"
+
+
+def gen(n, m, dtype, seed=1):
+    return make_np(n, m, dtype, "u32" if dtype == "int32" else "unit", seed=seed)
+
+
+# ------------------------------------------------------------------ worked example
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_fig3(libsat, fig3, variant, dtype):
+    a, _, b = fig3
+    x = dev(a.astype(dtype))
+    y = libsat.sat(x, variant=variant)
+    assert np.array_equal(y.cpu().numpy(), b.astype(dtype))
+
+
+# ------------------------------------------------------------------ shapes x variants
+SHAPES = [(1, 1), (1, 5), (5, 1), (3, 5), (15, 127), (16, 128), (17, 129), (63, 255),
+          (64, 256), (65, 257), (127, 129), (200, 1000), (1080, 1920), (333, 1001),
+          (1000, 4096), (2049, 513)]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: f"{s[0]}x{s[1]}")
+def test_shapes(libsat, variant, dtype, shape):
+    a = gen(*shape, dtype, seed=shape[0] * 7 + shape[1])
+    ref = oracle.sat(a)
+    check(libsat.sat(dev(a), variant=variant), ref, dtype)
+
+
+@pytest.mark.parametrize("tile_rows", [16, 32, 64])
+@pytest.mark.parametrize("generic", [False, True])
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_tile_configs(libsat, tile_rows, generic, variant):
+    for dtype in ("int32", "float32"):
+        a = gen(700, 1300, dtype, seed=tile_rows)
+        ref = oracle.sat(a)
+        check(libsat.sat(dev(a), variant=variant, tile_rows=tile_rows, force_generic=generic),
+              ref, dtype)
+        assert libsat.last_tile_rows() == tile_rows
+
+
+@pytest.mark.parametrize("r", [0.0, 0.1, 0.25, 0.5, 1.0])
+def test_1plusr_r_sweep(libsat, r):
+    a = gen(1500, 2000, "int32", seed=5)
+    ref = oracle.sat(a)
+    check(libsat.sat(dev(a), variant="1+rr1w", r=r, tile_rows=32), ref, "int32")
+    re = libsat.last_r_effective()
+    assert abs(re - r) < 0.15
+
+
+def test_in_place(libsat):
+    for variant in VARIANTS:
+        a = gen(517, 777, "int32", seed=3)
+        ref = oracle.sat(a)
+        x = dev(a)
+        y = libsat.sat(x, variant=variant, out=x)
+        assert y.data_ptr() == x.data_ptr()
+        check(x, ref, "int32")
+
+
+def test_input_not_modified(libsat):
+    a = gen(300, 400, "float32", seed=2)
+    x = dev(a)
+    for variant in VARIANTS:
+        libsat.sat(x, variant=variant)
+        assert np.array_equal(x.cpu().numpy(), a)
+
+
+def test_closed_forms(libsat):
+    n, m = 1024, 3000
+    ones = torch.ones(n, m, dtype=torch.int32, device="cuda")
+    i = np.arange(n, dtype=np.int64)[:, None] + 1
+    j = np.arange(m, dtype=np.int64)[None, :] + 1
+    for variant in VARIANTS:
+        got = libsat.sat(ones, variant=variant).cpu().numpy().astype(np.int64)
+        assert np.array_equal(got, i * j), variant
+    # float32 all-ones is exact while the SAT <= 2^24
+    f = torch.ones(2048, 2048, dtype=torch.float32, device="cuda")
+    for variant in VARIANTS:
+        got = libsat.sat(f, variant=variant).cpu().numpy()
+        assert np.array_equal(got, (np.arange(1, 2049)[:, None] * np.arange(1, 2049)[None, :]).astype(np.float32))
+
+
+def test_repeated_calls_fresh_tags(libsat):
+    """Descriptors are never cleared between calls: per-launch tags must keep
+    stale words from being taken (SURVEY 7 'flag reset between calls')."""
+    for k in range(40):
+        shape = (300 + 37 * k, 200 + 91 * k)
+        a = gen(*shape, "int32", seed=100 + k)
+        check(libsat.sat(dev(a)), oracle.sat(a), "int32")
+        assert libsat.last_launch_count() == 1
+
+
+def test_lookback_jitter_stress(libsat):
+    for th in (16, 32, 64):
+        a = gen(3000, 2500, "int32", seed=th)
+        check(libsat.sat(dev(a), tile_rows=th, jitter=20000), oracle.sat(a), "int32")
+        af = gen(3000, 2500, "float32", seed=th)
+        check(libsat.sat(dev(af), tile_rows=th, jitter=20000), oracle.sat(af), "float32")
+
+
+def test_int32_deterministic(libsat):
+    a = dev(gen(4096, 4096, "int32", seed=9))
+    r1 = libsat.sat(a).cpu()
+    for _ in range(3):
+        assert torch.equal(libsat.sat(a).cpu(), r1)
+
+
+# ------------------------------------------------------------------ batch / seeded / sharded
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_batched(libsat, variant):
+    for dtype in ("int32", "float32"):
+        a = make_np(130, 300, dtype, "u32" if dtype == "int32" else "unit", seed=4, batch=5)
+        y = libsat.sat_batched(dev(a), variant=variant).cpu().numpy()
+        for b in range(5):
+            check(y[b], oracle.sat(a[b]), dtype)
+
+
+def test_batched_images_cfg5_slice(libsat):
+    a = make_np(1080, 1920, "float32", "unit", seed=77, batch=4)
+    y = libsat.sat_batched(dev(a)).cpu().numpy()
+    for b in range(4):
+        check(y[b], oracle.sat(a[b]), "float32")
+    assert libsat.last_launch_count() == 1
+
+
+def test_seeded(libsat):
+    for dtype in ("int32", "float32"):
+        full = gen(900, 1100, dtype, seed=8)
+        ref = oracle.sat(full)
+        r0 = 311
+        strip = dev(full[r0:])
+        if dtype == "int32":
+            carry = oracle.column_totals(full[:r0])
+        else:
+            carry = full[:r0].astype(np.float64).sum(axis=0).astype(np.float32)
+        check(libsat.sat_seeded(strip, carry_row=dev(carry)), ref[r0:], dtype)
+        check(libsat.sat_seeded(strip, sat_row=dev(ref[r0 - 1].astype(dtype))), ref[r0:], dtype)
+
+
+def test_column_totals_and_exscan(libsat):
+    for dtype in ("int32", "float32"):
+        a = gen(5000, 1234, dtype, seed=6)
+        t = libsat.column_totals(dev(a)).cpu().numpy()
+        ref = oracle.column_totals(a)
+        if dtype == "int32":
+            assert np.array_equal(t, ref)
+        else:
+            assert np.max(np.abs(t - ref) / np.maximum(ref, 1e-30)) < 1e-5
+        g = gen(6, 1234, dtype, seed=7)
+        for rank in range(6):
+            e = libsat.rank_exscan(dev(g), rank).cpu().numpy()
+            r = oracle.rank_exscan(g, rank)
+            if dtype == "int32":
+                assert np.array_equal(e, r)
+            else:
+                assert np.allclose(e, r, rtol=1e-6, atol=0)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+def test_sharded_abi_single_process(libsat, P):
+    """sat_compute_sharded with a fake all-gather: P ranks simulated one after
+    another on one GPU; the concatenated strips must equal the unsharded SAT."""
+    from paper_conf_icpp_kasagini14_b200.dist import partition_rows
+    n, m = 2000, 1500
+    for dtype in ("int32", "float32"):
+        full = gen(n, m, dtype, seed=P)
+        ref = oracle.sat(full)
+        bounds = [partition_rows(n, P, p) for p in range(P)]
+        strips = [dev(full[r0:r1]) for r0, r1 in bounds]
+        totals = [libsat.column_totals(s) for s in strips]
+        totals[-1] = torch.zeros_like(totals[-1])
+        outs = []
+        for p in range(P):
+            def ag(send, recv, p=p):
+                torch.cuda.synchronize()
+                assert torch.equal(send, totals[p])
+                recv.copy_(torch.stack(totals))
+            o, st = libsat.sat_sharded_abi(strips[p], p, P, ag)
+            outs.append(o.cpu().numpy())
+            rows = bounds[p][1] - bounds[p][0]
+            assert st["extra_bytes_read"] == (rows * m * 4 if (P > 1 and p < P - 1) else 0)
+        check(np.concatenate(outs), ref, dtype)
+
+
+# ------------------------------------------------------------------ host e2e
+@pytest.mark.parametrize("pinned", [True, False])
+def test_host_end_to_end(libsat, pinned):
+    for dtype in ("int32", "float32"):
+        a = gen(3000, 2048, dtype, seed=12)
+        x = torch.from_numpy(a)
+        if pinned:
+            x = x.pin_memory()
+        y = libsat.sat_host(x)
+        check(y.numpy(), oracle.sat(a), dtype)
+
+
+# ------------------------------------------------------------------ BASELINE.json configs
+def test_cfg1_1024_int32(libsat):
+    a = gen(1024, 1024, "int32", seed=1001)
+    check(libsat.sat(dev(a)), oracle.sat(a), "int32")
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_cfg2_4096_float32(libsat, variant):
+    a = gen(4096, 4096, "float32", seed=2001)
+    check(libsat.sat(dev(a), variant=variant), oracle.sat(a), "float32")
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("n", [16384, 18432])
+def test_cfg3_full_int32(libsat, n):
+    """Full-size parity in the launch configuration bench.py times."""
+    x = make_torch(n, n, "int32", "u32", seed=3001, device="cuda")
+    y = libsat.sat(x).cpu().numpy()
+    a = x.cpu().numpy()
+    del x
+    st = oracle.Stream(n, True)
+    step = 2048
+    for r0 in range(0, n, step):
+        ref = st.feed(a[r0:r0 + step])
+        assert np.array_equal(y[r0:r0 + step], ref), f"rows {r0}.."
+
+
+@pytest.mark.slow
+def test_cfg3_float32_16k(libsat):
+    n = 16384
+    x = make_torch(n, n, "float32", "unit", seed=3002, device="cuda")
+    y = libsat.sat(x).cpu().numpy()
+    a = x.cpu().numpy()
+    st = oracle.Stream(n, False)
+    worst = 0.0
+    for r0 in range(0, n, 2048):
+        ref = st.feed(a[r0:r0 + 2048])
+        worst = max(worst, oracle.max_rel_err(y[r0:r0 + 2048], ref))
+    assert worst <= FTOL, worst
+
+
+@pytest.mark.slow
+def test_cfg4_65536_properties(libsat):
+    """64K x 64K int32 (16 GiB): closed form on all-ones (wrap pins:
+    b[65535][65535] = 0, b[32767][65535] = INT32_MIN) and sampled exact
+    elements of a random matrix via the oracle's one-element sum."""
+    n = 65536
+    x = torch.ones(n, n, dtype=torch.int32, device="cuda")
+    libsat.sat(x, out=x)
+    assert int(x[65535, 65535]) == 0
+    assert int(x[32767, 65535]) == -2**31
+    for r in (0, 1, 4095, 30000, 65535):
+        row = x[r].cpu().numpy().view(np.uint32).astype(np.int64)
+        assert np.array_equal(row, ((r + 1) * np.arange(1, n + 1, dtype=np.int64)) % 2**32)
+    del x
+    torch.cuda.empty_cache()
+    x = make_torch(n, n, "int32", "u32", seed=4001, device="cuda")
+    y = libsat.sat(x)
+    torch.cuda.synchronize()
+    # exact elements near the top-left (oracle one-element sums on a host block)
+    blk = x[:512, :].cpu().numpy()
+    for (i, j) in [(0, 0), (511, 65535), (300, 40000), (17, 65535)]:
+        assert int(y[i, j]) == int(oracle.sat_at(blk, i, j))
+    # inclusion-exclusion recovers the input on sampled 2x2 windows everywhere
+    rng = np.random.default_rng(0)
+    for _ in range(200):
+        i = int(rng.integers(1, n)); j = int(rng.integers(1, n))
+        w = y[i - 1:i + 1, j - 1:j + 1].cpu().numpy().view(np.uint32)
+        with np.errstate(over="ignore"):
+            rec = w[1, 1] - w[0, 1] - w[1, 0] + w[0, 0]
+        assert rec == np.uint32(int(x[i, j]) & 0xFFFFFFFF)
