@@ -163,6 +163,14 @@ size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype);
 int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t cols,
                      int dtype, int variant, void *stream);
 
+/* Debug/profiling: the next 1R1W-family band launch on this thread records,
+ * per (band, chunk) of TH x 128 elements, four 64-bit globaltimer stamps
+ * (ns) into dev_buf[(band*nchunks + chunk)*4 + e]: e=0 tile data arrived,
+ * e=1 band-local reductions done, e=2 look-back done (bits 48..63 = number
+ * of look-back hops), e=3 tile store issued.  dev_buf (device, caller-owned)
+ * must hold ceil(rows/TH)*batch*ceil(cols/128)*32 bytes; NULL disarms. */
+int sat_debug_trace(void *dev_buf);
+
 /* Number of kernels launched by the last successful call on this thread. */
 int sat_last_launch_count(void);
 /* Band height used by the last 1R1W-family call on this thread. */

@@ -54,6 +54,7 @@ _SIGS = {
                              ctypes.POINTER(SatShardStats)], _I),
     "sat_sharded_workspace_bytes": ([_I64, _I, _I], ctypes.c_size_t),
     "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
+    "sat_debug_trace": ([_P], _I),
     "sat_last_launch_count": ([], _I),
     "sat_last_tile_rows": ([], _I),
     "sat_last_r_effective": ([], ctypes.c_double),
@@ -265,3 +266,9 @@ def abi_version() -> int:
 
 
 lib = _lib
+
+
+def debug_trace(buf) -> None:
+    """Arm event tracing of the next band launch on this thread (see
+    ``sat_debug_trace`` in include/sat.h); ``buf`` is a CUDA int64 tensor."""
+    _check(_lib.sat_debug_trace(None if buf is None else buf.data_ptr()))

@@ -29,6 +29,7 @@ thread_local std::string t_err;
 thread_local int t_launches = 0;
 thread_local int t_th = 0;
 thread_local double t_r = 0.0;
+thread_local unsigned long long* t_trace = nullptr;
 
 int fail(int code, const std::string& msg) {
     t_err = msg;
@@ -271,6 +272,10 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * p.nc : p.total_bands;
     p.jitter = j.jitter;
+    if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
+        p.trace = t_trace;
+        t_trace = nullptr;
+    }
     Workspace& ws = *j.ws;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
         const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t);
@@ -737,6 +742,11 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     cudaEventDestroy(ev_start);
     for (int k = 0; k < nstrips; ++k) { cudaEventDestroy(ev_in[k]); cudaEventDestroy(ev_done[k]); }
     t_launches = launches;
+    return SAT_OK;
+}
+
+int sat_debug_trace(void* dev_buf) {
+    t_trace = static_cast<unsigned long long*>(dev_buf);
     return SAT_OK;
 }
 

@@ -160,6 +160,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 }
                 if constexpr (TMA) {
                     mbar_wait(&full[s], ph);
+                    if (p.trace && warp == 0 && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 0] = globaltimer();
                     const T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
@@ -260,6 +262,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     const int J = j0 + k;
                     const int c0 = J * TW + 4 * lane;
                     mbar_wait(&colr[s], ph);
+                    if (p.trace && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 1] = globaltimer();
+                    unsigned long long hops = 0;
                     V4<T> agg = lds4<T>(xbuf + size_t(s) * W * TW + 4 * lane);
                     for (int w2 = 1; w2 < W; ++w2)
                         add4(agg, lds4<T>(xbuf + (size_t(s) * W + w2) * TW + 4 * lane));
@@ -333,6 +338,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                     }
                                 }
                                 --kb;
+                                ++hops;
                             }
                             top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
                         }
@@ -344,6 +350,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             st_relaxed_v2(my + 2, (uint64_t(tP) << 32) | to_bits(inc.z), (uint64_t(tP) << 32) | to_bits(inc.w));
                         }
                     }
+                    if (p.trace && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 2] = (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
                     sts4(topb + size_t(s) * TW + 4 * lane, top);
                     mbar_arrive(&topr[s]);
                 }
@@ -368,6 +376,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         const int s = it % S;
                         const uint32_t ph = (it / S) & 1;
                         mbar_wait(&done[s], ph);
+                        if (p.trace)
+                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 4 + 3] = globaltimer();
                         tma_store_3d(&tm_out, tiles + size_t(s) * SM::tile_elems, (j0 + k) * TW, row0, img, pol);
                         bulk_commit();
                         if (k + S < nch) { bulk_wait_read<0>(); load(k + S); }

@@ -57,6 +57,7 @@ struct BandParams {
     const void* TopX;          // [total_bands][nc*TW] external SAT row above, nullable
     void* Lb;                  // [total_bands*TH] band-final row carry out, nullable
     int jitter;                // debug: random publish delay (ns scale), 0 = off
+    unsigned long long* trace; // debug: [total_bands*nc][4] event times (ns), nullable
 };
 
 }  // namespace sat

@@ -94,6 +94,12 @@ __device__ __forceinline__ void ld_relaxed_v2(const uint64_t* p, uint64_t& a, ui
     asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 
+__device__ __forceinline__ unsigned long long globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
 // ------------------------------------------------------------- arithmetic
 // int32 SATs are computed in uint32 (mod 2^32); float32 in IEEE fp32 adds.
 template <typename T> __device__ __forceinline__ uint32_t to_bits(T v);

@@ -1,0 +1,31 @@
+"""Record per-(band, chunk) look-back event times of one 1R1W launch.
+
+python tools/trace_lookback.py rows cols tile_rows out.npz
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import paper_conf_icpp_kasagini14_b200 as libsat
+from sat_inputs import make_torch
+
+rows, cols, th = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
+out = sys.argv[4]
+x = make_torch(rows, cols, "int32", "u32", seed=1, device="cuda")
+y = torch.empty_like(x)
+for _ in range(3):
+    libsat.sat(x, out=y, tile_rows=th)
+nb, nc = (rows + th - 1) // th, (cols + 127) // 128
+buf = torch.zeros(nb * nc * 4, dtype=torch.int64, device="cuda")
+torch.cuda.synchronize()
+s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+libsat.debug_trace(buf)
+s.record()
+libsat.sat(x, out=y, tile_rows=th)
+e.record()
+torch.cuda.synchronize()
+print("ms", s.elapsed_time(e), "th", libsat.last_tile_rows())
+np.savez_compressed(out, trace=buf.cpu().numpy().reshape(nb, nc, 4), ms=s.elapsed_time(e))
