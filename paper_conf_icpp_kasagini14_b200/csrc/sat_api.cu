@@ -175,19 +175,19 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
 
 // ------------------------------------------------------------------ band kernel dispatch
 struct BandCfg {
-    int R, W, S, MINB;
+    int R, W, S, D, MINB;
 };
 // TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
-// S*W*512 (warp bottom rows) + S*512 (SAT row above) + barriers.
-constexpr BandCfg kCfg16{2, 8, 4, 4};
-constexpr BandCfg kCfg32{4, 8, 4, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 2};
+// (D+1)*W*512 (warp bottom rows / add vectors) + barriers.
+constexpr BandCfg kCfg16{2, 8, 8, 2, 2};
+constexpr BandCfg kCfg32{4, 8, 6, 2, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 1, 2};
 
-template <typename T, int R, int W, int S, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int D, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, MODE, TMA, MINB>;
-    const size_t smem = BandSmem<T, R, W, S>::total;
+    auto kern = sat_band_kernel<T, R, W, S, D, MODE, TMA, MINB>;
+    const size_t smem = BandSmem<T, R, W, S, D>::total;
     const int threads = (W + 2) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
@@ -206,13 +206,14 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     return SAT_OK;
 }
 
+#define SAT_CFG(c) c.R, c.W, c.S, c.D
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {
     switch (th) {
-        case 16: return launch_band_t<T, kCfg16.R, kCfg16.W, kCfg16.S, MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
-        case 32: return launch_band_t<T, kCfg32.R, kCfg32.W, kCfg32.S, MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
-        case 64: return launch_band_t<T, kCfg64.R, kCfg64.W, kCfg64.S, MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
+        case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
+        case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
+        case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
     }
     return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32 or 64");
 }

@@ -8,17 +8,22 @@
 // everything:
 //   * a CTA takes a band of TH rows (ticket order = band order, so every band
 //     it waits on is held by a running or finished CTA) and walks it left to
-//     right in TH x 128 chunks staged through a TMA ring in shared memory;
+//     right in TH x 128 chunks staged through an S-slot TMA ring in smem;
 //   * the horizontal carry (the paper's R) is the per-row running sum L held
 //     in registers by the warp that owns the row;
 //   * the vertical carry (the paper's C and S, i.e. the SAT row above the
-//     band) comes from a decoupled look-back over flag-guarded descriptors:
-//     each (band, chunk) publishes the bottom row of its band-local SAT as an
-//     "aggregate", then -- once it knows the SAT row above -- the final SAT
-//     bottom row as "inclusive";
-//   * inside a chunk, Step 3-1/3-2 of 2R1W become: row scan
-//     (in-thread + warp shuffle) with L, column prefix down the warp's R rows,
-//     a cross-warp exchange of warp bottom rows, then + (SAT row above).
+//     band) comes from a decoupled look-back over self-validating descriptor
+//     words: each (band, chunk) publishes the bottom row of its band-local SAT
+//     as an "aggregate", then -- once it knows the SAT row above -- the final
+//     SAT bottom row as "inclusive".  The look-back reads a
+//     window of LBW bands per round trip;
+//   * inside a chunk, Step 3-1/3-2 of 2R1W become two passes over
+//     the smem slot: local() = row scans with L + column prefix down the
+//     warp's R rows (written back in place; the warp's bottom row goes to
+//     xbuf); finish() = + (SAT row above the band + bottom rows of the warps
+//     above), computed by the control warp.  finish(k) runs D chunks after
+//     local(k), so the look-back latency of chunk k overlaps the local work
+//     of chunks k+1..k+D.
 //
 // The same kernel, with MODE/TopSrc switches, is the column pass and row pass
 // of 2R2W, Step 3 of 2R1W with external carries
@@ -50,18 +55,65 @@ __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S>
+template <typename T, int R, int W, int S, int D>
 struct BandSmem {
     static constexpr int TH = R * W;
+    static constexpr int XS = D + 1;                 // xbuf slots
     static constexpr size_t tile_elems = size_t(TH) * TW;
     static constexpr size_t tiles = S * tile_elems * sizeof(T);
-    static constexpr size_t xbuf = size_t(S) * W * TW * sizeof(T);
-    static constexpr size_t topb = size_t(S) * TW * sizeof(T);
+    static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
     static constexpr size_t bars = size_t(4) * S * sizeof(uint64_t) + 16;
-    static constexpr size_t total = tiles + xbuf + topb + bars;
+    static constexpr size_t total = tiles + xbuf + bars;
 };
 
-template <typename T, int R, int W, int S, int MODE, bool TMA, int MINB>
+constexpr int LBW = 4;   // look-back window: bands read per round trip
+
+__device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
+    return uint32_t((base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
+}
+
+template <typename T>
+__device__ __forceinline__ void publish4(uint64_t* my, uint32_t tag, const V4<T>& v) {
+    st_relaxed_v2(my, (uint64_t(tag) << 32) | to_bits(v.x), (uint64_t(tag) << 32) | to_bits(v.y));
+    st_relaxed_v2(my + 2, (uint64_t(tag) << 32) | to_bits(v.z), (uint64_t(tag) << 32) | to_bits(v.w));
+}
+
+// Row-wise inclusive prefix-sums of R rows of 128 columns (lane owns 4
+// consecutive columns), continuing from the running row sums L, which are
+// advanced to the end of the chunk.  Rows are interleaved step by step so the
+// shuffles of different rows overlap.
+template <typename T, int R>
+__device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
+    T inc[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        v[r].y += v[r].x; v[r].z += v[r].y; v[r].w += v[r].z;
+        inc[r] = v[r].w;
+    }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const T y = __shfl_up_sync(0xffffffffu, inc[r], d);
+            if (lane >= d) inc[r] += y;
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        T exc;
+        if constexpr (std::is_same<T, uint32_t>::value) {
+            exc = inc[r] - v[r].w;                 // exact in Z/2^32
+        } else {
+            exc = __shfl_up_sync(0xffffffffu, inc[r], 1);
+            if (lane == 0) exc = T(0);
+        }
+        const T off = L[r] + exc;
+        v[r].x += off; v[r].y += off; v[r].z += off; v[r].w += off;
+        L[r] += __shfl_sync(0xffffffffu, inc[r], 31);
+    }
+}
+
+template <typename T, int R, int W, int S, int D, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + 2) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const __grid_constant__ CUtensorMap tm_out,
@@ -71,17 +123,18 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int CW = W;          // control warp
     constexpr int PW = W + 1;      // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S>;
+    using SM = BandSmem<T, R, W, S, D>;
+    constexpr int XS = SM::XS;
+    static_assert(S >= D + 2, "ring must hold D finished-pending chunks plus a prefetch");
 
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
-    T* topb = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf + SM::topb);
-    uint64_t* full = bars;
-    uint64_t* colr = bars + S;
-    uint64_t* topr = bars + 2 * S;
-    uint64_t* done = bars + 3 * S;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf);
+    uint64_t* full = bars;          // TMA load landed (tx count)
+    uint64_t* colr = bars + S;      // every compute warp finished local()
+    uint64_t* topr = bars + 2 * S;  // control warp wrote the add vectors
+    uint64_t* done = bars + 3 * S;  // every compute warp finished finish()
     long long* s_unit = reinterpret_cast<long long*>(bars + 4 * S);
 
     const int warp = threadIdx.x >> 5;
@@ -134,39 +187,31 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             T L[R];
 #pragma unroll
             for (int r = 0; r < R; ++r) L[r] = T(0);
-            auto load_L = [&](int J) {
-                if (p.Lx != nullptr) {
-                    const T* lx = reinterpret_cast<const T*>(p.Lx) + int64_t(J) * lx_stride
-                                  + int64_t(gb) * TH + rbase;
+            if (p.Lx != nullptr) {
+                const T* lx = reinterpret_cast<const T*>(p.Lx) + int64_t(j0) * lx_stride
+                              + int64_t(gb) * TH + rbase;
 #pragma unroll
-                    for (int r = 0; r < R; ++r) L[r] = lx[r];
-                }
-            };
-            load_L(j0);
-
+                for (int r = 0; r < R; ++r) L[r] = lx[r];
+            }
             const T* gin = reinterpret_cast<const T*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
 
-            // local(): load chunk k, row scans with L, column prefix, publish warp bottom row
-            auto local = [&](V4<T> (&v)[R], int k) {
+            // local(k): row scans with L, column prefix down this warp's rows,
+            // result back into the slot, warp bottom row into xbuf
+            auto local = [&](int k) {
                 const uint32_t it = g + k;
                 const int s = it % S;
                 const uint32_t ph = (it / S) & 1;
-                const int J = j0 + k;
-                if (p.tile_units && k == 0) load_L(J);
-                if constexpr (!TMA) {
-                    // generic path: slot s is free once every warp finished its previous use
-                    if (it >= uint32_t(S)) mbar_wait(&done[s], ph ^ 1u);
-                }
+                T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
+                V4<T> v[R];
                 if constexpr (TMA) {
                     mbar_wait(&full[s], ph);
                     if (p.trace && warp == 0 && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 0] = globaltimer();
-                    const T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
+                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 4 + 0] = globaltimer();
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
                 } else {
-                    const int64_t c = int64_t(J) * TW + 4 * lane;
+                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
                         const int64_t row = row0 + rbase + r;
@@ -177,49 +222,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         v[r] = V4<T>{e[0], e[1], e[2], e[3]};
                     }
                 }
-                if constexpr (MODE != MODE_COL) {
-                    // row-wise prefix-sums (the paper's R carry lives in L)
-#pragma unroll
-                    for (int r = 0; r < R; ++r) {
-                        v[r].y += v[r].x; v[r].z += v[r].y; v[r].w += v[r].z;
-                        const T inc = warp_inclusive_scan(v[r].w, lane);
-                        T exc = __shfl_up_sync(0xffffffffu, inc, 1);
-                        if (lane == 0) exc = T(0);
-                        const T off = L[r] + exc;
-                        v[r].x += off; v[r].y += off; v[r].z += off; v[r].w += off;
-                        L[r] += __shfl_sync(0xffffffffu, inc, 31);
-                    }
-                }
+                if constexpr (MODE != MODE_COL) row_scan<T, R>(v, L, lane);
                 if constexpr (MODE != MODE_ROW) {
-                    // column-wise prefix-sums down this warp's rows
 #pragma unroll
                     for (int r = 1; r < R; ++r) add4(v[r], v[r - 1]);
-                    sts4(xbuf + (size_t(s) * W + warp) * TW + 4 * lane, v[R - 1]);
-                    mbar_arrive(&colr[s]);
+                    sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
                 }
-            };
-            // finish(): + (SAT row above the band) + (bottom rows of the warps above), store
-            auto finish = [&](V4<T> (&v)[R], int k) {
-                const uint32_t it = g + k;
-                const int s = it % S;
-                const uint32_t ph = (it / S) & 1;
-                const int J = j0 + k;
-                if constexpr (MODE != MODE_ROW) {
-                    mbar_wait(&topr[s], ph);
-                    V4<T> add = lds4<T>(topb + size_t(s) * TW + 4 * lane);
-                    for (int w2 = 0; w2 < warp; ++w2)
-                        add4(add, lds4<T>(xbuf + (size_t(s) * W + w2) * TW + 4 * lane));
-#pragma unroll
-                    for (int r = 0; r < R; ++r) add4(v[r], add);
-                }
-                if constexpr (TMA) {
-                    T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
-#pragma unroll
-                    for (int r = 0; r < R; ++r) sts4(t + r * TW, v[r]);
-                    fence_proxy_async_smem();
-                    mbar_arrive(&done[s]);
-                } else {
-                    const int64_t c = int64_t(J) * TW + 4 * lane;
+                if constexpr (MODE == MODE_ROW && !TMA) {
+                    // the row pass is final: write straight out
+                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
                         const int64_t row = row0 + rbase + r;
@@ -230,20 +241,59 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                 if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
                         }
                     }
+                } else {
+#pragma unroll
+                    for (int r = 0; r < R; ++r) sts4(t + r * TW, v[r]);
+                }
+                if constexpr (MODE == MODE_ROW) {
+                    if constexpr (TMA) fence_proxy_async_smem();
                     mbar_arrive(&done[s]);
+                } else {
+                    mbar_arrive(&colr[s]);
                 }
             };
-
-            V4<T> va[R], vb[R];
-            if (nch > 0) {
-                local(va, 0);
-                for (int k = 0; k < nch; k += 2) {
-                    if (k + 1 < nch) local(vb, k + 1);
-                    finish(va, k);
-                    if (k + 1 >= nch) break;
-                    if (k + 2 < nch) local(va, k + 2);
-                    finish(vb, k + 1);
+            // finish(k): + (SAT row above + bottom rows of the warps above), store
+            auto finish = [&](int k) {
+                const uint32_t it = g + k;
+                const int s = it % S;
+                const uint32_t ph = (it / S) & 1;
+                mbar_wait(&topr[s], ph);
+                const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
+                T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
+                if constexpr (TMA) {
+#pragma unroll
+                    for (int r = 0; r < R; ++r) {
+                        V4<T> v = lds4<T>(t + r * TW);
+                        add4(v, add);
+                        sts4(t + r * TW, v);
+                    }
+                    fence_proxy_async_smem();
+                } else {
+                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
+#pragma unroll
+                    for (int r = 0; r < R; ++r) {
+                        V4<T> v = lds4<T>(t + r * TW);
+                        add4(v, add);
+                        const int64_t row = row0 + rbase + r;
+                        if (row < p.rows) {
+                            const T e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                            for (int i = 0; i < 4; ++i)
+                                if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
+                        }
+                    }
                 }
+                mbar_arrive(&done[s]);
+            };
+
+            if constexpr (MODE == MODE_ROW) {
+                for (int k = 0; k < nch; ++k) local(k);
+            } else {
+                for (int k = 0; k < nch; ++k) {
+                    local(k);
+                    if (k >= D) finish(k - D);
+                }
+                for (int k = (nch > D ? nch - D : 0); k < nch; ++k) finish(k);
             }
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;
@@ -253,7 +303,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         } else if (warp == CW) {
             // ================= control warp: descriptors + look-back =================
             if constexpr (MODE != MODE_ROW) {
-                const uint32_t tagbase = uint32_t((p.base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
+                const uint32_t tagbase = band_tag(p.base, gb);
+                const bool lookback = (p.top_src == TOP_LOOKBACK);
+                const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
+                const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
                 if (band == 0) seedrun = T(0);
                 for (int k = 0; k < nch; ++k) {
                     const uint32_t it = g + k;
@@ -261,55 +314,70 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     const uint32_t ph = (it / S) & 1;
                     const int J = j0 + k;
                     const int c0 = J * TW + 4 * lane;
+                    T* xb = xbuf + size_t(it % XS) * W * TW + 4 * lane;
                     mbar_wait(&colr[s], ph);
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 4 + 1] = globaltimer();
-                    unsigned long long hops = 0;
-                    V4<T> agg = lds4<T>(xbuf + size_t(s) * W * TW + 4 * lane);
-                    for (int w2 = 1; w2 < W; ++w2)
-                        add4(agg, lds4<T>(xbuf + (size_t(s) * W + w2) * TW + 4 * lane));
+                    V4<T> agg = lds4<T>(xb);
+#pragma unroll
+                    for (int w2 = 1; w2 < W; ++w2) add4(agg, lds4<T>(xb + w2 * TW));
+                    uint64_t* my = p.desc + int64_t(gb) * desc_w + c0;
+                    if (p.jitter && lookback) {
+                        uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ lane;
+                        h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
+                        __nanosleep(h % (uint32_t)p.jitter);
+                    }
+                    if (publish && band > 0) publish4<T>(my, tagbase | 1u, agg);
                     V4<T> top{T(0), T(0), T(0), T(0)};
-                    if (p.top_src == TOP_EXTERNAL) {
+                    unsigned long long hops = 0;
+                    if (!lookback) {
                         top = lds4<T>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0);
-                    } else {
-                        uint64_t* my = p.desc + int64_t(gb) * desc_w + c0;
-                        if (p.jitter) {
-                            uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ lane;
-                            h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
-                            __nanosleep(h % (uint32_t)p.jitter);
-                        }
-                        if (band == 0) {
-                            if (p.seed_kind != SEED_NONE && img == 0) {
-                                const T* sd = reinterpret_cast<const T*>(p.seed);
-                                T e[4];
+                    } else if (band == 0) {
+                        if (p.seed_kind != SEED_NONE && img == 0) {
+                            const T* sd = reinterpret_cast<const T*>(p.seed);
+                            T e[4];
 #pragma unroll
-                                for (int i = 0; i < 4; ++i) e[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
-                                if (p.seed_kind == SEED_COLSUM && MODE == MODE_SAT) {
-                                    // SAT row above = row prefix of the column sums above
-                                    e[1] += e[0]; e[2] += e[1]; e[3] += e[2];
-                                    const T inc = warp_inclusive_scan(e[3], lane);
-                                    T exc = __shfl_up_sync(0xffffffffu, inc, 1);
-                                    if (lane == 0) exc = T(0);
-                                    const T off = seedrun + exc;
+                            for (int i = 0; i < 4; ++i) e[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
+                            if (p.seed_kind == SEED_COLSUM && MODE == MODE_SAT) {
+                                // SAT row above = row prefix of the column sums above
+                                e[1] += e[0]; e[2] += e[1]; e[3] += e[2];
+                                const T inc = warp_inclusive_scan(e[3], lane);
+                                T exc = __shfl_up_sync(0xffffffffu, inc, 1);
+                                if (lane == 0) exc = T(0);
+                                const T off = seedrun + exc;
 #pragma unroll
-                                    for (int i = 0; i < 4; ++i) e[i] += off;
-                                    seedrun += __shfl_sync(0xffffffffu, inc, 31);
-                                }
-                                top = V4<T>{e[0], e[1], e[2], e[3]};
+                                for (int i = 0; i < 4; ++i) e[i] += off;
+                                seedrun += __shfl_sync(0xffffffffu, inc, 31);
                             }
-                        } else {
-                            // publish aggregate (band-local), then look back
-                            const uint32_t tA = tagbase | 1u;
-                            st_relaxed_v2(my, (uint64_t(tA) << 32) | to_bits(agg.x), (uint64_t(tA) << 32) | to_bits(agg.y));
-                            st_relaxed_v2(my + 2, (uint64_t(tA) << 32) | to_bits(agg.z), (uint64_t(tA) << 32) | to_bits(agg.w));
-                            T acc[4] = {T(0), T(0), T(0), T(0)};
-                            uint32_t pend = 0xFu;
-                            int kb = band - 1;
-                            const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
-                            while (pend) {
-                                if (p.region == REG_C && kb + J < p.tA) {
-                                    // tile (kb, J) belongs to (A): its final SAT row is in `out`
-                                    const int64_t row = int64_t(kb + 1) * TH - 1;
+                            top = V4<T>{e[0], e[1], e[2], e[3]};
+                        }
+                    } else {
+                        // decoupled look-back over bands band-1, band-2, ...,
+                        // LBW descriptor rows per round trip
+                        T acc[4] = {T(0), T(0), T(0), T(0)};
+                        uint32_t pend = 0xFu;
+                        int kb = band - 1;
+                        while (pend) {
+                            uint64_t wv[LBW][4];
+#pragma unroll
+                            for (int q = 0; q < LBW; ++q) {
+                                const int b2 = kb - q;
+                                if (b2 >= 0) {
+                                    const uint64_t* qp = p.desc + (int64_t(gb) - (band - b2)) * desc_w + c0;
+                                    ld_relaxed_v2(qp, wv[q][0], wv[q][1]);
+                                    ld_relaxed_v2(qp + 2, wv[q][2], wv[q][3]);
+                                } else {
+                                    wv[q][0] = wv[q][1] = wv[q][2] = wv[q][3] = 0;
+                                }
+                            }
+                            bool stalled = false;
+#pragma unroll
+                            for (int q = 0; q < LBW; ++q) {
+                                if (!pend || stalled) break;
+                                const int b2 = kb - q;
+                                if (p.region == REG_C && b2 + J < p.tA) {
+                                    // tile (b2, J) belongs to (A): its final SAT row is in `out`
+                                    const int64_t row = int64_t(b2 + 1) * TH - 1;
 #pragma unroll
                                     for (int i = 0; i < 4; ++i)
                                         if ((pend >> i) & 1u)
@@ -317,42 +385,44 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                     pend = 0;
                                     break;
                                 }
-                                const uint64_t* q = p.desc + (int64_t(gb) - (band - kb)) * desc_w + c0;
-                                const uint32_t tk = uint32_t((p.base + (unsigned long long)(gb - (band - kb))) & 0x3FFFFFFFull) << 2;
-                                uint64_t w0, w1, w2, w3;
-                                ld_relaxed_v2(q, w0, w1);
-                                ld_relaxed_v2(q + 2, w2, w3);
-                                const uint64_t ws[4] = {w0, w1, w2, w3};
+                                const uint32_t tk = band_tag(p.base, gb - (band - b2));
                                 bool ready = true;
 #pragma unroll
                                 for (int i = 0; i < 4; ++i) {
-                                    const uint32_t t = uint32_t(ws[i] >> 32);
+                                    const uint32_t t = uint32_t(wv[q][i] >> 32);
                                     ready = ready && ((t & ~3u) == tk) && (t & 3u);
                                 }
-                                if (!ready) { __nanosleep(16); continue; }
+                                if (!ready) { stalled = true; kb = b2; break; }
 #pragma unroll
                                 for (int i = 0; i < 4; ++i) {
                                     if ((pend >> i) & 1u) {
-                                        acc[i] += from_bits<T>(uint32_t(ws[i]));
-                                        if ((uint32_t(ws[i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
+                                        acc[i] += from_bits<T>(uint32_t(wv[q][i]));
+                                        if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
                                     }
                                 }
-                                --kb;
                                 ++hops;
                             }
-                            top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
+                            if (stalled) __nanosleep(32);
+                            else kb -= LBW;
                         }
-                        if (p.nb > 1) {
-                            V4<T> inc = agg;
-                            add4(inc, top);
-                            const uint32_t tP = tagbase | 2u;
-                            st_relaxed_v2(my, (uint64_t(tP) << 32) | to_bits(inc.x), (uint64_t(tP) << 32) | to_bits(inc.y));
-                            st_relaxed_v2(my + 2, (uint64_t(tP) << 32) | to_bits(inc.z), (uint64_t(tP) << 32) | to_bits(inc.w));
-                        }
+                        top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
+                    }
+                    if (publish) {
+                        V4<T> inc = agg;
+                        add4(inc, top);
+                        publish4<T>(my, tagbase | 2u, inc);
                     }
                     if (p.trace && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 2] = (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
-                    sts4(topb + size_t(s) * TW + 4 * lane, top);
+                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 2] =
+                            (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
+                    // add vectors for finish(): top + bottom rows of the warps above
+                    V4<T> run = top;
+#pragma unroll
+                    for (int w2 = 0; w2 < W; ++w2) {
+                        const V4<T> b = lds4<T>(xb + w2 * TW);
+                        sts4(xb + w2 * TW, run);
+                        add4(run, b);
+                    }
                     mbar_arrive(&topr[s]);
                 }
             }

@@ -5,6 +5,7 @@
 // by every SAT kernel.  Nothing here is shared with the CPU oracle.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda.h>
 
 namespace sat {

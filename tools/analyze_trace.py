@@ -1,0 +1,30 @@
+"""Summarise a look-back trace written by tools/trace_lookback.py."""
+import sys
+
+import numpy as np
+
+d = np.load(sys.argv[1])
+t = d["trace"].astype(np.int64)
+nb, nc, _ = t.shape
+hops = (t[:, :, 2] >> 48) & 0xFFFF
+t &= (1 << 48) - 1
+lo = t[:, :, 0][t[:, :, 0] > 0].min()
+t = (t - lo) / 1000.0                          # us since first tile arrival
+print(f"kernel ms {float(d['ms']):.3f}  bands {nb} chunks {nc}")
+start = t[:, 0, 0]
+end = t[:, -1, 3]
+print("band start  (us): min %.1f med %.1f max %.1f" % (start.min(), np.median(start), start.max()))
+print("band end    (us): min %.1f med %.1f max %.1f" % (end.min(), np.median(end), end.max()))
+dur = end - start
+print("band dur    (us): min %.1f med %.1f max %.1f" % (dur.min(), np.median(dur), dur.max()))
+per = np.diff(t[:, :, 0], axis=1)
+print("chunk period (us, arrival-to-arrival): med %.2f p90 %.2f" % (np.median(per), np.percentile(per, 90)))
+loc = t[:, :, 1] - t[:, :, 0]
+lb = t[:, :, 2] - t[:, :, 1]
+st = t[:, :, 3] - t[:, :, 2]
+print("arrival->local done med %.2f | local->lookback done med %.2f p90 %.2f | lookback->store med %.2f" %
+      (np.median(loc), np.median(lb), np.percentile(lb, 90), np.median(st)))
+lag = t[1:, :, 2] - t[:-1, :, 2]
+print("inter-band lag of look-back completion (us): med %.2f p10 %.2f p90 %.2f" %
+      (np.median(lag), np.percentile(lag, 10), np.percentile(lag, 90)))
+print("hops: mean %.2f max %d; share of chunks with hops>1: %.3f" % (hops.mean(), hops.max(), (hops > 1).mean()))
