@@ -113,6 +113,7 @@ struct Workspace {
     unsigned long long next_base = 0;
     Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
     Buf part;                 // column totals partials
+    Buf seedrow;              // seeded mode: SAT row above the strip
     Buf shard;                // sharded default workspace
     Buf din, dout;            // host e2e device copies
     cudaStream_t cstream_in = nullptr, cstream_out = nullptr;
@@ -175,20 +176,20 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
 
 // ------------------------------------------------------------------ band kernel dispatch
 struct BandCfg {
-    int R, W, S, D, MINB;
+    int R, W, S, D, NCW, MINB;
 };
 // TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
 // (D+1)*W*512 (warp bottom rows / add vectors) + barriers.
-constexpr BandCfg kCfg16{2, 8, 8, 2, 2};
-constexpr BandCfg kCfg32{4, 8, 6, 2, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 1, 2};
+constexpr BandCfg kCfg16{2, 8, 8, 3, 3, 2};
+constexpr BandCfg kCfg32{4, 8, 6, 3, 3, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 1, 2, 2};
 
-template <typename T, int R, int W, int S, int D, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int D, int NCW, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, D, MODE, TMA, MINB>;
+    auto kern = sat_band_kernel<T, R, W, S, D, NCW, MODE, TMA, MINB>;
     const size_t smem = BandSmem<T, R, W, S, D>::total;
-    const int threads = (W + 2) * 32;
+    const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
@@ -206,7 +207,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     return SAT_OK;
 }
 
-#define SAT_CFG(c) c.R, c.W, c.S, c.D
+#define SAT_CFG(c) c.R, c.W, c.S, c.D, c.NCW
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {
@@ -437,8 +438,21 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     switch (variant) {
         case SAT_1R1W: {
             BandParams p = base_params();
+            if (seed && seed_kind == SEED_COLSUM) {
+                // column sums above the strip -> the SAT row just above it
+                SAT_TRY(ensure(ws->seedrow, size_t(cols) * 4, false));
+                if (dtype == SAT_INT32)
+                    sat_row_prefix_kernel<uint32_t><<<1, 1024, 0, st>>>(
+                        static_cast<const uint32_t*>(seed), static_cast<uint32_t*>(ws->seedrow.p), cols);
+                else
+                    sat_row_prefix_kernel<float><<<1, 1024, 0, st>>>(
+                        static_cast<const float*>(seed), static_cast<float*>(ws->seedrow.p), cols);
+                CUDA_TRY(cudaGetLastError());
+                ++t_launches;
+                seed = ws->seedrow.p;
+            }
             p.seed = seed;
-            p.seed_kind = seed ? seed_kind : SEED_NONE;
+            p.seed_kind = seed ? SEED_SATROW : SEED_NONE;
             return run_band(j, MODE_SAT, in, out, p);
         }
         case SAT_2R2W: {

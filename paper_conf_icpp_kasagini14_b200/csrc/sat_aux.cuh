@@ -223,4 +223,41 @@ __global__ void sat_rank_exscan_kernel(const T* __restrict__ gathered, T* __rest
     carry[c] = s;
 }
 
+// sat_row[c] = sum_{c' <= c} carry[c'] : the SAT row just above a strip whose
+// column sums above are `carry` (seeded mode).  One CTA of 1024 threads walks
+// the row in tiles of 8192 elements with a running carry.
+template <typename T>
+__global__ void __launch_bounds__(1024)
+sat_row_prefix_kernel(const T* __restrict__ carry, T* __restrict__ sat_row, int64_t cols)
+{
+    __shared__ T wsum[32];
+    __shared__ T s_run;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) s_run = T(0);
+    __syncthreads();
+    for (int64_t base = 0; base < cols; base += 8 * 1024) {
+        const int64_t c = base + int64_t(threadIdx.x) * 8;
+        T e[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) e[i] = (c + i < cols) ? carry[c + i] : T(0);
+#pragma unroll
+        for (int i = 1; i < 8; ++i) e[i] += e[i - 1];
+        const T inc = warp_inclusive_scan(e[7], lane);
+        if (lane == 31) wsum[warp] = inc;
+        __syncthreads();
+        if (warp == 0) {
+            const T w = warp_inclusive_scan(wsum[lane], lane);
+            wsum[lane] = w;
+        }
+        __syncthreads();
+        const T off = s_run + (warp > 0 ? wsum[warp - 1] : T(0)) + (inc - e[7]);
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+            if (c + i < cols) sat_row[c + i] = e[i] + off;
+        __syncthreads();
+        if (threadIdx.x == 0) s_run += wsum[31];
+        __syncthreads();
+    }
+}
+
 }  // namespace sat

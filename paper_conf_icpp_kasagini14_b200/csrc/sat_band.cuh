@@ -29,8 +29,10 @@
 // of 2R2W, Step 3 of 2R1W with external carries
 // and the 1R1W band (C) of (1+r)R1W.
 //
-// Roles (warps): 0..W-1 compute (R rows each), W = control (descriptors,
-// look-back), W+1 = producer (TMA loads and stores, one elected lane).
+// Roles (warps): 0..W-1 compute (R rows each), W..W+NCW-1 control
+// (descriptors and look-back; control warp c owns the chunks k = c mod NCW,
+// so NCW look-backs are in flight at once), W+NCW = producer (TMA loads and
+// stores, one elected lane).
 #pragma once
 #include "sat_common.h"
 #include "sat_device.cuh"
@@ -113,15 +115,15 @@ __device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
     }
 }
 
-template <typename T, int R, int W, int S, int D, int MODE, bool TMA, int MINB>
-__global__ void __launch_bounds__((W + 2) * 32, MINB)
+template <typename T, int R, int W, int S, int D, int NCW, int MODE, bool TMA, int MINB>
+__global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const __grid_constant__ CUtensorMap tm_out,
                 const BandParams p)
 {
     constexpr int TH = R * W;
-    constexpr int CW = W;          // control warp
-    constexpr int PW = W + 1;      // producer warp
+    constexpr int CW = W;          // first control warp
+    constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
     using SM = BandSmem<T, R, W, S, D>;
     constexpr int XS = SM::XS;
@@ -156,7 +158,6 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     const int desc_w = p.nc * TW;
     const int64_t lx_stride = int64_t(p.total_bands) * TH;
     uint32_t g = 0;                              // CTA-local chunk counter (ring position)
-    T seedrun = T(0);                            // control warp: running seed prefix
 
     for (;;) {
         if (threadIdx.x == 0)
@@ -300,15 +301,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                 for (int r = 0; r < R; ++r) lb[r] = L[r];
             }
-        } else if (warp == CW) {
+        } else if (warp < PW) {
             // ================= control warp: descriptors + look-back =================
             if constexpr (MODE != MODE_ROW) {
                 const uint32_t tagbase = band_tag(p.base, gb);
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
                 const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
-                if (band == 0) seedrun = T(0);
-                for (int k = 0; k < nch; ++k) {
+                for (int k = warp - CW; k < nch; k += NCW) {
                     const uint32_t it = g + k;
                     const int s = it % S;
                     const uint32_t ph = (it / S) & 1;
@@ -334,21 +334,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         top = lds4<T>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0);
                     } else if (band == 0) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
+                            // the SAT row just above the matrix (sat_api.cu turns a
+                            // column-sum seed into this row first)
                             const T* sd = reinterpret_cast<const T*>(p.seed);
                             T e[4];
 #pragma unroll
                             for (int i = 0; i < 4; ++i) e[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
-                            if (p.seed_kind == SEED_COLSUM && MODE == MODE_SAT) {
-                                // SAT row above = row prefix of the column sums above
-                                e[1] += e[0]; e[2] += e[1]; e[3] += e[2];
-                                const T inc = warp_inclusive_scan(e[3], lane);
-                                T exc = __shfl_up_sync(0xffffffffu, inc, 1);
-                                if (lane == 0) exc = T(0);
-                                const T off = seedrun + exc;
-#pragma unroll
-                                for (int i = 0; i < 4; ++i) e[i] += off;
-                                seedrun += __shfl_sync(0xffffffffu, inc, 31);
-                            }
                             top = V4<T>{e[0], e[1], e[2], e[3]};
                         }
                     } else {

@@ -16,7 +16,7 @@ constexpr int TW = 128;          // chunk width: 32 lanes x 4 elements (16 B)
 enum Mode { MODE_COL = 1, MODE_ROW = 2, MODE_SAT = 3 };
 enum TopSrc { TOP_LOOKBACK = 0, TOP_EXTERNAL = 1 };
 enum Region { REG_ALL = 0, REG_A = 1, REG_C = 2, REG_B = 3 };
-enum SeedKind { SEED_NONE = 0, SEED_COLSUM = 1, SEED_SATROW = 2 };
+enum SeedKind { SEED_NONE = 0, SEED_COLSUM = 1, SEED_SATROW = 2 };  // the kernel sees NONE/SATROW
 
 // Tile (I = band, J = chunk) regions of (1+r)R1W, bounded by tile
 // anti-diagonals (reading R10; Fig. 12):
@@ -48,8 +48,8 @@ struct BandParams {
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)
-    const void* seed;          // [cols] seed row (band 0 of image 0), nullable
-    int seed_kind;             // SeedKind
+    const void* seed;          // [cols] SAT row above band 0 of image 0, nullable
+    int seed_kind;             // SEED_NONE or SEED_SATROW
     int top_src;               // TopSrc
     int region;                // Region
     int tA;                    // (1+r)R1W threshold
