@@ -164,11 +164,13 @@ int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t 
                      int dtype, int variant, void *stream);
 
 /* Debug/profiling: the next 1R1W-family band launch on this thread records,
- * per (band, chunk) of TH x 128 elements, four 64-bit globaltimer stamps
- * (ns) into dev_buf[(band*nchunks + chunk)*4 + e]: e=0 tile data arrived,
+ * per (band, chunk) of TH x 128 elements, eight 64-bit globaltimer stamps
+ * (ns) into dev_buf[(band*nchunks + chunk)*8 + e]: e=0 tile data arrived,
  * e=1 band-local reductions done, e=2 look-back done (bits 48..63 = number
- * of look-back hops), e=3 tile store issued.  dev_buf (device, caller-owned)
- * must hold ceil(rows/TH)*batch*ceil(cols/128)*32 bytes; NULL disarms. */
+ * of look-back hops), e=3 tile store issued, e=4 tile load issued, e=5 the
+ * store's smem read completed, e=6 add vectors ready (finish starts), e=7
+ * unused.  dev_buf (device, caller-owned) must hold
+ * ceil(rows/TH)*batch*ceil(cols/128)*64 bytes; NULL disarms. */
 int sat_debug_trace(void *dev_buf);
 
 /* Number of kernels launched by the last successful call on this thread. */

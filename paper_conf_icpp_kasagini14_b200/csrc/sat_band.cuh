@@ -208,7 +208,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 if constexpr (TMA) {
                     mbar_wait(&full[s], ph);
                     if (p.trace && warp == 0 && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 4 + 0] = globaltimer();
+                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
                 } else {
@@ -259,6 +259,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const int s = it % S;
                 const uint32_t ph = (it / S) & 1;
                 mbar_wait(&topr[s], ph);
+                if (p.trace && warp == 0 && lane == 0)
+                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
                 const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
                 T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
                 if constexpr (TMA) {
@@ -317,7 +319,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     T* xb = xbuf + size_t(it % XS) * W * TW + 4 * lane;
                     mbar_wait(&colr[s], ph);
                     if (p.trace && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 1] = globaltimer();
+                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
                     V4<T> agg = lds4<T>(xb);
 #pragma unroll
                     for (int w2 = 1; w2 < W; ++w2) add4(agg, lds4<T>(xb + w2 * TW));
@@ -404,7 +406,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         publish4<T>(my, tagbase | 2u, inc);
                     }
                     if (p.trace && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 4 + 2] =
+                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
                             (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
                     // add vectors for finish(): top + bottom rows of the warps above
                     V4<T> run = top;
@@ -426,6 +428,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     auto load = [&](int k) {
                         const uint32_t it = g + k;
                         const int s = it % S;
+                        if (p.trace)
+                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 4] = globaltimer();
                         mbar_arrive_expect_tx(&full[s], TILE_BYTES);
                         tma_load_3d(tiles + size_t(s) * SM::tile_elems, &tm_in, &full[s],
                                     (j0 + k) * TW, row0, img, pol);
@@ -438,10 +442,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         const uint32_t ph = (it / S) & 1;
                         mbar_wait(&done[s], ph);
                         if (p.trace)
-                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 4 + 3] = globaltimer();
+                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
                         tma_store_3d(&tm_out, tiles + size_t(s) * SM::tile_elems, (j0 + k) * TW, row0, img, pol);
                         bulk_commit();
-                        if (k + S < nch) { bulk_wait_read<0>(); load(k + S); }
+                        if (k + S < nch) {
+                            bulk_wait_read<0>();
+                            if (p.trace)
+                                p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 5] = globaltimer();
+                            load(k + S);
+                        }
                     }
                 }
             }

@@ -19,7 +19,7 @@ y = torch.empty_like(x)
 for _ in range(3):
     libsat.sat(x, out=y, tile_rows=th)
 nb, nc = (rows + th - 1) // th, (cols + 127) // 128
-buf = torch.zeros(nb * nc * 4, dtype=torch.int64, device="cuda")
+buf = torch.zeros(nb * nc * 8, dtype=torch.int64, device="cuda")
 torch.cuda.synchronize()
 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 libsat.debug_trace(buf)
@@ -28,4 +28,4 @@ libsat.sat(x, out=y, tile_rows=th)
 e.record()
 torch.cuda.synchronize()
 print("ms", s.elapsed_time(e), "th", libsat.last_tile_rows())
-np.savez_compressed(out, trace=buf.cpu().numpy().reshape(nb, nc, 4), ms=s.elapsed_time(e))
+np.savez_compressed(out, trace=buf.cpu().numpy().reshape(nb, nc, 8), ms=s.elapsed_time(e))
