@@ -68,7 +68,7 @@ struct BandSmem {
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
-constexpr int LBW = 4;   // look-back window: bands read per round trip
+constexpr int LBW = 8;   // look-back window: bands read per round trip
 
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
     return uint32_t((base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
@@ -199,14 +199,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 
             // local(k): row scans with L, column prefix down this warp's rows,
             // result back into the slot, warp bottom row into xbuf
-            auto local = [&](int k) {
+            auto local = [&](int k, bool landed) {
                 const uint32_t it = g + k;
                 const int s = it % S;
                 const uint32_t ph = (it / S) & 1;
                 T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
                 V4<T> v[R];
                 if constexpr (TMA) {
-                    mbar_wait(&full[s], ph);
+                    if (!landed) mbar_wait(&full[s], ph);
                     if (p.trace && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
 #pragma unroll
@@ -290,13 +290,29 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             };
 
             if constexpr (MODE == MODE_ROW) {
-                for (int k = 0; k < nch; ++k) local(k);
+                for (int k = 0; k < nch; ++k) local(k, false);
             } else {
-                for (int k = 0; k < nch; ++k) {
-                    local(k);
-                    if (k >= D) finish(k - D);
+                // whichever is ready first: finish the oldest chunk whose add
+                // vectors are published, or start local() on the next chunk
+                // that has landed (at most D chunks ahead of the oldest
+                // unfinished one: xbuf holds D+1 chunks)
+                int nl = 0, nf = 0;
+                while (nf < nch) {
+                    if (nf < nl) {
+                        const uint32_t it = g + nf;
+                        if (mbar_try_wait(&topr[it % S], (it / S) & 1)) { finish(nf); ++nf; continue; }
+                    }
+                    if (nl < nch && nl <= nf + D) {
+                        if constexpr (TMA) {
+                            const uint32_t it = g + nl;
+                            if (mbar_try_wait(&full[it % S], (it / S) & 1)) { local(nl, true); ++nl; continue; }
+                        } else {
+                            local(nl, true);
+                            ++nl;
+                            continue;
+                        }
+                    }
                 }
-                for (int k = (nch > D ? nch - D : 0); k < nch; ++k) finish(k);
             }
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;
