@@ -176,19 +176,19 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
 
 // ------------------------------------------------------------------ band kernel dispatch
 struct BandCfg {
-    int R, W, S, D, NCW, MINB;
+    int R, W, S, NCW, MINB;
 };
 // TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
-// (D+1)*W*512 (warp bottom rows / add vectors) + barriers.
-constexpr BandCfg kCfg16{2, 8, 8, 3, 3, 2};
-constexpr BandCfg kCfg32{4, 8, 6, 3, 3, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 1, 2, 2};
+// S*W*512 (warp bottom rows) + barriers.
+constexpr BandCfg kCfg16{2, 8, 8, 4, 2};
+constexpr BandCfg kCfg32{4, 8, 5, 4, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 4, 2};
 
-template <typename T, int R, int W, int S, int D, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int NCW, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, D, NCW, MODE, TMA, MINB>;
-    const size_t smem = BandSmem<T, R, W, S, D>::total;
+    auto kern = sat_band_kernel<T, R, W, S, NCW, MODE, TMA, MINB>;
+    const size_t smem = BandSmem<T, R, W, S>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
@@ -207,7 +207,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     return SAT_OK;
 }
 
-#define SAT_CFG(c) c.R, c.W, c.S, c.D, c.NCW
+#define SAT_CFG(c) c.R, c.W, c.S, c.NCW
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {

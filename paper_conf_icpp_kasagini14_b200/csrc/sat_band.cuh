@@ -18,12 +18,12 @@
 //     SAT bottom row as "inclusive".  The look-back reads a
 //     window of LBW bands per round trip;
 //   * inside a chunk, Step 3-1/3-2 of 2R1W become two passes over
-//     the smem slot: local() = row scans with L + column prefix down the
-//     warp's R rows (written back in place; the warp's bottom row goes to
-//     xbuf); finish() = + (SAT row above the band + bottom rows of the warps
-//     above), computed by the control warp.  finish(k) runs D chunks after
-//     local(k), so the look-back latency of chunk k overlaps the local work
-//     of chunks k+1..k+D.
+//     the smem slot: the compute warps' local() = row scans with L + column
+//     prefix down the warp's R rows (written back in place; the warp's bottom
+//     row goes to xbuf); the control warp's finish = + (SAT row above the
+//     band + bottom rows of the warps above).  The compute warps never wait
+//     for a look-back: they run ahead as far as the S-slot ring allows, and
+//     NCW control warps keep NCW look-backs (and finishes) in flight.
 //
 // The same kernel, with MODE/TopSrc switches, is the column pass and row pass
 // of 2R2W, Step 3 of 2R1W with external carries
@@ -57,10 +57,10 @@ __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int D>
+template <typename T, int R, int W, int S>
 struct BandSmem {
     static constexpr int TH = R * W;
-    static constexpr int XS = D + 1;                 // xbuf slots
+    static constexpr int XS = S;                     // xbuf slots (one per ring slot)
     static constexpr size_t tile_elems = size_t(TH) * TW;
     static constexpr size_t tiles = S * tile_elems * sizeof(T);
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
@@ -68,7 +68,7 @@ struct BandSmem {
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
-constexpr int LBW = 8;   // look-back window: bands read per round trip
+constexpr int LBW = 4;   // look-back window: bands read per round trip
 
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
     return uint32_t((base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
@@ -115,7 +115,7 @@ __device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
     }
 }
 
-template <typename T, int R, int W, int S, int D, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int NCW, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const __grid_constant__ CUtensorMap tm_out,
@@ -125,9 +125,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S, D>;
+    using SM = BandSmem<T, R, W, S>;
     constexpr int XS = SM::XS;
-    static_assert(S >= D + 2, "ring must hold D finished-pending chunks plus a prefetch");
 
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
@@ -135,8 +134,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf);
     uint64_t* full = bars;          // TMA load landed (tx count)
     uint64_t* colr = bars + S;      // every compute warp finished local()
-    uint64_t* topr = bars + 2 * S;  // control warp wrote the add vectors
-    uint64_t* done = bars + 3 * S;  // every compute warp finished finish()
+    uint64_t* done = bars + 3 * S;  // the slot holds final values (control warp / row pass)
     long long* s_unit = reinterpret_cast<long long*>(bars + 4 * S);
 
     const int warp = threadIdx.x >> 5;
@@ -146,8 +144,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&colr[s], W * 32);
-            mbar_init(&topr[s], 32);
-            mbar_init(&done[s], W * 32);
+            mbar_init(&done[s], MODE == MODE_ROW ? W * 32 : 32);
         }
         fence_mbar_init();
     }
@@ -199,14 +196,18 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 
             // local(k): row scans with L, column prefix down this warp's rows,
             // result back into the slot, warp bottom row into xbuf
-            auto local = [&](int k, bool landed) {
+            auto local = [&](int k) {
                 const uint32_t it = g + k;
                 const int s = it % S;
                 const uint32_t ph = (it / S) & 1;
                 T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
                 V4<T> v[R];
+                if constexpr (!TMA) {
+                    // the slot is free once the control warp finished chunk it-S
+                    if (it >= uint32_t(S)) mbar_wait(&done[s], ph ^ 1u);
+                }
                 if constexpr (TMA) {
-                    if (!landed) mbar_wait(&full[s], ph);
+                    mbar_wait(&full[s], ph);
                     if (p.trace && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
 #pragma unroll
@@ -253,67 +254,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     mbar_arrive(&colr[s]);
                 }
             };
-            // finish(k): + (SAT row above + bottom rows of the warps above), store
-            auto finish = [&](int k) {
-                const uint32_t it = g + k;
-                const int s = it % S;
-                const uint32_t ph = (it / S) & 1;
-                mbar_wait(&topr[s], ph);
-                if (p.trace && warp == 0 && lane == 0)
-                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
-                const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
-                T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
-                if constexpr (TMA) {
-#pragma unroll
-                    for (int r = 0; r < R; ++r) {
-                        V4<T> v = lds4<T>(t + r * TW);
-                        add4(v, add);
-                        sts4(t + r * TW, v);
-                    }
-                    fence_proxy_async_smem();
-                } else {
-                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
-#pragma unroll
-                    for (int r = 0; r < R; ++r) {
-                        V4<T> v = lds4<T>(t + r * TW);
-                        add4(v, add);
-                        const int64_t row = row0 + rbase + r;
-                        if (row < p.rows) {
-                            const T e[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-                            for (int i = 0; i < 4; ++i)
-                                if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
-                        }
-                    }
-                }
-                mbar_arrive(&done[s]);
-            };
-
-            if constexpr (MODE == MODE_ROW) {
-                for (int k = 0; k < nch; ++k) local(k, false);
-            } else {
-                // whichever is ready first: finish the oldest chunk whose add
-                // vectors are published, or start local() on the next chunk
-                // that has landed (at most D chunks ahead of the oldest
-                // unfinished one: xbuf holds D+1 chunks)
-                int nl = 0, nf = 0;
-                while (nf < nch) {
-                    if (nf < nl) {
-                        const uint32_t it = g + nf;
-                        if (mbar_try_wait(&topr[it % S], (it / S) & 1)) { finish(nf); ++nf; continue; }
-                    }
-                    if (nl < nch && nl <= nf + D) {
-                        if constexpr (TMA) {
-                            const uint32_t it = g + nl;
-                            if (mbar_try_wait(&full[it % S], (it / S) & 1)) { local(nl, true); ++nl; continue; }
-                        } else {
-                            local(nl, true);
-                            ++nl;
-                            continue;
-                        }
-                    }
-                }
-            }
+            for (int k = 0; k < nch; ++k) local(k);
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;
 #pragma unroll
@@ -424,15 +365,39 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
                             (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
-                    // add vectors for finish(): top + bottom rows of the warps above
+                    // finish: + (SAT row above the band + bottom rows of the
+                    // warps above); the slot then holds final values
+                    if (p.trace && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 6] = globaltimer();
+                    T* t = tiles + size_t(s) * SM::tile_elems + 4 * lane;
+                    const int64_t cg = int64_t(J) * TW + 4 * lane;
+                    T* go = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
                     V4<T> run = top;
-#pragma unroll
+#pragma unroll 1
                     for (int w2 = 0; w2 < W; ++w2) {
                         const V4<T> b = lds4<T>(xb + w2 * TW);
-                        sts4(xb + w2 * TW, run);
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            T* tr = t + (w2 * R + r) * TW;
+                            V4<T> v = lds4<T>(tr);
+                            add4(v, run);
+                            if constexpr (TMA) {
+                                sts4(tr, v);
+                            } else {
+                                const int64_t row = row0 + w2 * R + r;
+                                if (row < p.rows) {
+                                    const T e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                                    for (int i = 0; i < 4; ++i)
+                                        if (cg + i < p.cols) go[row * p.cols + cg + i] = e[i];
+                                }
+                            }
+                        }
                         add4(run, b);
                     }
-                    mbar_arrive(&topr[s]);
+                    if constexpr (TMA) fence_proxy_async_smem();
+                    __syncwarp();
+                    mbar_arrive(&done[s]);
                 }
             }
         } else {

@@ -31,8 +31,8 @@ ld = t[:, :, 0] - t[:, :, 4]
 print("load issue->arrival med %.2f p90 %.2f" % (np.median(ld[t[:, :, 4] > -1e8]), np.percentile(ld, 90)))
 srd = t[:, :-3, 5] - t[:, :-3, 3]
 print("store issue->smem read done med %.2f p90 %.2f" % (np.median(srd), np.percentile(srd, 90)))
-fw = t[:, :, 6] - t[:, :, 2]
-print("lookback done->finish start med %.2f ; local done(ctrl seen)->finish start med %.2f" % (np.median(fw), np.median(t[:, :, 6] - t[:, :, 1])))
+fw = t[:, :, 3] - t[:, :, 6]
+print("finish start->store issue med %.2f" % np.median(fw))
 b0 = t[0]
 print("band0: period %.2f, load lat %.2f, arr->colr %.2f, colr->lb %.2f, lb->fin %.2f, fin->store %.2f" % (
     np.median(np.diff(b0[:, 0])), np.median(b0[:, 0] - b0[:, 4]), np.median(b0[:, 1] - b0[:, 0]),
