@@ -82,7 +82,7 @@ typedef struct sat_options {
     double r;            /* SAT_1PLUSR_R1W: target fraction of tiles done by 2R1W
                             (0..1, default 0.25); the realised value is the tile
                             count ratio, see sat_last_r_effective() */
-    int tile_rows;       /* band height TH in {16, 32, 64}; 0 = automatic */
+    int tile_rows;       /* band height TH in {16, 32, 48, 64}; 0 = automatic */
     int force_generic;   /* 1 = use the non-TMA load/store path (tests) */
     int jitter;          /* debug: random delay (ns) before descriptor
                             publication, to stress the look-back; 0 = off */
@@ -166,10 +166,10 @@ int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t 
 /* Debug/profiling: the next 1R1W-family band launch on this thread records,
  * per (band, chunk) of TH x 128 elements, eight 64-bit globaltimer stamps
  * (ns) into dev_buf[(band*nchunks + chunk)*8 + e]: e=0 tile data arrived,
- * e=1 band-local reductions done, e=2 look-back done (bits 48..63 = number
- * of look-back hops), e=3 tile store issued, e=4 tile load issued, e=5 the
- * store's smem read completed, e=6 add vectors ready (finish starts), e=7
- * unused.  dev_buf (device, caller-owned) must hold
+ * e=1 band-local reductions done, e=2 look-back done (bits 48..55 = look-
+ * back hops, 56..63 = polls of unpublished descriptors), e=3 tile store
+ * issued, e=4 tile load issued, e=5 the store's smem read completed, e=6
+ * finish (carry injection) starts, e=7 unused.  dev_buf (device, caller-owned) must hold
  * ceil(rows/TH)*batch*ceil(cols/128)*64 bytes; NULL disarms. */
 int sat_debug_trace(void *dev_buf);
 

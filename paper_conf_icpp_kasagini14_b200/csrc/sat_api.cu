@@ -181,8 +181,9 @@ struct BandCfg {
 // TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
 // S*W*512 (warp bottom rows) + barriers.
 constexpr BandCfg kCfg16{2, 8, 8, 4, 2};
-constexpr BandCfg kCfg32{4, 8, 5, 4, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 4, 2};
+constexpr BandCfg kCfg32{8, 4, 6, 4, 2};
+constexpr BandCfg kCfg48{8, 6, 4, 4, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 3, 2};
 
 template <typename T, int R, int W, int S, int NCW, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
@@ -214,9 +215,10 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
     switch (th) {
         case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
         case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
+        case 48: return launch_band_t<T, SAT_CFG(kCfg48), MODE, TMA, kCfg48.MINB>(p, ti, to, di, st, grid);
         case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
     }
-    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32 or 64");
+    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48 or 64");
 }
 
 template <typename T, int MODE>
@@ -417,8 +419,9 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     sat_options o;
     sat_options_init(&o);
     if (opt) o = *opt;
-    if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 64)
-        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32 or 64");
+    if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 48 &&
+        o.tile_rows != 64)
+        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48 or 64");
     if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     int dev;

@@ -127,6 +127,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
     using SM = BandSmem<T, R, W, S>;
     constexpr int XS = SM::XS;
+    // A control warp waits on colr[] of chunk k only after finishing chunk
+    // k-NCW, which implies local(k-S) completed iff NCW <= S; otherwise the
+    // parity wait could pass on a stale phase.
+    static_assert(NCW <= S, "more control warps than ring slots");
 
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
@@ -288,7 +292,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     }
                     if (publish && band > 0) publish4<T>(my, tagbase | 1u, agg);
                     V4<T> top{T(0), T(0), T(0), T(0)};
-                    unsigned long long hops = 0;
+                    unsigned long long hops = 0, polls = 0;
                     if (!lookback) {
                         top = lds4<T>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0);
                     } else if (band == 0) {
@@ -307,6 +311,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         T acc[4] = {T(0), T(0), T(0), T(0)};
                         uint32_t pend = 0xFu;
                         int kb = band - 1;
+                        SpinGuard guard;
                         while (pend) {
                             uint64_t wv[LBW][4];
 #pragma unroll
@@ -352,7 +357,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                 }
                                 ++hops;
                             }
-                            if (stalled) __nanosleep(32);
+                            if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
                             else kb -= LBW;
                         }
                         top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
@@ -364,7 +369,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     }
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
-                            (globaltimer() & 0xFFFFFFFFFFFFull) | (hops << 48);
+                            (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
                     // finish: + (SAT row above the band + bottom rows of the
                     // warps above); the slot then holds final values
                     if (p.trace && lane == 0)
@@ -376,17 +381,19 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll 1
                     for (int w2 = 0; w2 < W; ++w2) {
                         const V4<T> b = lds4<T>(xb + w2 * TW);
+                        T* tr = t + (w2 * R) * TW;
+                        V4<T> v[R];
+#pragma unroll
+                        for (int r = 0; r < R; ++r) v[r] = lds4<T>(tr + r * TW);   // loads first (ILP)
 #pragma unroll
                         for (int r = 0; r < R; ++r) {
-                            T* tr = t + (w2 * R + r) * TW;
-                            V4<T> v = lds4<T>(tr);
-                            add4(v, run);
+                            add4(v[r], run);
                             if constexpr (TMA) {
-                                sts4(tr, v);
+                                sts4(tr + r * TW, v[r]);
                             } else {
                                 const int64_t row = row0 + w2 * R + r;
                                 if (row < p.rows) {
-                                    const T e[4] = {v.x, v.y, v.z, v.w};
+                                    const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
 #pragma unroll
                                     for (int i = 0; i < 4; ++i)
                                         if (cg + i < p.cols) go[row * p.cols + cg + i] = e[i];

@@ -37,8 +37,33 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
                  : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
     return ok != 0;
 }
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Watchdog for every spin in libsat: a wait that exceeds kSpinLimitNs is a
+// protocol bug (no legitimate wait lasts that long), so the kernel traps and
+// the call surfaces as SAT_ERR_CUDA instead of hanging the GPU.
+constexpr unsigned long long kSpinLimitNs = 4000000000ull;   // 4 s
+
+struct SpinGuard {
+    unsigned long long t0 = 0;
+    unsigned n = 0;
+    __device__ __forceinline__ void tick() {
+        if ((++n & 1023u) == 0) {
+            const unsigned long long t = globaltimer_ns();
+            if (t0 == 0) t0 = t;
+            else if (t - t0 > kSpinLimitNs) __trap();
+        }
+    }
+};
+
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    while (!mbar_try_wait(bar, parity)) { }
+    if (mbar_try_wait(bar, parity)) return;
+    SpinGuard guard;
+    while (!mbar_try_wait(bar, parity)) guard.tick();
 }
 
 // ------------------------------------------------------------- TMA

@@ -54,7 +54,7 @@ def test_validation_without_gpu():
     assert L.sat_compute(None, None, 0, 5, 0, 2, None) == 0
     assert L.sat_compute(None, None, 5, 0, 1, 2, None) == 0
     # bad options
-    o = libsat.options(tile_rows=48)
+    o = libsat.options(tile_rows=40)
     assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 2, ctypes.byref(o), None) == -1
     o = libsat.options(r=1.5)
     assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 3, ctypes.byref(o), None) == -1

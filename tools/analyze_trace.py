@@ -6,7 +6,8 @@ import numpy as np
 d = np.load(sys.argv[1])
 t = d["trace"].astype(np.int64)
 nb, nc, _ = t.shape
-hops = (t[:, :, 2] >> 48) & 0xFFFF
+hops = (t[:, :, 2] >> 48) & 0xFF
+polls = (t[:, :, 2] >> 56) & 0xFF
 t &= (1 << 48) - 1
 lo = t[:, :, 0][t[:, :, 0] > 0].min()
 t = (t - lo) / 1000.0                          # us since first tile arrival
@@ -37,4 +38,7 @@ b0 = t[0]
 print("band0: period %.2f, load lat %.2f, arr->colr %.2f, colr->lb %.2f, lb->fin %.2f, fin->store %.2f" % (
     np.median(np.diff(b0[:, 0])), np.median(b0[:, 0] - b0[:, 4]), np.median(b0[:, 1] - b0[:, 0]),
     np.median(b0[:, 2] - b0[:, 1]), np.median(b0[:, 6] - b0[:, 2]), np.median(b0[:, 3] - b0[:, 6])))
-print("hops: mean %.2f max %d; share of chunks with hops>1: %.3f" % (hops.mean(), hops.max(), (hops > 1).mean()))
+print("hops: mean %.2f max %d; share of chunks with hops>1: %.3f; polls mean %.2f max %d" % (hops.mean(), hops.max(), (hops > 1).mean(), polls.mean(), polls.max()))
+bi = np.arange(nb)
+for q in (0, 1, 2, nb // 4, nb // 2, nb - 1):
+    print("  band %4d: lb med %.2f hops %.1f polls %.1f end %.1f" % (q, np.median(t[q, :, 2] - t[q, :, 1]), hops[q].mean(), polls[q].mean(), t[q, -1, 3]))
