@@ -176,20 +176,23 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
 
 // ------------------------------------------------------------------ band kernel dispatch
 struct BandCfg {
-    int R, W, S, NCW, MINB;
+    int R, W, S, DT, NCW, MINB;
 };
-// TH = R*W rows per band.  Shared memory per CTA: S*TH*128*4 (ring) +
-// S*W*512 (warp bottom rows) + barriers.
-constexpr BandCfg kCfg16{2, 8, 8, 4, 2};
-constexpr BandCfg kCfg32{8, 4, 6, 4, 2};
-constexpr BandCfg kCfg48{8, 6, 4, 4, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 3, 2};
+// TH = R*W rows per band, W compute warps of R rows.  Shared memory per CTA:
+// S*TH*512 B (TMA load ring) + DT*W*512 B (bottom rows / add vectors) +
+// barriers; TMEM per CTA: DT chunks x 4R words per compute thread
+// (DESIGN.md Sec. 4).  Two CTAs per SM.
+constexpr BandCfg kCfg16{2, 8, 6, 8, 4, 2};
+constexpr BandCfg kCfg32{4, 8, 4, 8, 4, 2};
+constexpr BandCfg kCfg48{8, 6, 3, 4, 4, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 4, 4, 2};
 
-template <typename T, int R, int W, int S, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int NCW, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, NCW, MODE, TMA, MINB>;
-    const size_t smem = BandSmem<T, R, W, S>::total;
+    (void)to;
+    auto kern = sat_band_kernel<T, R, W, S, DT, NCW, MODE, TMA, MINB>;
+    const size_t smem = BandSmem<T, R, W, S, DT>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
@@ -202,13 +205,13 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
     if (grid < 1) grid = 1;
     grid_out = int(grid);
-    kern<<<int(grid), threads, smem, st>>>(ti, to, p);
+    kern<<<int(grid), threads, smem, st>>>(ti, p);
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     return SAT_OK;
 }
 
-#define SAT_CFG(c) c.R, c.W, c.S, c.NCW
+#define SAT_CFG(c) c.R, c.W, c.S, c.DT, c.NCW
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {
@@ -302,7 +305,6 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     std::memset(&to, 0, sizeof(to));
     if (j.tma) {
         SAT_TRY(make_tmap(&ti, in, j.dtype, j.batch, j.rows, j.cols, j.th));
-        SAT_TRY(make_tmap(&to, out, j.dtype, j.batch, j.rows, j.cols, j.th));
     }
     int grid = 0;
     int s = (j.dtype == SAT_INT32)

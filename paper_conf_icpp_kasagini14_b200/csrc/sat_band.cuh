@@ -8,7 +8,8 @@
 // everything:
 //   * a CTA takes a band of TH rows (ticket order = band order, so every band
 //     it waits on is held by a running or finished CTA) and walks it left to
-//     right in TH x 128 chunks staged through an S-slot TMA ring in smem;
+//     right in TH x 128 chunks; a producer warp streams the chunks into an
+//     S-slot shared-memory ring with TMA (cp.async.bulk.tensor);
 //   * the horizontal carry (the paper's R) is the per-row running sum L held
 //     in registers by the warp that owns the row;
 //   * the vertical carry (the paper's C and S, i.e. the SAT row above the
@@ -17,13 +18,15 @@
 //     as an "aggregate", then -- once it knows the SAT row above -- the final
 //     SAT bottom row as "inclusive".  The look-back reads a
 //     window of LBW bands per round trip;
-//   * inside a chunk, Step 3-1/3-2 of 2R1W become two passes over
-//     the smem slot: the compute warps' local() = row scans with L + column
-//     prefix down the warp's R rows (written back in place; the warp's bottom
-//     row goes to xbuf); the control warp's finish = + (SAT row above the
-//     band + bottom rows of the warps above).  The compute warps never wait
-//     for a look-back: they run ahead as far as the S-slot ring allows, and
-//     NCW control warps keep NCW look-backs (and finishes) in flight.
+//   * inside a chunk, Step 3-1/3-2 of 2R1W become: the compute
+//     warps' local() = row scans with L + column prefix down the warp's R
+//     rows; the result is parked in tensor memory (tcgen05.st) and the smem
+//     slot is released at once; NCW control warps do the look-backs and turn
+//     the carries into one add vector per warp (SAT row above the band +
+//     bottom rows of the warps above); DT-1 chunks later the compute warp
+//     takes its values back (tcgen05.ld), adds, and writes them to HBM with
+//     coalesced 16-B stores.  The look-back latency is thus hidden by DT
+//     chunks parked in TMEM instead of occupying the smem ring.
 //
 // The same kernel, with MODE/TopSrc switches, is the column pass and row pass
 // of 2R2W, Step 3 of 2R1W with external carries
@@ -31,8 +34,8 @@
 //
 // Roles (warps): 0..W-1 compute (R rows each), W..W+NCW-1 control
 // (descriptors and look-back; control warp c owns the chunks k = c mod NCW,
-// so NCW look-backs are in flight at once), W+NCW = producer (TMA loads and
-// stores, one elected lane).
+// so NCW look-backs are in flight at once), W+NCW = producer (TMA loads, one
+// elected lane).
 #pragma once
 #include "sat_common.h"
 #include "sat_device.cuh"
@@ -51,20 +54,25 @@ template <typename T>
 __device__ __forceinline__ void sts4(T* p, const V4<T>& v) {
     *reinterpret_cast<uint4*>(p) = make_uint4(to_bits(v.x), to_bits(v.y), to_bits(v.z), to_bits(v.w));
 }
+// 16-B streaming store (evict-first: the SAT is not re-read by this kernel)
+template <typename T>
+__device__ __forceinline__ void st_global_v4(T* p, const V4<T>& v) {
+    __stcs(reinterpret_cast<uint4*>(p), make_uint4(to_bits(v.x), to_bits(v.y), to_bits(v.z), to_bits(v.w)));
+}
 template <typename T>
 __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
     a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S>
+template <typename T, int R, int W, int S, int DT>
 struct BandSmem {
     static constexpr int TH = R * W;
-    static constexpr int XS = S;                     // xbuf slots (one per ring slot)
+    static constexpr int XS = DT;                    // carry slots: one per parked chunk
     static constexpr size_t tile_elems = size_t(TH) * TW;
     static constexpr size_t tiles = S * tile_elems * sizeof(T);
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
-    static constexpr size_t bars = size_t(4) * S * sizeof(uint64_t) + 16;
+    static constexpr size_t bars = size_t(2 * S + 2 * XS) * sizeof(uint64_t) + 16;
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
@@ -115,31 +123,113 @@ __device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
     }
 }
 
-template <typename T, int R, int W, int S, int NCW, int MODE, bool TMA, int MINB>
+// ---------------------------------------------------------------- TMEM
+// The band-local results of a chunk wait for their look-back in tensor memory
+// (256 KB per SM, otherwise idle in a scan): each compute thread parks its
+// R x 4 values in its own TMEM lane with one tcgen05.st and takes them back
+// with one tcgen05.ld when the carries are known.  This keeps the look-back
+// latency out of the shared-memory ring, which then only has to cover the
+// HBM load latency.
+template <int N>
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const uint32_t (&r)[N]);
+template <int N>
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&r)[N]);
+
+template <>
+__device__ __forceinline__ void tmem_st<8>(uint32_t t, const uint32_t (&r)[8]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+                 :: "r"(t), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]),
+                    "r"(r[6]), "r"(r[7]) : "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_ld<8>(uint32_t t, uint32_t (&r)[8]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                   "=r"(r[6]), "=r"(r[7]) : "r"(t) : "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_st<16>(uint32_t t, const uint32_t (&r)[16]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,"
+                 "%9,%10,%11,%12,%13,%14,%15,%16};"
+                 :: "r"(t), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]),
+                    "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]),
+                    "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]) : "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_ld<16>(uint32_t t, uint32_t (&r)[16]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,"
+                 "%10,%11,%12,%13,%14,%15}, [%16];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                   "=r"(r[6]), "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]),
+                   "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]) : "r"(t) : "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_st<32>(uint32_t t, const uint32_t (&r)[32]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,"
+                 "%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,"
+                 "%27,%28,%29,%30,%31,%32};"
+                 :: "r"(t), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]),
+                    "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]),
+                    "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]),
+                    "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]),
+                    "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]), "r"(r[29]),
+                    "r"(r[30]), "r"(r[31]) : "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_ld<32>(uint32_t t, uint32_t (&r)[32]) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,"
+                 "%10,%11,%12,%13,%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,"
+                 "%28,%29,%30,%31}, [%32];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                   "=r"(r[6]), "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]),
+                   "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]),
+                   "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+                   "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]),
+                   "=r"(r[30]), "=r"(r[31]) : "r"(t) : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tmem_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// TMEM columns per CTA for W compute warps holding DT chunks of R x 4 words.
+template <int R, int W, int DT>
+struct TmemCols {
+    static constexpr int per_warp = DT * 4 * R;
+    static constexpr int need = per_warp * ((W + 3) / 4);       // warps w, w+4, .. share lanes
+    static constexpr int alloc = need <= 32 ? 32 : need <= 64 ? 64 : need <= 128 ? 128
+                                 : need <= 256 ? 256 : 512;
+    static_assert(need <= 512, "TMEM holds at most 512 columns");
+};
+
+template <typename T, int R, int W, int S, int DT, int NCW, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
-                const __grid_constant__ CUtensorMap tm_out,
                 const BandParams p)
 {
     constexpr int TH = R * W;
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S>;
+    using SM = BandSmem<T, R, W, S, DT>;
+    using TC = TmemCols<R, W, DT>;
     constexpr int XS = SM::XS;
+    constexpr bool HOLD = (MODE != MODE_ROW);    // chunks wait for a vertical carry
     // A control warp waits on colr[] of chunk k only after finishing chunk
-    // k-NCW, which implies local(k-S) completed iff NCW <= S; otherwise the
+    // k-NCW, which implies local(k-XS) completed iff NCW <= XS; otherwise the
     // parity wait could pass on a stale phase.
-    static_assert(NCW <= S, "more control warps than ring slots");
+    static_assert(NCW <= XS, "more control warps than carry slots");
 
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf);
-    uint64_t* full = bars;          // TMA load landed (tx count)
-    uint64_t* colr = bars + S;      // every compute warp finished local()
-    uint64_t* done = bars + 3 * S;  // the slot holds final values (control warp / row pass)
-    long long* s_unit = reinterpret_cast<long long*>(bars + 4 * S);
+    uint64_t* full = bars;              // [S]  TMA load landed (tx count)
+    uint64_t* empty = bars + S;         // [S]  every compute warp read the slot
+    uint64_t* colr = bars + 2 * S;      // [XS] every compute warp published its bottom row
+    uint64_t* topr = bars + 2 * S + XS; // [XS] the control warp wrote the add vectors
+    long long* s_unit = reinterpret_cast<long long*>(bars + 2 * S + 2 * XS);
+    uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 1);
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -147,13 +237,24 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&colr[s], W * 32);
-            mbar_init(&done[s], MODE == MODE_ROW ? W * 32 : 32);
+            mbar_init(&empty[s], W * 32);
+        }
+        for (int x = 0; x < XS; ++x) {
+            mbar_init(&colr[x], W * 32);
+            mbar_init(&topr[x], 32);
         }
         fence_mbar_init();
     }
-    if (TMA && warp == PW && lane == 0) { prefetch_tmap(&tm_in); prefetch_tmap(&tm_out); }
+    if (HOLD && warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_u32(s_tmem)), "r"(TC::alloc) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    if (TMA && warp == PW && lane == 0) prefetch_tmap(&tm_in);
+    tmem_fence_before();
     __syncthreads();
+    tmem_fence_after();
+    const uint32_t tmem_base = HOLD ? *s_tmem : 0u;
 
     const int64_t img_elems = p.rows * p.cols;
     const int desc_w = p.nc * TW;
@@ -197,25 +298,44 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             }
             const T* gin = reinterpret_cast<const T*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
+            // this warp's TMEM lanes (32*(warp%4) ..) and column range
+            const uint32_t tm_warp = tmem_base + ((uint32_t(32 * (warp & 3))) << 16)
+                                     + uint32_t((warp >> 2) * TC::per_warp);
 
-            // local(k): row scans with L, column prefix down this warp's rows,
-            // result back into the slot, warp bottom row into xbuf
+            // store R rows of 4 values to the output (16-B vectors on the TMA
+            // path, where cols % 4 == 0; guarded scalars otherwise)
+            auto store_rows = [&](const V4<T> (&v)[R], int k) {
+                const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const int64_t row = row0 + rbase + r;
+                    if (row < p.rows) {
+                        if constexpr (TMA) {
+                            if (c < p.cols) st_global_v4(gout + row * p.cols + c, v[r]);
+                        } else {
+                            const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+                            for (int i = 0; i < 4; ++i)
+                                if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
+                        }
+                    }
+                }
+            };
+
+            // local(k): row scans with L, column prefix down this warp's rows;
+            // park the result in TMEM, warp bottom row into xbuf
             auto local = [&](int k) {
                 const uint32_t it = g + k;
-                const int s = it % S;
-                const uint32_t ph = (it / S) & 1;
-                T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
                 V4<T> v[R];
-                if constexpr (!TMA) {
-                    // the slot is free once the control warp finished chunk it-S
-                    if (it >= uint32_t(S)) mbar_wait(&done[s], ph ^ 1u);
-                }
                 if constexpr (TMA) {
-                    mbar_wait(&full[s], ph);
+                    const int s = it % S;
+                    mbar_wait(&full[s], (it / S) & 1);
                     if (p.trace && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
+                    const T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
+                    mbar_arrive(&empty[s]);
                 } else {
                     const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
 #pragma unroll
@@ -229,56 +349,73 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     }
                 }
                 if constexpr (MODE != MODE_COL) row_scan<T, R>(v, L, lane);
-                if constexpr (MODE != MODE_ROW) {
+                if constexpr (!HOLD) {
+                    store_rows(v, k);                    // the row pass is final
+                } else {
 #pragma unroll
                     for (int r = 1; r < R; ++r) add4(v[r], v[r - 1]);
-                    sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
-                }
-                if constexpr (MODE == MODE_ROW && !TMA) {
-                    // the row pass is final: write straight out
-                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
+                    uint32_t u[4 * R];
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
-                        const int64_t row = row0 + rbase + r;
-                        if (row < p.rows) {
-                            const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
-#pragma unroll
-                            for (int i = 0; i < 4; ++i)
-                                if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
-                        }
+                        u[4 * r + 0] = to_bits(v[r].x); u[4 * r + 1] = to_bits(v[r].y);
+                        u[4 * r + 2] = to_bits(v[r].z); u[4 * r + 3] = to_bits(v[r].w);
                     }
-                } else {
-#pragma unroll
-                    for (int r = 0; r < R; ++r) sts4(t + r * TW, v[r]);
-                }
-                if constexpr (MODE == MODE_ROW) {
-                    if constexpr (TMA) fence_proxy_async_smem();
-                    mbar_arrive(&done[s]);
-                } else {
-                    mbar_arrive(&colr[s]);
+                    tmem_st<4 * R>(tm_warp + uint32_t((it % DT) * 4 * R), u);
+                    sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
+                    mbar_arrive(&colr[it % XS]);
                 }
             };
-            for (int k = 0; k < nch; ++k) local(k);
+            // finish(k): + (SAT row above the band + bottom rows of the warps
+            // above), from the add vector the control warp left in xbuf
+            auto finish = [&](int k) {
+                const uint32_t it = g + k;
+                mbar_wait(&topr[it % XS], (it / XS) & 1);
+                if (p.trace && warp == 0 && lane == 0)
+                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
+                const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
+                uint32_t u[4 * R];
+                tmem_wait_st();
+                tmem_ld<4 * R>(tm_warp + uint32_t((it % DT) * 4 * R), u);
+                tmem_wait_ld();
+                V4<T> v[R];
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    v[r] = V4<T>{from_bits<T>(u[4 * r]), from_bits<T>(u[4 * r + 1]),
+                                 from_bits<T>(u[4 * r + 2]), from_bits<T>(u[4 * r + 3])};
+                    add4(v[r], add);
+                }
+                store_rows(v, k);
+                if (p.trace && warp == 0 && lane == 0)
+                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
+            };
+
+            if constexpr (!HOLD) {
+                for (int k = 0; k < nch; ++k) local(k);
+            } else {
+                for (int k = 0; k < nch; ++k) {
+                    local(k);
+                    if (k >= DT - 1) finish(k - (DT - 1));
+                }
+                for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
+            }
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;
 #pragma unroll
                 for (int r = 0; r < R; ++r) lb[r] = L[r];
             }
         } else if (warp < PW) {
-            // ================= control warp: descriptors + look-back =================
-            if constexpr (MODE != MODE_ROW) {
+            // ================= control warps: descriptors + look-back =================
+            if constexpr (HOLD) {
                 const uint32_t tagbase = band_tag(p.base, gb);
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
                 const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
                 for (int k = warp - CW; k < nch; k += NCW) {
                     const uint32_t it = g + k;
-                    const int s = it % S;
-                    const uint32_t ph = (it / S) & 1;
                     const int J = j0 + k;
                     const int c0 = J * TW + 4 * lane;
                     T* xb = xbuf + size_t(it % XS) * W * TW + 4 * lane;
-                    mbar_wait(&colr[s], ph);
+                    mbar_wait(&colr[it % XS], (it / XS) & 1);
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
                     V4<T> agg = lds4<T>(xb);
@@ -370,75 +507,31 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
                             (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
-                    // finish: + (SAT row above the band + bottom rows of the
-                    // warps above); the slot then holds final values
-                    if (p.trace && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 6] = globaltimer();
-                    T* t = tiles + size_t(s) * SM::tile_elems + 4 * lane;
-                    const int64_t cg = int64_t(J) * TW + 4 * lane;
-                    T* go = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
+                    // add vectors for finish(): top + bottom rows of the warps above
                     V4<T> run = top;
-#pragma unroll 1
+#pragma unroll
                     for (int w2 = 0; w2 < W; ++w2) {
                         const V4<T> b = lds4<T>(xb + w2 * TW);
-                        T* tr = t + (w2 * R) * TW;
-                        V4<T> v[R];
-#pragma unroll
-                        for (int r = 0; r < R; ++r) v[r] = lds4<T>(tr + r * TW);   // loads first (ILP)
-#pragma unroll
-                        for (int r = 0; r < R; ++r) {
-                            add4(v[r], run);
-                            if constexpr (TMA) {
-                                sts4(tr + r * TW, v[r]);
-                            } else {
-                                const int64_t row = row0 + w2 * R + r;
-                                if (row < p.rows) {
-                                    const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
-#pragma unroll
-                                    for (int i = 0; i < 4; ++i)
-                                        if (cg + i < p.cols) go[row * p.cols + cg + i] = e[i];
-                                }
-                            }
-                        }
+                        sts4(xb + w2 * TW, run);
                         add4(run, b);
                     }
-                    if constexpr (TMA) fence_proxy_async_smem();
-                    __syncwarp();
-                    mbar_arrive(&done[s]);
+                    mbar_arrive(&topr[it % XS]);
                 }
             }
         } else {
-            // ================= producer warp: TMA ring =================
+            // ================= producer warp: TMA load ring =================
             if constexpr (TMA) {
-                if (lane == 0 && nch > 0) {
+                if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
-                    bulk_wait_read<0>();          // previous unit's stores done reading smem
-                    auto load = [&](int k) {
+                    for (int k = 0; k < nch; ++k) {
                         const uint32_t it = g + k;
                         const int s = it % S;
+                        if (it >= uint32_t(S)) mbar_wait(&empty[s], ((it / S) & 1) ^ 1u);
                         if (p.trace)
                             p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 4] = globaltimer();
                         mbar_arrive_expect_tx(&full[s], TILE_BYTES);
                         tma_load_3d(tiles + size_t(s) * SM::tile_elems, &tm_in, &full[s],
                                     (j0 + k) * TW, row0, img, pol);
-                    };
-                    const int pre = nch < S ? nch : S;
-                    for (int k = 0; k < pre; ++k) load(k);
-                    for (int k = 0; k < nch; ++k) {
-                        const uint32_t it = g + k;
-                        const int s = it % S;
-                        const uint32_t ph = (it / S) & 1;
-                        mbar_wait(&done[s], ph);
-                        if (p.trace)
-                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
-                        tma_store_3d(&tm_out, tiles + size_t(s) * SM::tile_elems, (j0 + k) * TW, row0, img, pol);
-                        bulk_commit();
-                        if (k + S < nch) {
-                            bulk_wait_read<0>();
-                            if (p.trace)
-                                p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 5] = globaltimer();
-                            load(k + S);
-                        }
                     }
                 }
             }
@@ -446,7 +539,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         g += nch;
         __syncthreads();
     }
-    if (TMA && warp == PW && lane == 0) bulk_wait<0>();
+    if (HOLD) {
+        tmem_fence_before();
+        __syncthreads();
+        tmem_fence_after();
+        if (warp == 0)
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;"
+                         :: "r"(tmem_base), "r"(TC::alloc) : "memory");
+    }
 }
 
 }  // namespace sat
