@@ -177,6 +177,8 @@ int sat_debug_trace(void *dev_buf);
 int sat_last_launch_count(void);
 /* Band height used by the last 1R1W-family call on this thread. */
 int sat_last_tile_rows(void);
+/* Grid size (persistent CTAs) of the last band-kernel launch on this thread. */
+int sat_last_grid(void);
 /* Realised r of the last SAT_1PLUSR_R1W call on this thread. */
 double sat_last_r_effective(void);
 

@@ -57,6 +57,7 @@ _SIGS = {
     "sat_debug_trace": ([_P], _I),
     "sat_last_launch_count": ([], _I),
     "sat_last_tile_rows": ([], _I),
+    "sat_last_grid": ([], _I),
     "sat_last_r_effective": ([], ctypes.c_double),
     "sat_strerror": ([_I], ctypes.c_char_p),
     "sat_last_error": ([], ctypes.c_char_p),
@@ -255,6 +256,10 @@ def last_launch_count() -> int:
 
 def last_tile_rows() -> int:
     return _lib.sat_last_tile_rows()
+
+
+def last_grid() -> int:
+    return _lib.sat_last_grid()
 
 
 def last_r_effective() -> float:

@@ -28,6 +28,7 @@ namespace {
 thread_local std::string t_err;
 thread_local int t_launches = 0;
 thread_local int t_th = 0;
+thread_local int t_grid = 0;
 thread_local double t_r = 0.0;
 thread_local unsigned long long* t_trace = nullptr;
 
@@ -205,6 +206,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
     if (grid < 1) grid = 1;
     grid_out = int(grid);
+    t_grid = int(grid);
     kern<<<int(grid), threads, smem, st>>>(ti, p);
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
@@ -772,6 +774,7 @@ int sat_debug_trace(void* dev_buf) {
 
 int sat_last_launch_count(void) { return t_launches; }
 int sat_last_tile_rows(void) { return t_th; }
+int sat_last_grid(void) { return t_grid; }
 double sat_last_r_effective(void) { return t_r; }
 
 const char* sat_strerror(int status) {

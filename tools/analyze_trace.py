@@ -30,12 +30,10 @@ print("inter-band lag of look-back completion (us): med %.2f p10 %.2f p90 %.2f" 
       (np.median(lag), np.percentile(lag, 10), np.percentile(lag, 90)))
 ld = t[:, :, 0] - t[:, :, 4]
 print("load issue->arrival med %.2f p90 %.2f" % (np.median(ld[t[:, :, 4] > -1e8]), np.percentile(ld, 90)))
-srd = t[:, :-3, 5] - t[:, :-3, 3]
-print("store issue->smem read done med %.2f p90 %.2f" % (np.median(srd), np.percentile(srd, 90)))
-fw = t[:, :, 3] - t[:, :, 6]
-print("finish start->store issue med %.2f" % np.median(fw))
+print("lookback done->finish start med %.2f | finish start->stores issued med %.2f | arrival->finish start (TMEM residency) med %.2f" % (
+    np.median(t[:, :, 6] - t[:, :, 2]), np.median(t[:, :, 3] - t[:, :, 6]), np.median(t[:, :, 6] - t[:, :, 0])))
 b0 = t[0]
-print("band0: period %.2f, load lat %.2f, arr->colr %.2f, colr->lb %.2f, lb->fin %.2f, fin->store %.2f" % (
+print("band0: period %.2f, load lat %.2f, arr->colr %.2f, colr->lb %.2f, lb->fin %.2f, fin->stores %.2f" % (
     np.median(np.diff(b0[:, 0])), np.median(b0[:, 0] - b0[:, 4]), np.median(b0[:, 1] - b0[:, 0]),
     np.median(b0[:, 2] - b0[:, 1]), np.median(b0[:, 6] - b0[:, 2]), np.median(b0[:, 3] - b0[:, 6])))
 print("hops: mean %.2f max %d; share of chunks with hops>1: %.3f; polls mean %.2f max %d" % (hops.mean(), hops.max(), (hops > 1).mean(), polls.mean(), polls.max()))
