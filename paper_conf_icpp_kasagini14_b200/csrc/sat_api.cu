@@ -11,6 +11,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -59,6 +60,7 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
 struct DevInfo {
     int sms = 0;
     int smem_optin = 0;
+    int smem_sm = 0;
     bool ok = false;
 };
 
@@ -73,6 +75,7 @@ int get_dev(int& dev, DevInfo& info) {
     if (!d.ok) {
         CUDA_TRY(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
         CUDA_TRY(cudaDeviceGetAttribute(&d.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+        CUDA_TRY(cudaDeviceGetAttribute(&d.smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
         d.ok = true;
     }
     if (!g_encode) {
@@ -198,11 +201,22 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                      int(cudaSharedmemCarveoutMaxShared)));
         configured = 1;
     }
-    int occ = 0;
-    CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, smem));
+    // Resident CTAs per SM, from the kernel's own resources.  (The runtime's
+    // occupancy query reports 1 for kernels that allocate tensor memory; two
+    // CTAs of ours fit: TC::alloc <= 256 columns of the SM's 512.)
+    cudaFuncAttributes fa;
+    CUDA_TRY(cudaFuncGetAttributes(&fa, kern));
+    const int warps = threads / 32;
+    const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
+    int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
+                        di.smem_sm / int(smem + fa.sharedSizeBytes + 1024),
+                        MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT>::alloc, 32});
     if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
+    if (const char* e = getenv("SAT_DEBUG_OCC")) occ = atoi(e);
     long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
     if (grid < 1) grid = 1;
     grid_out = int(grid);

@@ -27,5 +27,5 @@ s.record()
 libsat.sat(x, out=y, tile_rows=th)
 e.record()
 torch.cuda.synchronize()
-print("ms", s.elapsed_time(e), "th", libsat.last_tile_rows(), "grid", libsat.last_grid())
+print("ms", s.elapsed_time(e), "th", libsat.last_tile_rows(), "grid", libsat.last_grid(), "SAT_DEBUG_OCC", os.environ.get("SAT_DEBUG_OCC"))
 np.savez_compressed(out, trace=buf.cpu().numpy().reshape(nb, nc, 8), ms=s.elapsed_time(e))
