@@ -65,12 +65,13 @@ __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int DT>
+template <typename T, int R, int W, int S, int DT, int SUB>
 struct BandSmem {
     static constexpr int TH = R * W;
     static constexpr int XS = DT;                    // carry slots: one per parked chunk
-    static constexpr size_t tile_elems = size_t(TH) * TW;
-    static constexpr size_t tiles = S * tile_elems * sizeof(T);
+    static constexpr size_t tile_elems = size_t(TH) * TW;            // one 128-column chunk
+    static constexpr size_t slot_elems = tile_elems * SUB;           // one ring slot
+    static constexpr size_t tiles = S * slot_elems * sizeof(T);
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
     static constexpr size_t bars = size_t(2 * S + 2 * XS) * sizeof(uint64_t) + 16;
     static constexpr size_t total = tiles + xbuf + bars;
@@ -202,7 +203,7 @@ struct TmemCols {
     static_assert(need <= 512, "TMEM holds at most 512 columns");
 };
 
-template <typename T, int R, int W, int S, int DT, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -211,7 +212,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S, DT>;
+    using SM = BandSmem<T, R, W, S, DT, SUB>;
     using TC = TmemCols<R, W, DT>;
     constexpr int XS = SM::XS;
     constexpr bool HOLD = (MODE != MODE_ROW);    // chunks wait for a vertical carry
@@ -259,7 +260,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     const int64_t img_elems = p.rows * p.cols;
     const int desc_w = p.nc * TW;
     const int64_t lx_stride = int64_t(p.total_bands) * TH;
-    uint32_t g = 0;                              // CTA-local chunk counter (ring position)
+    uint32_t g = 0;                              // CTA-local chunk counter (carry / TMEM slots)
+    uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
 
     for (;;) {
         if (threadIdx.x == 0)
@@ -328,14 +330,16 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const uint32_t it = g + k;
                 V4<T> v[R];
                 if constexpr (TMA) {
-                    const int s = it % S;
-                    mbar_wait(&full[s], (it / S) & 1);
+                    const uint32_t q = gq + uint32_t(k / SUB);     // ring slot of chunk k
+                    const int s = q % S;
+                    if (k % SUB == 0) mbar_wait(&full[s], (q / S) & 1);
                     if (p.trace && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
-                    const T* t = tiles + size_t(s) * SM::tile_elems + size_t(rbase) * TW + 4 * lane;
+                    const T* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
+                                 + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
-                    mbar_arrive(&empty[s]);
+                    if (k % SUB == SUB - 1 || k == nch - 1) mbar_arrive(&empty[s]);
                 } else {
                     const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
 #pragma unroll
@@ -523,20 +527,23 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if constexpr (TMA) {
                 if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
-                    for (int k = 0; k < nch; ++k) {
-                        const uint32_t it = g + k;
-                        const int s = it % S;
-                        if (it >= uint32_t(S)) mbar_wait(&empty[s], ((it / S) & 1) ^ 1u);
+                    for (int k0 = 0; k0 < nch; k0 += SUB) {
+                        const uint32_t q = gq + uint32_t(k0 / SUB);
+                        const int s = q % S;
+                        const int nsub = nch - k0 < SUB ? nch - k0 : SUB;
+                        if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
                         if (p.trace)
-                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 4] = globaltimer();
-                        mbar_arrive_expect_tx(&full[s], TILE_BYTES);
-                        tma_load_3d(tiles + size_t(s) * SM::tile_elems, &tm_in, &full[s],
-                                    (j0 + k) * TW, row0, img, pol);
+                            p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();
+                        mbar_arrive_expect_tx(&full[s], TILE_BYTES * nsub);
+                        for (int j = 0; j < nsub; ++j)   // adjacent boxes: SUB*512 B per row
+                            tma_load_3d(tiles + size_t(s) * SM::slot_elems + size_t(j) * SM::tile_elems,
+                                        &tm_in, &full[s], (j0 + k0 + j) * TW, row0, img, pol);
                     }
                 }
             }
         }
         g += nch;
+        gq += uint32_t((nch + SUB - 1) / SUB);
         __syncthreads();
     }
     if (HOLD) {
