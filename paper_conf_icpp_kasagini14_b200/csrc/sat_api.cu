@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -232,6 +233,17 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {
+    if constexpr (MODE == MODE_SAT && TMA && std::is_same<T, uint32_t>::value) {
+        // debug: alternative TH=16 configurations (SAT_DEBUG_CFG=1|2)
+        if (const char* e = getenv("SAT_DEBUG_CFG")) {
+            if (th == 16 && atoi(e) == 1)
+                return launch_band_t<T, 4, 4, 3, 8, 1, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 16 && atoi(e) == 2)
+                return launch_band_t<T, 2, 8, 3, 8, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 16 && atoi(e) == 3)
+                return launch_band_t<T, 4, 4, 3, 4, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+        }
+    }
     switch (th) {
         case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
         case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);

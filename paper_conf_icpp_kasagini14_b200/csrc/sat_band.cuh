@@ -339,7 +339,19 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                  + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
-                    if (k % SUB == SUB - 1 || k == nch - 1) mbar_arrive(&empty[s]);
+                    if (k % SUB == SUB - 1 || k == nch - 1) {
+                        // release the slot to the next TMA write only once the
+                        // generic-proxy reads have landed in registers (the
+                        // asm consumes them) and are ordered before the async
+                        // proxy: without this, a quick refill overtook the LDS
+                        // (seen as corrupted rows with 4 compute warps)
+#pragma unroll
+                        for (int r = 0; r < R; ++r)
+                            asm volatile("" :: "r"(to_bits(v[r].x)), "r"(to_bits(v[r].y)),
+                                         "r"(to_bits(v[r].z)), "r"(to_bits(v[r].w)));
+                        fence_proxy_async_smem();
+                        mbar_arrive(&empty[s]);
+                    }
                 } else {
                     const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
 #pragma unroll
