@@ -313,10 +313,8 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         t_trace = nullptr;
     }
     Workspace& ws = *j.ws;
-    const size_t plane = size_t(p.total_bands) * size_t(p.nc) * TW;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
-        // two value planes (aggregate, inclusive) + one flag per (band, chunk)
-        const size_t need = (2 * plane + size_t(p.total_bands) * size_t(p.nc)) * sizeof(uint32_t);
+        const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t);
         SAT_TRY(ensure(ws.desc, need, true));
     }
     SAT_TRY(ensure(ws.ticket, sizeof(unsigned long long), true));
@@ -328,9 +326,7 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         CUDA_TRY(cudaMemsetAsync(ws.ticket.p, 0, sizeof(unsigned long long), j.st));
         ws.next_base = 0;
     }
-    p.dval = static_cast<uint32_t*>(ws.desc.p);
-    p.dflag = p.dval ? p.dval + 2 * plane : nullptr;
-    p.dplane = int64_t(plane);
+    p.desc = static_cast<uint64_t*>(ws.desc.p);
     p.ticket = static_cast<unsigned long long*>(ws.ticket.p);
     p.base = ws.next_base;
     CUtensorMap ti, to;

@@ -13,12 +13,11 @@
 //   * the horizontal carry (the paper's R) is the per-row running sum L held
 //     in registers by the warp that owns the row;
 //   * the vertical carry (the paper's C and S, i.e. the SAT row above the
-//     band) comes from a decoupled look-back over flag-guarded descriptors:
-//     each (band, chunk) publishes the bottom row of its band-local SAT as an
-//     "aggregate", then -- once it knows the SAT row above -- the final SAT
-//     bottom row as "inclusive".  The look-back reads the
-//     flags of 32 bands per round trip (one per lane) and then the values of
-//     the bands up to the nearest inclusive;
+//     band) comes from a decoupled look-back over self-validating descriptor
+//     words: each (band, chunk) publishes the bottom row of its band-local SAT
+//     as an "aggregate", then -- once it knows the SAT row above -- the final
+//     SAT bottom row as "inclusive".  The look-back reads a
+//     window of LBW bands per round trip;
 //   * inside a chunk, Step 3-1/3-2 of 2R1W become: the compute
 //     warps' local() = row scans with L + column prefix down the warp's R
 //     rows; the result is parked in tensor memory (tcgen05.st) and the smem
@@ -78,8 +77,16 @@ struct BandSmem {
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
+constexpr int LBW = 4;   // look-back window: bands read per round trip
+
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
     return uint32_t((base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
+}
+
+template <typename T>
+__device__ __forceinline__ void publish4(uint64_t* my, uint32_t tag, const V4<T>& v) {
+    st_relaxed_v2(my, (uint64_t(tag) << 32) | to_bits(v.x), (uint64_t(tag) << 32) | to_bits(v.y));
+    st_relaxed_v2(my + 2, (uint64_t(tag) << 32) | to_bits(v.z), (uint64_t(tag) << 32) | to_bits(v.w));
 }
 
 // Row-wise inclusive prefix-sums of R rows of 128 columns (lane owns 4
@@ -430,21 +437,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     V4<T> agg = lds4<T>(xb);
 #pragma unroll
                     for (int w2 = 1; w2 < W; ++w2) add4(agg, lds4<T>(xb + w2 * TW));
-                    // publish (state 1 = aggregate, 2 = inclusive): values,
-                    // gpu fence, warp barrier, then one release-stored flag
-                    auto publish_state = [&](uint32_t state, const V4<T>& v) {
-                        st_relaxed_v4_b32(p.dval + int64_t(state - 1) * p.dplane + int64_t(gb) * desc_w + c0,
-                                          to_bits(v.x), to_bits(v.y), to_bits(v.z), to_bits(v.w));
-                        fence_acq_rel_gpu();
-                        __syncwarp();
-                        if (lane == 0) st_release_b32(p.dflag + int64_t(gb) * p.nc + J, tagbase | state);
-                    };
+                    uint64_t* my = p.desc + int64_t(gb) * desc_w + c0;
                     if (p.jitter && lookback) {
                         uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ lane;
                         h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
                         __nanosleep(h % (uint32_t)p.jitter);
                     }
-                    if (publish && band > 0) publish_state(1u, agg);
+                    if (publish && band > 0) publish4<T>(my, tagbase | 1u, agg);
                     V4<T> top{T(0), T(0), T(0), T(0)};
                     unsigned long long hops = 0, polls = 0;
                     if (!lookback) {
@@ -460,69 +459,66 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             top = V4<T>{e[0], e[1], e[2], e[3]};
                         }
                     } else {
-                        // decoupled look-back: lane q reads the flag of band
-                        // kb-q (32 bands per round trip); the nearest band with
-                        // an inclusive (or, in region C, a final SAT row in
-                        // `out`) ends the walk; the aggregates of the bands in
-                        // between are summed; an unpublished band stalls it.
+                        // decoupled look-back over bands band-1, band-2, ...,
+                        // LBW descriptor rows per round trip
+                        T acc[4] = {T(0), T(0), T(0), T(0)};
+                        uint32_t pend = 0xFu;
                         int kb = band - 1;
                         SpinGuard guard;
-                        for (;;) {
-                            const int bq = kb - lane;
-                            uint32_t st = 0;
-                            if (bq >= 0) {
-                                if (p.region == REG_C && bq + J < p.tA) {
-                                    st = 3u;           // tile (bq, J) is in (A): final row in `out`
+                        while (pend) {
+                            uint64_t wv[LBW][4];
+#pragma unroll
+                            for (int q = 0; q < LBW; ++q) {
+                                const int b2 = kb - q;
+                                if (b2 >= 0) {
+                                    const uint64_t* qp = p.desc + (int64_t(gb) - (band - b2)) * desc_w + c0;
+                                    ld_relaxed_v2(qp, wv[q][0], wv[q][1]);
+                                    ld_relaxed_v2(qp + 2, wv[q][2], wv[q][3]);
                                 } else {
-                                    const int gq2 = gb - (band - bq);
-                                    const uint32_t f = ld_acquire_b32(p.dflag + int64_t(gq2) * p.nc + J);
-                                    if ((f & ~3u) == band_tag(p.base, gq2)) st = f & 3u;
+                                    wv[q][0] = wv[q][1] = wv[q][2] = wv[q][3] = 0;
                                 }
                             }
-                            __syncwarp();                    // order the acquires before the value reads
-                            const uint32_t term = __ballot_sync(0xffffffffu, st >= 2u);
-                            const uint32_t zero = __ballot_sync(0xffffffffu, st == 0u);
-                            const int ft = term ? __ffs(term) - 1 : 32;
-                            const int fz = zero ? __ffs(zero) - 1 : 32;
-                            const int take = ft < fz ? ft + 1 : fz;
-                            for (int q0 = 0; q0 < take; q0 += 8) {
-                                V4<T> vv[8];
+                            bool stalled = false;
 #pragma unroll
-                                for (int i = 0; i < 8; ++i) {
-                                    const int q = q0 + i;
-                                    const uint32_t sq = __shfl_sync(0xffffffffu, st, q & 31);
-                                    vv[i] = V4<T>{T(0), T(0), T(0), T(0)};
-                                    if (q < take) {
-                                        const int b2 = kb - q;
-                                        if (sq == 3u) {
-                                            const int64_t row = int64_t(b2 + 1) * TH - 1;
-                                            T e[4];
+                            for (int q = 0; q < LBW; ++q) {
+                                if (!pend || stalled) break;
+                                const int b2 = kb - q;
+                                if (p.region == REG_C && b2 + J < p.tA) {
+                                    // tile (b2, J) belongs to (A): its final SAT row is in `out`
+                                    const int64_t row = int64_t(b2 + 1) * TH - 1;
 #pragma unroll
-                                            for (int c = 0; c < 4; ++c)
-                                                e[c] = (c0 + c < p.cols) ? gout[row * p.cols + c0 + c] : T(0);
-                                            vv[i] = V4<T>{e[0], e[1], e[2], e[3]};
-                                        } else {
-                                            const uint4 u = ld_relaxed_v4_b32(
-                                                p.dval + int64_t(sq - 1) * p.dplane
-                                                + int64_t(gb - (band - b2)) * desc_w + c0);
-                                            vv[i] = V4<T>{from_bits<T>(u.x), from_bits<T>(u.y),
-                                                          from_bits<T>(u.z), from_bits<T>(u.w)};
-                                        }
+                                    for (int i = 0; i < 4; ++i)
+                                        if ((pend >> i) & 1u)
+                                            acc[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
+                                    pend = 0;
+                                    break;
+                                }
+                                const uint32_t tk = band_tag(p.base, gb - (band - b2));
+                                bool ready = true;
+#pragma unroll
+                                for (int i = 0; i < 4; ++i) {
+                                    const uint32_t t = uint32_t(wv[q][i] >> 32);
+                                    ready = ready && ((t & ~3u) == tk) && (t & 3u);
+                                }
+                                if (!ready) { stalled = true; kb = b2; break; }
+#pragma unroll
+                                for (int i = 0; i < 4; ++i) {
+                                    if ((pend >> i) & 1u) {
+                                        acc[i] += from_bits<T>(uint32_t(wv[q][i]));
+                                        if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
                                     }
                                 }
-#pragma unroll
-                                for (int i = 0; i < 8; ++i) add4(top, vv[i]);
+                                ++hops;
                             }
-                            hops += take;
-                            if (ft < fz) break;
-                            kb -= take;
-                            if (fz < 32) { __nanosleep(32); guard.tick(); ++polls; }
+                            if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
+                            else kb -= LBW;
                         }
+                        top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
                     }
                     if (publish) {
                         V4<T> inc = agg;
                         add4(inc, top);
-                        publish_state(2u, inc);
+                        publish4<T>(my, tagbase | 2u, inc);
                     }
                     if (p.trace && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =

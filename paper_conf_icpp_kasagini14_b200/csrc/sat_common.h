@@ -45,9 +45,7 @@ struct BandParams {
     int total_bands;           // batch * nb
     long long total_units;     // bands (band units) or bands*nc (tile units)
     int tile_units;            // 1: one ticket = one tile (external carries)
-    uint32_t* dval;            // [2][total_bands][nc*TW] descriptor values: aggregate, inclusive
-    uint32_t* dflag;           // [total_bands][nc] descriptor flags: tag << 2 | state
-    int64_t dplane;            // total_bands * nc * TW (one value plane)
+    uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)
     const void* seed;          // [cols] SAT row above band 0 of image 0, nullable

@@ -126,31 +126,6 @@ __device__ __forceinline__ unsigned long long globaltimer() {
     return t;
 }
 
-// Flag-guarded descriptors: 32-bit values are written
-// with relaxed gpu-scope stores, ordered by a gpu fence and a warp barrier
-// before one lane release-stores the (tag | state) flag; readers acquire the
-// flag, synchronise the warp, then read values at gpu scope (never from L1).
-__device__ __forceinline__ void st_relaxed_v4_b32(uint32_t* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
-    asm volatile("st.relaxed.gpu.global.v4.b32 [%0], {%1, %2, %3, %4};" :: "l"(p), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
-}
-__device__ __forceinline__ uint4 ld_relaxed_v4_b32(const uint32_t* p) {
-    uint4 v;
-    asm volatile("ld.relaxed.gpu.global.v4.b32 {%0, %1, %2, %3}, [%4];"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_b32(uint32_t* p, uint32_t v) {
-    asm volatile("st.release.gpu.global.b32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ uint32_t ld_acquire_b32(const uint32_t* p) {
-    uint32_t v;
-    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void fence_acq_rel_gpu() {
-    asm volatile("fence.acq_rel.gpu;" ::: "memory");
-}
-
 // ------------------------------------------------------------- arithmetic
 // int32 SATs are computed in uint32 (mod 2^32); float32 in IEEE fp32 adds.
 template <typename T> __device__ __forceinline__ uint32_t to_bits(T v);
