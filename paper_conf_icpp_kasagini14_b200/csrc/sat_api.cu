@@ -181,23 +181,23 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
 
 // ------------------------------------------------------------------ band kernel dispatch
 struct BandCfg {
-    int R, W, S, DT, SUB, NCW, MINB;
+    int R, W, S, DT, SUB, NCW, NS, MINB;
 };
 // TH = R*W rows per band, W compute warps of R rows.  Shared memory per CTA:
 // S ring slots of SUB adjacent TH x 128 chunks (SUB*512 B per row per load:
 // wider row segments keep HBM pages busy) + DT*W*512 B
 // (bottom rows / add vectors) + barriers; TMEM per CTA: DT chunks x 4R words
 // per compute thread.  Two CTAs per SM.
-constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 2};
-constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 2};
-constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 2};
+constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 2, 2};
+constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 2, 2};
+constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 2, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 2, 2};
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
     (void)to;
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, MODE, TMA, MINB>;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB>;
     const size_t smem = BandSmem<T, R, W, S, DT, SUB>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
@@ -229,19 +229,18 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     return SAT_OK;
 }
 
-#define SAT_CFG(c) c.R, c.W, c.S, c.DT, c.SUB, c.NCW
+#define SAT_CFG(c) c.R, c.W, c.S, c.DT, c.SUB, c.NCW, c.NS
 template <typename T, int MODE, bool TMA>
 int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                    const DevInfo& di, cudaStream_t st, int& grid) {
     if constexpr (MODE == MODE_SAT && TMA && std::is_same<T, uint32_t>::value) {
-        // debug: alternative TH=16 configurations (SAT_DEBUG_CFG=1|2)
+        // debug: column split of the control warps (SAT_DEBUG_CFG=1|2|4 -> NS)
         if (const char* e = getenv("SAT_DEBUG_CFG")) {
-            if (th == 16 && atoi(e) == 1)
-                return launch_band_t<T, 4, 4, 3, 8, 1, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 16 && atoi(e) == 2)
-                return launch_band_t<T, 2, 8, 3, 8, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 16 && atoi(e) == 3)
-                return launch_band_t<T, 4, 4, 3, 4, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            const int ns = atoi(e);
+            if (th == 64 && ns == 1) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 1, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 64 && ns == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 32 && ns == 1) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 1, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
         }
     }
     switch (th) {

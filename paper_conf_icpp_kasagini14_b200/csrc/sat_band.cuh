@@ -33,9 +33,9 @@
 // and the 1R1W band (C) of (1+r)R1W.
 //
 // Roles (warps): 0..W-1 compute (R rows each), W..W+NCW-1 control
-// (descriptors and look-back; control warp c owns the chunks k = c mod NCW,
-// so NCW look-backs are in flight at once), W+NCW = producer (TMA loads, one
-// elected lane).
+// (descriptors and look-back, in NCW/NS groups of NS warps that split a
+// chunk's columns; group g owns the chunks k = g mod NCW/NS), W+NCW =
+// producer (TMA loads, one elected lane).
 #pragma once
 #include "sat_common.h"
 #include "sat_device.cuh"
@@ -77,16 +77,57 @@ struct BandSmem {
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
-constexpr int LBW = 4;   // look-back window: bands read per round trip
-
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
     return uint32_t((base + (unsigned long long)gb) & 0x3FFFFFFFull) << 2;
 }
 
-template <typename T>
-__device__ __forceinline__ void publish4(uint64_t* my, uint32_t tag, const V4<T>& v) {
-    st_relaxed_v2(my, (uint64_t(tag) << 32) | to_bits(v.x), (uint64_t(tag) << 32) | to_bits(v.y));
-    st_relaxed_v2(my + 2, (uint64_t(tag) << 32) | to_bits(v.z), (uint64_t(tag) << 32) | to_bits(v.w));
+// CPL consecutive columns (4, 2 or 1) as one shared-memory vector access.
+template <typename T, int CPL>
+__device__ __forceinline__ void lds_cols(const T* p, T (&v)[CPL]) {
+    if constexpr (CPL == 4) {
+        const uint4 u = *reinterpret_cast<const uint4*>(p);
+        v[0] = from_bits<T>(u.x); v[1] = from_bits<T>(u.y); v[2] = from_bits<T>(u.z); v[3] = from_bits<T>(u.w);
+    } else if constexpr (CPL == 2) {
+        const uint2 u = *reinterpret_cast<const uint2*>(p);
+        v[0] = from_bits<T>(u.x); v[1] = from_bits<T>(u.y);
+    } else {
+        v[0] = *p;
+    }
+}
+template <typename T, int CPL>
+__device__ __forceinline__ void sts_cols(T* p, const T (&v)[CPL]) {
+    if constexpr (CPL == 4) {
+        *reinterpret_cast<uint4*>(p) = make_uint4(to_bits(v[0]), to_bits(v[1]), to_bits(v[2]), to_bits(v[3]));
+    } else if constexpr (CPL == 2) {
+        *reinterpret_cast<uint2*>(p) = make_uint2(to_bits(v[0]), to_bits(v[1]));
+    } else {
+        *p = v[0];
+    }
+}
+
+// Descriptor words (tag << 32 | value bits) of CPL consecutive columns.
+template <int CPL>
+__device__ __forceinline__ void load_words(const uint64_t* q, uint64_t (&w)[CPL]) {
+    if constexpr (CPL == 4) {
+        ld_relaxed_v2(q, w[0], w[1]);
+        ld_relaxed_v2(q + 2, w[2], w[3]);
+    } else if constexpr (CPL == 2) {
+        ld_relaxed_v2(q, w[0], w[1]);
+    } else {
+        asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w[0]) : "l"(q) : "memory");
+    }
+}
+template <typename T, int CPL>
+__device__ __forceinline__ void publish_words(uint64_t* my, uint32_t tag, const T (&v)[CPL]) {
+    const uint64_t hi = uint64_t(tag) << 32;
+    if constexpr (CPL == 4) {
+        st_relaxed_v2(my, hi | to_bits(v[0]), hi | to_bits(v[1]));
+        st_relaxed_v2(my + 2, hi | to_bits(v[2]), hi | to_bits(v[3]));
+    } else if constexpr (CPL == 2) {
+        st_relaxed_v2(my, hi | to_bits(v[0]), hi | to_bits(v[1]));
+    } else {
+        asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" :: "l"(my), "l"(hi | to_bits(v[0])) : "memory");
+    }
 }
 
 // Row-wise inclusive prefix-sums of R rows of 128 columns (lane owns 4
@@ -203,7 +244,7 @@ struct TmemCols {
     static_assert(need <= 512, "TMEM holds at most 512 columns");
 };
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -219,7 +260,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     // A control warp waits on colr[] of chunk k only after finishing chunk
     // k-NCW, which implies local(k-XS) completed iff NCW <= XS; otherwise the
     // parity wait could pass on a stale phase.
-    static_assert(NCW <= XS, "more control warps than carry slots");
+    static_assert(NCW % NS == 0 && (NS == 1 || NS == 2 || NS == 4), "control warps split columns 1, 2 or 4 ways");
+    static_assert(NCW / NS <= XS, "more control groups than carry slots");
 
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
@@ -242,7 +284,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         }
         for (int x = 0; x < XS; ++x) {
             mbar_init(&colr[x], W * 32);
-            mbar_init(&topr[x], 32);
+            mbar_init(&topr[x], 32 * NS);
         }
         fence_mbar_init();
     }
@@ -421,61 +463,75 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             }
         } else if (warp < PW) {
             // ================= control warps: descriptors + look-back =================
+            // NCW warps form G = NCW/NS groups; group g owns the chunks
+            // k = g mod G and its NS warps split the 128 columns (CPL per
+            // lane), so one round trip reads LBW = 16/CPL bands' words in the
+            // same 32 registers per lane.
             if constexpr (HOLD) {
+                constexpr int CPL = 4 / NS;
+                constexpr int G = NCW / NS;
+                constexpr int LBW = 16 / CPL;
+                const int cw = warp - CW;
+                const int grp = cw / NS;
+                const int cl = (cw % NS) * (TW / NS) + lane * CPL;   // column within the chunk
                 const uint32_t tagbase = band_tag(p.base, gb);
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
                 const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
-                for (int k = warp - CW; k < nch; k += NCW) {
+                for (int k = grp; k < nch; k += G) {
                     const uint32_t it = g + k;
                     const int J = j0 + k;
-                    const int c0 = J * TW + 4 * lane;
-                    T* xb = xbuf + size_t(it % XS) * W * TW + 4 * lane;
+                    const int c0 = J * TW + cl;
+                    T* xb = xbuf + size_t(it % XS) * W * TW + cl;
                     mbar_wait(&colr[it % XS], (it / XS) & 1);
-                    if (p.trace && lane == 0)
+                    if (p.trace && cw == grp * NS && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
-                    V4<T> agg = lds4<T>(xb);
+                    T agg[CPL];
+                    lds_cols<T, CPL>(xb, agg);
 #pragma unroll
-                    for (int w2 = 1; w2 < W; ++w2) add4(agg, lds4<T>(xb + w2 * TW));
+                    for (int w2 = 1; w2 < W; ++w2) {
+                        T b[CPL];
+                        lds_cols<T, CPL>(xb + w2 * TW, b);
+#pragma unroll
+                        for (int i = 0; i < CPL; ++i) agg[i] += b[i];
+                    }
                     uint64_t* my = p.desc + int64_t(gb) * desc_w + c0;
                     if (p.jitter && lookback) {
-                        uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ lane;
+                        uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ (uint32_t(cl) * 97u);
                         h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
                         __nanosleep(h % (uint32_t)p.jitter);
                     }
-                    if (publish && band > 0) publish4<T>(my, tagbase | 1u, agg);
-                    V4<T> top{T(0), T(0), T(0), T(0)};
+                    if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                    T top[CPL];
+#pragma unroll
+                    for (int i = 0; i < CPL; ++i) top[i] = T(0);
                     unsigned long long hops = 0, polls = 0;
                     if (!lookback) {
-                        top = lds4<T>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0);
+                        lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
                     } else if (band == 0) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
                             // the SAT row just above the matrix (sat_api.cu turns a
                             // column-sum seed into this row first)
                             const T* sd = reinterpret_cast<const T*>(p.seed);
-                            T e[4];
 #pragma unroll
-                            for (int i = 0; i < 4; ++i) e[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
-                            top = V4<T>{e[0], e[1], e[2], e[3]};
+                            for (int i = 0; i < CPL; ++i) top[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
                         }
                     } else {
                         // decoupled look-back over bands band-1, band-2, ...,
                         // LBW descriptor rows per round trip
-                        T acc[4] = {T(0), T(0), T(0), T(0)};
-                        uint32_t pend = 0xFu;
+                        uint32_t pend = (1u << CPL) - 1u;
                         int kb = band - 1;
                         SpinGuard guard;
                         while (pend) {
-                            uint64_t wv[LBW][4];
+                            uint64_t wv[LBW][CPL];
 #pragma unroll
                             for (int q = 0; q < LBW; ++q) {
                                 const int b2 = kb - q;
                                 if (b2 >= 0) {
-                                    const uint64_t* qp = p.desc + (int64_t(gb) - (band - b2)) * desc_w + c0;
-                                    ld_relaxed_v2(qp, wv[q][0], wv[q][1]);
-                                    ld_relaxed_v2(qp + 2, wv[q][2], wv[q][3]);
+                                    load_words<CPL>(p.desc + (int64_t(gb) - (band - b2)) * desc_w + c0, wv[q]);
                                 } else {
-                                    wv[q][0] = wv[q][1] = wv[q][2] = wv[q][3] = 0;
+#pragma unroll
+                                    for (int i = 0; i < CPL; ++i) wv[q][i] = 0;
                                 }
                             }
                             bool stalled = false;
@@ -487,24 +543,24 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                     // tile (b2, J) belongs to (A): its final SAT row is in `out`
                                     const int64_t row = int64_t(b2 + 1) * TH - 1;
 #pragma unroll
-                                    for (int i = 0; i < 4; ++i)
+                                    for (int i = 0; i < CPL; ++i)
                                         if ((pend >> i) & 1u)
-                                            acc[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
+                                            top[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
                                     pend = 0;
                                     break;
                                 }
                                 const uint32_t tk = band_tag(p.base, gb - (band - b2));
                                 bool ready = true;
 #pragma unroll
-                                for (int i = 0; i < 4; ++i) {
+                                for (int i = 0; i < CPL; ++i) {
                                     const uint32_t t = uint32_t(wv[q][i] >> 32);
                                     ready = ready && ((t & ~3u) == tk) && (t & 3u);
                                 }
                                 if (!ready) { stalled = true; kb = b2; break; }
 #pragma unroll
-                                for (int i = 0; i < 4; ++i) {
+                                for (int i = 0; i < CPL; ++i) {
                                     if ((pend >> i) & 1u) {
-                                        acc[i] += from_bits<T>(uint32_t(wv[q][i]));
+                                        top[i] += from_bits<T>(uint32_t(wv[q][i]));
                                         if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
                                     }
                                 }
@@ -513,23 +569,24 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
                             else kb -= LBW;
                         }
-                        top = V4<T>{acc[0], acc[1], acc[2], acc[3]};
                     }
                     if (publish) {
-                        V4<T> inc = agg;
-                        add4(inc, top);
-                        publish4<T>(my, tagbase | 2u, inc);
+                        T inc[CPL];
+#pragma unroll
+                        for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
+                        publish_words<T, CPL>(my, tagbase | 2u, inc);
                     }
-                    if (p.trace && lane == 0)
+                    if (p.trace && cw == grp * NS && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
                             (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
                     // add vectors for finish(): top + bottom rows of the warps above
-                    V4<T> run = top;
 #pragma unroll
                     for (int w2 = 0; w2 < W; ++w2) {
-                        const V4<T> b = lds4<T>(xb + w2 * TW);
-                        sts4(xb + w2 * TW, run);
-                        add4(run, b);
+                        T b[CPL];
+                        lds_cols<T, CPL>(xb + w2 * TW, b);
+                        sts_cols<T, CPL>(xb + w2 * TW, top);
+#pragma unroll
+                        for (int i = 0; i < CPL; ++i) top[i] += b[i];
                     }
                     mbar_arrive(&topr[it % XS]);
                 }
