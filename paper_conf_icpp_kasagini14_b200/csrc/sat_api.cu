@@ -188,10 +188,10 @@ struct BandCfg {
 // wider row segments keep HBM pages busy) + DT*W*512 B
 // (bottom rows / add vectors) + barriers; TMEM per CTA: DT chunks x 4R words
 // per compute thread.  Two CTAs per SM.
-constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 2, 2};
-constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 2, 2};
-constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 2, 2};
-constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 2, 2};
+constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 1, 2};
+constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
+constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 1, 2};
+constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
@@ -237,9 +237,9 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         // debug: column split of the control warps (SAT_DEBUG_CFG=1|2|4 -> NS)
         if (const char* e = getenv("SAT_DEBUG_CFG")) {
             const int ns = atoi(e);
-            if (th == 64 && ns == 1) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 1, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 64 && ns == 2) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
             if (th == 64 && ns == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 32 && ns == 1) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 1, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 32 && ns == 2) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
             if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
         }
     }
