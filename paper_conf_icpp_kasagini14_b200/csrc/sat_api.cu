@@ -193,12 +193,13 @@ constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
 constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 1, 2};
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
+          int CL = 1>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
     (void)to;
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB>;
-    const size_t smem = BandSmem<T, R, W, S, DT, SUB>::total;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB>;
+    const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
@@ -219,11 +220,36 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
                         MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT>::alloc, 32});
     if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
     if (const char* e = getenv("SAT_DEBUG_OCC")) occ = atoi(e);
-    long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
-    if (grid < 1) grid = 1;
-    grid_out = int(grid);
-    t_grid = int(grid);
-    kern<<<int(grid), threads, smem, st>>>(ti, p);
+    if constexpr (CL > 1) {
+        // clusters of CL CTAs (CL consecutive bands); persistent, one ticket
+        // per cluster.  Clusters that cannot be co-resident simply start
+        // late and find no ticket left.
+        long long ncl = std::min<long long>(p.total_units, (long long)occ * di.sms / CL);
+        if (ncl < 1) ncl = 1;
+        const long long grid = ncl * CL;
+        grid_out = int(grid);
+        t_grid = int(grid);
+        cudaLaunchConfig_t cfg;
+        std::memset(&cfg, 0, sizeof(cfg));
+        cfg.gridDim = dim3(unsigned(grid));
+        cfg.blockDim = dim3(unsigned(threads));
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = st;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = CL;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ti, p));
+    } else {
+        long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
+        if (grid < 1) grid = 1;
+        grid_out = int(grid);
+        t_grid = int(grid);
+        kern<<<int(grid), threads, smem, st>>>(ti, p);
+    }
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     return SAT_OK;
@@ -242,6 +268,12 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
             if (th == 32 && ns == 2) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
             if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
         }
+    }
+    if constexpr (MODE == MODE_SAT && TMA) {
+        if (p.cluster == 8 && th == 64)
+            return launch_band_t<T, 8, 8, 3, 3, 1, 3, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
+        if (p.cluster == 8 && th == 48)
+            return launch_band_t<T, 8, 6, 2, 4, 2, 4, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
     }
     switch (th) {
         case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
@@ -306,6 +338,18 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.nc = int((j.cols + TW - 1) / TW);
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * p.nc : p.total_bands;
+    // Clusters of 8 bands pass the vertical carry through DSMEM (DESIGN.md
+    // Sec. 4.5): plain 1R1W on the TMA path, when few virtual bands pad the
+    // last cluster of each image.
+    p.cluster = 1;
+    if (mode == MODE_SAT && j.tma && p.region == REG_ALL && p.top_src == TOP_LOOKBACK &&
+        !p.tile_units && (j.th == 64 || j.th == 48) && (p.nb % 8 == 0 || p.nb >= 160))
+        p.cluster = 8;
+    if (const char* e = getenv("SAT_DEBUG_CL")) {
+        if (atoi(e) <= 1) p.cluster = 1;
+    }
+    if (p.cluster > 1)
+        p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
     p.jitter = j.jitter;
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
         p.trace = t_trace;

@@ -65,7 +65,7 @@ __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int DT, int SUB>
+template <typename T, int R, int W, int S, int DT, int SUB, int CL = 1>
 struct BandSmem {
     static constexpr int TH = R * W;
     static constexpr int XS = DT;                    // carry slots: one per parked chunk
@@ -73,8 +73,11 @@ struct BandSmem {
     static constexpr size_t slot_elems = tile_elems * SUB;           // one ring slot
     static constexpr size_t tiles = S * slot_elems * sizeof(T);
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
-    static constexpr size_t bars = size_t(2 * S + 2 * XS) * sizeof(uint64_t) + 16;
-    static constexpr size_t total = tiles + xbuf + bars;
+    // clusters: incoming partial aggregate (chain) and cluster top row per carry slot
+    static constexpr size_t cbuf = CL > 1 ? size_t(2) * XS * TW * sizeof(T) : 0;
+    static constexpr size_t nbars = 2 * S + 2 * XS + (CL > 1 ? 4 * XS : 0);
+    static constexpr size_t bars = nbars * sizeof(uint64_t) + 16;
+    static constexpr size_t total = tiles + xbuf + cbuf + bars;
 };
 
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
@@ -244,7 +247,7 @@ struct TmemCols {
     static_assert(need <= 512, "TMEM holds at most 512 columns");
 };
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int CL, int MODE, bool TMA, int MINB>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -253,7 +256,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S, DT, SUB>;
+    using SM = BandSmem<T, R, W, S, DT, SUB, CL>;
+    static_assert(CL == 1 || (MODE == MODE_SAT && NS == 1), "clusters: 1R1W band kernel only");
     using TC = TmemCols<R, W, DT>;
     constexpr int XS = SM::XS;
     constexpr bool HOLD = (MODE != MODE_ROW);    // chunks wait for a vertical carry
@@ -266,13 +270,23 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf);
+    T* chain = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);        // [XS][TW] (CL > 1)
+    T* ctop = chain + size_t(XS) * TW;                                    // [XS][TW] (CL > 1)
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf + SM::cbuf);
     uint64_t* full = bars;              // [S]  TMA load landed (tx count)
     uint64_t* empty = bars + S;         // [S]  every compute warp read the slot
     uint64_t* colr = bars + 2 * S;      // [XS] every compute warp published its bottom row
     uint64_t* topr = bars + 2 * S + XS; // [XS] the control warp wrote the add vectors
-    long long* s_unit = reinterpret_cast<long long*>(bars + 2 * S + 2 * XS);
+    // clusters (CL > 1), per carry slot: chainb = partial aggregate from rank-1
+    // arrived; chainfree = rank+1 consumed ours; ctopb = cluster top row from
+    // rank 0 arrived; ctopfree (rank 0) = every other rank consumed it
+    uint64_t* chainb = bars + 2 * S + 2 * XS;
+    uint64_t* chainfree = chainb + XS;
+    uint64_t* ctopb = chainb + 2 * XS;
+    uint64_t* ctopfree = chainb + 3 * XS;
+    long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
     uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 1);
+    const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -285,6 +299,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         for (int x = 0; x < XS; ++x) {
             mbar_init(&colr[x], W * 32);
             mbar_init(&topr[x], 32 * NS);
+            if constexpr (CL > 1) {
+                mbar_init(&chainb[x], 32);
+                mbar_init(&chainfree[x], 32);
+                mbar_init(&ctopb[x], 32);
+                mbar_init(&ctopfree[x], 32 * (CL - 1));
+            }
         }
         fence_mbar_init();
     }
@@ -296,6 +316,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     if (TMA && warp == PW && lane == 0) prefetch_tmap(&tm_in);
     tmem_fence_before();
     __syncthreads();
+    if constexpr (CL > 1) cluster_sync_all();    // peers' barriers initialised before any remote arrive
     tmem_fence_after();
     const uint32_t tmem_base = HOLD ? *s_tmem : 0u;
 
@@ -306,14 +327,31 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
 
     for (;;) {
-        if (threadIdx.x == 0)
-            *s_unit = (long long)(atomicAdd(p.ticket, 1ull) - p.base);
-        __syncthreads();
+        if constexpr (CL > 1) {
+            // one ticket per cluster: CL consecutive bands, rank r takes band CL*u + r
+            if (crank == 0 && threadIdx.x == 0) {
+                const unsigned long long u = atomicAdd(p.ticket, 1ull) - p.base;
+                for (uint32_t r = 0; r < CL; ++r) st_cluster_u64(mapa(smem_u32(s_unit), r), u);
+            }
+            cluster_sync_all();
+        } else {
+            if (threadIdx.x == 0)
+                *s_unit = (long long)(atomicAdd(p.ticket, 1ull) - p.base);
+            __syncthreads();
+        }
         const long long unit = *s_unit;
         if (unit >= p.total_units) break;
 
         int gb, j0, j1;
-        if (p.tile_units) {
+        int gcb = 0, cb = 0;                           // cluster-band (CL > 1)
+        if constexpr (CL > 1) {
+            const int upi = (p.nb + CL - 1) / CL;       // cluster-bands per image
+            gcb = int(unit);
+            const int im = gcb / upi;
+            cb = gcb - im * upi;
+            gb = im * p.nb + cb * CL + int(crank);      // may exceed the image: a virtual band
+            j0 = 0; j1 = p.nc;
+        } else if (p.tile_units) {
             gb = int(unit / p.nc);
             const int J = int(unit % p.nc);
             int r0, r1;
@@ -323,10 +361,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             gb = int(unit);
             region_range(p.region, p.tA, p.nb, p.nc, gb % p.nb, j0, j1);
         }
-        const int img = gb / p.nb;
-        const int band = gb - img * p.nb;
+        const int img = CL > 1 ? gcb / ((p.nb + CL - 1) / CL) : gb / p.nb;
+        const int band = gb - img * p.nb;              // >= p.nb: virtual (rows all beyond the matrix)
         const int nch = j1 - j0;
         const int row0 = band * TH;
+        const bool traced = p.trace != nullptr && band < p.nb;
 
         if (warp < W) {
             // ================= compute warps =================
@@ -375,7 +414,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     const uint32_t q = gq + uint32_t(k / SUB);     // ring slot of chunk k
                     const int s = q % S;
                     if (k % SUB == 0) mbar_wait(&full[s], (q / S) & 1);
-                    if (p.trace && warp == 0 && lane == 0)
+                    if (traced && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
                     const T* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
                                  + size_t(rbase) * TW + 4 * lane;
@@ -428,7 +467,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             auto finish = [&](int k) {
                 const uint32_t it = g + k;
                 mbar_wait(&topr[it % XS], (it / XS) & 1);
-                if (p.trace && warp == 0 && lane == 0)
+                if (traced && warp == 0 && lane == 0)
                     p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
                 const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
                 uint32_t u[4 * R];
@@ -443,7 +482,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     add4(v[r], add);
                 }
                 store_rows(v, k);
-                if (p.trace && warp == 0 && lane == 0)
+                if (traced && warp == 0 && lane == 0)
                     p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
             };
 
@@ -484,7 +523,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     const int c0 = J * TW + cl;
                     T* xb = xbuf + size_t(it % XS) * W * TW + cl;
                     mbar_wait(&colr[it % XS], (it / XS) & 1);
-                    if (p.trace && cw == grp * NS && lane == 0)
+                    if (traced && cw == grp * NS && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
                     T agg[CPL];
                     lds_cols<T, CPL>(xb, agg);
@@ -501,82 +540,146 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
                         __nanosleep(h % (uint32_t)p.jitter);
                     }
-                    if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
                     T top[CPL];
 #pragma unroll
                     for (int i = 0; i < CPL; ++i) top[i] = T(0);
                     unsigned long long hops = 0, polls = 0;
-                    if (!lookback) {
-                        lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
-                    } else if (band == 0) {
+                    // decoupled look-back from descriptor row gidx (index idx
+                    // within its image) over rows idx-1, idx-2, ...: adds the
+                    // SAT row above row idx to acc
+                    auto walk = [&](int gidx, int idx, T (&acc)[CPL]) {
+                        T (&top)[CPL] = acc;
+                    // decoupled look-back over bands band-1, band-2, ...,
+                    // LBW descriptor rows per round trip
+                    uint32_t pend = (1u << CPL) - 1u;
+                    int kb = idx - 1;
+                    SpinGuard guard;
+                    while (pend) {
+                        uint64_t wv[LBW][CPL];
+#pragma unroll
+                        for (int q = 0; q < LBW; ++q) {
+                            const int b2 = kb - q;
+                            if (b2 >= 0) {
+                                load_words<CPL>(p.desc + (int64_t(gidx) - (idx - b2)) * desc_w + c0, wv[q]);
+                            } else {
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i) wv[q][i] = 0;
+                            }
+                        }
+                        bool stalled = false;
+#pragma unroll
+                        for (int q = 0; q < LBW; ++q) {
+                            if (!pend || stalled) break;
+                            const int b2 = kb - q;
+                            if (CL == 1 && p.region == REG_C && b2 + J < p.tA) {
+                                // tile (b2, J) belongs to (A): its final SAT row is in `out`
+                                const int64_t row = int64_t(b2 + 1) * TH - 1;
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i)
+                                    if ((pend >> i) & 1u)
+                                        top[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
+                                pend = 0;
+                                break;
+                            }
+                            const uint32_t tk = band_tag(p.base, gidx - (idx - b2));
+                            bool ready = true;
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i) {
+                                const uint32_t t = uint32_t(wv[q][i] >> 32);
+                                ready = ready && ((t & ~3u) == tk) && (t & 3u);
+                            }
+                            if (!ready) { stalled = true; kb = b2; break; }
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i) {
+                                if ((pend >> i) & 1u) {
+                                    top[i] += from_bits<T>(uint32_t(wv[q][i]));
+                                    if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
+                                }
+                            }
+                            ++hops;
+                        }
+                        if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
+                        else kb -= LBW;
+                    }
+                    };
+                    auto seed_row = [&](T (&acc)[CPL]) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
                             // the SAT row just above the matrix (sat_api.cu turns a
                             // column-sum seed into this row first)
                             const T* sd = reinterpret_cast<const T*>(p.seed);
 #pragma unroll
-                            for (int i = 0; i < CPL; ++i) top[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
+                            for (int i = 0; i < CPL; ++i) acc[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
+                        }
+                    };
+                    if constexpr (CL > 1) {
+                        // Cluster of CL bands (DSMEM): the
+                        // partial aggregates S_r = agg_0 + .. + agg_r run down a
+                        // chain rank 0 -> 1 -> .. -> CL-1; rank 0 looks back over
+                        // the cluster-band descriptors and broadcasts the SAT row
+                        // T above the cluster; rank r's top = T + S_{r-1}; rank
+                        // CL-1 publishes the cluster's aggregate S_{CL-1} and
+                        // inclusive T + S_{CL-1}.
+                        const uint32_t x = it % XS, ph = (it / XS) & 1u;
+                        const int upi = (p.nb + CL - 1) / CL;
+                        const bool pubc = cb + 1 < upi;
+                        uint64_t* myc = p.desc + int64_t(gcb) * desc_w + c0;
+                        const uint32_t ctag = band_tag(p.base, gcb);
+                        T Sa[CPL] = {}, Sp[CPL] = {};
+                        auto send_chain = [&]() {
+                            if (it >= uint32_t(XS)) mbar_wait_cluster(&chainfree[x], ph ^ 1u);
+                            st_cluster_v4(mapa(smem_u32(chain + size_t(x) * TW + cl), crank + 1),
+                                          to_bits(Sa[0]), to_bits(Sa[1]), to_bits(Sa[2]), to_bits(Sa[3]));
+                            mbar_arrive_remote(mapa(smem_u32(&chainb[x]), crank + 1));
+                        };
+                        if (crank == 0) {
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i) { Sa[i] = agg[i]; Sp[i] = T(0); }
+                            send_chain();
+                            if (cb == 0) seed_row(top);
+                            else walk(gcb, cb, top);
+                            if (it >= uint32_t(XS)) mbar_wait_cluster(&ctopfree[x], ph ^ 1u);
+                            for (uint32_t r2 = 1; r2 < CL; ++r2) {
+                                st_cluster_v4(mapa(smem_u32(ctop + size_t(x) * TW + cl), r2),
+                                              to_bits(top[0]), to_bits(top[1]), to_bits(top[2]), to_bits(top[3]));
+                                mbar_arrive_remote(mapa(smem_u32(&ctopb[x]), r2));
+                            }
+                        } else {
+                            mbar_wait_cluster(&chainb[x], ph);
+                            lds_cols<T, CPL>(chain + size_t(x) * TW + cl, Sp);
+                            mbar_arrive_remote(mapa(smem_u32(&chainfree[x]), crank - 1));
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i) Sa[i] = Sp[i] + agg[i];
+                            if (crank + 1 < CL) send_chain();
+                            else if (pubc) publish_words<T, CPL>(myc, ctag | 1u, Sa);
+                            mbar_wait_cluster(&ctopb[x], ph);
+                            lds_cols<T, CPL>(ctop + size_t(x) * TW + cl, top);
+                            mbar_arrive_remote(mapa(smem_u32(&ctopfree[x]), 0));
+                            if (crank + 1 == CL && pubc) {
+                                T inc[CPL];
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i) inc[i] = top[i] + Sa[i];
+                                publish_words<T, CPL>(myc, ctag | 2u, inc);
+                            }
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i) top[i] += Sp[i];
                         }
                     } else {
-                        // decoupled look-back over bands band-1, band-2, ...,
-                        // LBW descriptor rows per round trip
-                        uint32_t pend = (1u << CPL) - 1u;
-                        int kb = band - 1;
-                        SpinGuard guard;
-                        while (pend) {
-                            uint64_t wv[LBW][CPL];
+                        if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                        if (!lookback) {
+                            lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
+                        } else if (band == 0) {
+                            seed_row(top);
+                        } else {
+                            walk(gb, band, top);
+                        }
+                        if (publish) {
+                            T inc[CPL];
 #pragma unroll
-                            for (int q = 0; q < LBW; ++q) {
-                                const int b2 = kb - q;
-                                if (b2 >= 0) {
-                                    load_words<CPL>(p.desc + (int64_t(gb) - (band - b2)) * desc_w + c0, wv[q]);
-                                } else {
-#pragma unroll
-                                    for (int i = 0; i < CPL; ++i) wv[q][i] = 0;
-                                }
-                            }
-                            bool stalled = false;
-#pragma unroll
-                            for (int q = 0; q < LBW; ++q) {
-                                if (!pend || stalled) break;
-                                const int b2 = kb - q;
-                                if (p.region == REG_C && b2 + J < p.tA) {
-                                    // tile (b2, J) belongs to (A): its final SAT row is in `out`
-                                    const int64_t row = int64_t(b2 + 1) * TH - 1;
-#pragma unroll
-                                    for (int i = 0; i < CPL; ++i)
-                                        if ((pend >> i) & 1u)
-                                            top[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
-                                    pend = 0;
-                                    break;
-                                }
-                                const uint32_t tk = band_tag(p.base, gb - (band - b2));
-                                bool ready = true;
-#pragma unroll
-                                for (int i = 0; i < CPL; ++i) {
-                                    const uint32_t t = uint32_t(wv[q][i] >> 32);
-                                    ready = ready && ((t & ~3u) == tk) && (t & 3u);
-                                }
-                                if (!ready) { stalled = true; kb = b2; break; }
-#pragma unroll
-                                for (int i = 0; i < CPL; ++i) {
-                                    if ((pend >> i) & 1u) {
-                                        top[i] += from_bits<T>(uint32_t(wv[q][i]));
-                                        if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
-                                    }
-                                }
-                                ++hops;
-                            }
-                            if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
-                            else kb -= LBW;
+                            for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
+                            publish_words<T, CPL>(my, tagbase | 2u, inc);
                         }
                     }
-                    if (publish) {
-                        T inc[CPL];
-#pragma unroll
-                        for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
-                        publish_words<T, CPL>(my, tagbase | 2u, inc);
-                    }
-                    if (p.trace && cw == grp * NS && lane == 0)
+                    if (traced && cw == grp * NS && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
                             (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
                     // add vectors for finish(): top + bottom rows of the warps above
@@ -601,7 +704,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         const int s = q % S;
                         const int nsub = nch - k0 < SUB ? nch - k0 : SUB;
                         if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
-                        if (p.trace)
+                        if (traced)
                             p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();
                         mbar_arrive_expect_tx(&full[s], TILE_BYTES * nsub);
                         for (int j = 0; j < nsub; ++j)   // adjacent boxes: SUB*512 B per row
@@ -613,7 +716,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         }
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
-        __syncthreads();
+        if constexpr (CL > 1) cluster_sync_all();      // before rank 0 overwrites s_unit
+        else __syncthreads();
     }
     if (HOLD) {
         tmem_fence_before();

@@ -45,6 +45,7 @@ struct BandParams {
     int total_bands;           // batch * nb
     long long total_units;     // bands (band units) or bands*nc (tile units)
     int tile_units;            // 1: one ticket = one tile (external carries)
+    int cluster;               // CTAs per cluster (1, or 8: one ticket = 8 bands)
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)
