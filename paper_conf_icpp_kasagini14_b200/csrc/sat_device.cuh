@@ -101,8 +101,10 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity
     SpinGuard guard;
     while (!mbar_try_wait_cluster(bar, parity)) guard.tick();
 }
+// every thread of every CTA of the cluster (non-.aligned: lanes may arrive
+// from divergent paths)
 __device__ __forceinline__ void cluster_sync_all() {
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
 }
 
 // ------------------------------------------------------------- TMA
