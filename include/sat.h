@@ -173,6 +173,13 @@ int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t 
  * ceil(rows/TH)*batch*ceil(cols/128)*64 bytes; NULL disarms. */
 int sat_debug_trace(void *dev_buf);
 
+/* Debug: record, in host-mapped memory, what every spinning warp waits on
+ * once a wait exceeds half the 4-s watchdog (before the kernel traps);
+ * sat_debug_diag_dump prints the records to stderr (also after a failed
+ * launch) and returns their number. */
+int sat_debug_diag_enable(void);
+int sat_debug_diag_dump(void);
+
 /* Number of kernels launched by the last successful call on this thread. */
 int sat_last_launch_count(void);
 /* Band height used by the last 1R1W-family call on this thread. */

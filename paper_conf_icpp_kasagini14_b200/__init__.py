@@ -55,6 +55,8 @@ _SIGS = {
     "sat_sharded_workspace_bytes": ([_I64, _I, _I], ctypes.c_size_t),
     "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
     "sat_debug_trace": ([_P], _I),
+    "sat_debug_diag_enable": ([], _I),
+    "sat_debug_diag_dump": ([], _I),
     "sat_last_launch_count": ([], _I),
     "sat_last_tile_rows": ([], _I),
     "sat_last_grid": ([], _I),

@@ -837,6 +837,34 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     return SAT_OK;
 }
 
+static unsigned int* g_diag_host = nullptr;
+static const size_t kDiagWords = size_t(4096) * 32 * 4;
+
+int sat_debug_diag_enable(void) {
+    if (!g_diag_host) {
+        CUDA_TRY(cudaHostAlloc(&g_diag_host, kDiagWords * 4, cudaHostAllocMapped));
+        std::memset(g_diag_host, 0, kDiagWords * 4);
+    }
+    unsigned int* dptr = nullptr;
+    CUDA_TRY(cudaHostGetDevicePointer(&dptr, g_diag_host, 0));
+    CUDA_TRY(cudaMemcpyToSymbol(sat::g_sat_diag, &dptr, sizeof(dptr)));
+    return SAT_OK;
+}
+
+int sat_debug_diag_dump(void) {
+    if (!g_diag_host) return 0;
+    int n = 0;
+    for (size_t i = 0; i < kDiagWords; i += 4) {
+        if ((g_diag_host[i + 2] & 0xFFFF0000u) == 0xC0DE0000u) {
+            std::fprintf(stderr, "diag block %u warp %zu thread %u: what 0x%08x extra %u\n",
+                         g_diag_host[i + 2] & 0xFFFFu, (i / 4) % 32, g_diag_host[i + 3],
+                         g_diag_host[i], g_diag_host[i + 1]);
+            ++n;
+        }
+    }
+    return n;
+}
+
 int sat_debug_trace(void* dev_buf) {
     t_trace = static_cast<unsigned long long*>(dev_buf);
     return SAT_OK;

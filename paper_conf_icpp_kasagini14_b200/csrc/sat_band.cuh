@@ -553,7 +553,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     // LBW descriptor rows per round trip
                     uint32_t pend = (1u << CPL) - 1u;
                     int kb = idx - 1;
-                    SpinGuard guard;
+                    SpinGuard guard(0x80000000u | uint32_t(J), uint32_t(gidx));
                     while (pend) {
                         uint64_t wv[LBW][CPL];
 #pragma unroll

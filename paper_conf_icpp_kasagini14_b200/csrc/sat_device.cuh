@@ -48,21 +48,36 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 // the call surfaces as SAT_ERR_CUDA instead of hanging the GPU.
 constexpr unsigned long long kSpinLimitNs = 4000000000ull;   // 4 s
 
+// Debug: when set (sat_debug_diag_enable), a spin that passes half the limit
+// records {what, extra, block, warp} in host-mapped memory before the trap, so
+// a protocol deadlock can be read back after the launch fails.
+__device__ unsigned int* g_sat_diag = nullptr;
+
 struct SpinGuard {
     unsigned long long t0 = 0;
     unsigned n = 0;
+    uint32_t what = 0, extra = 0;
+    __device__ __forceinline__ SpinGuard() {}
+    __device__ __forceinline__ SpinGuard(uint32_t w, uint32_t e) : what(w), extra(e) {}
     __device__ __forceinline__ void tick() {
         if ((++n & 1023u) == 0) {
             const unsigned long long t = globaltimer_ns();
-            if (t0 == 0) t0 = t;
-            else if (t - t0 > kSpinLimitNs) __trap();
+            if (t0 == 0) {
+                t0 = t;
+            } else if (t - t0 > kSpinLimitNs) {
+                __trap();
+            } else if (t - t0 > kSpinLimitNs / 2 && g_sat_diag != nullptr && (n & 0xFFFFFu) == 0) {
+                volatile unsigned int* d = g_sat_diag + (blockIdx.x * 32u + (threadIdx.x >> 5)) * 4u;
+                d[0] = what; d[1] = extra; d[2] = 0xC0DE0000u | blockIdx.x; d[3] = threadIdx.x;
+                __threadfence_system();
+            }
         }
     }
 };
 
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     if (mbar_try_wait(bar, parity)) return;
-    SpinGuard guard;
+    SpinGuard guard(smem_u32(bar), parity);
     while (!mbar_try_wait(bar, parity)) guard.tick();
 }
 
@@ -98,7 +113,7 @@ __device__ __forceinline__ bool mbar_try_wait_cluster(uint64_t* bar, uint32_t pa
 }
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
     if (mbar_try_wait_cluster(bar, parity)) return;
-    SpinGuard guard;
+    SpinGuard guard(smem_u32(bar) | 0x40000000u, parity);
     while (!mbar_try_wait_cluster(bar, parity)) guard.tick();
 }
 // every thread of every CTA of the cluster (non-.aligned: lanes may arrive
