@@ -225,6 +225,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
         // per cluster.  Clusters that cannot be co-resident simply start
         // late and find no ticket left.
         long long ncl = std::min<long long>(p.total_units, (long long)occ * di.sms / CL);
+        if (const char* e = getenv("SAT_DEBUG_NCL")) ncl = atoi(e);
         if (ncl < 1) ncl = 1;
         const long long grid = ncl * CL;
         grid_out = int(grid);
@@ -838,7 +839,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
 }
 
 static unsigned int* g_diag_host = nullptr;
-static const size_t kDiagWords = size_t(4096) * 32 * 4;
+static const size_t kDiagWords = size_t(4096) * 32 * 4 * 2;
 
 int sat_debug_diag_enable(void) {
     if (!g_diag_host) {
@@ -854,7 +855,21 @@ int sat_debug_diag_enable(void) {
 int sat_debug_diag_dump(void) {
     if (!g_diag_host) return 0;
     int n = 0;
-    for (size_t i = 0; i < kDiagWords; i += 4) {
+    for (size_t i = kDiagWords / 2; i < kDiagWords; i += 4) {
+        if ((g_diag_host[i + 2] & 0xFFFF0000u) == 0xC0DE0000u)
+            std::fprintf(stderr, "mark block %u warp %zu: unit %u step %u mark %u\n", g_diag_host[i + 3],
+                         ((i - kDiagWords / 2) / 4) % 32, g_diag_host[i], g_diag_host[i + 1],
+                         g_diag_host[i + 2] & 0xFFFFu);
+    }
+    for (size_t b = 0; b < 4096; ++b) {
+        const unsigned int* h = g_diag_host + kDiagWords / 2 + size_t(4096) * 32 * 2 + b * 16;
+        if (h[15]) {
+            std::fprintf(stderr, "units block %zu:", b);
+            for (unsigned int q = 0; q < h[15] && q < 15; ++q) std::fprintf(stderr, " %u", h[q]);
+            std::fprintf(stderr, "\n");
+        }
+    }
+    for (size_t i = 0; i < kDiagWords / 2; i += 4) {
         if ((g_diag_host[i + 2] & 0xFFFF0000u) == 0xC0DE0000u) {
             std::fprintf(stderr, "diag block %u warp %zu thread %u: what 0x%08x extra %u\n",
                          g_diag_host[i + 2] & 0xFFFFu, (i / 4) % 32, g_diag_host[i + 3],

@@ -340,6 +340,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             __syncthreads();
         }
         const long long unit = *s_unit;
+        diag_mark(uint32_t(unit), 0, 1);
+        if (g_sat_diag != nullptr && threadIdx.x == 0) {
+            // per-block history of units (debug)
+            volatile unsigned int* h = g_sat_diag + 4096u * 32u * 4u + 4096u * 32u * 2u + blockIdx.x * 16u;
+            const unsigned int n = h[15];
+            if (n < 15) { h[n] = uint32_t(unit); h[15] = n + 1; }
+        }
         if (unit >= p.total_units) break;
 
         int gb, j0, j1;
@@ -491,7 +498,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             } else {
                 for (int k = 0; k < nch; ++k) {
                     local(k);
+                    diag_mark(uint32_t(unit), uint32_t(k), 2);
                     if (k >= DT - 1) finish(k - (DT - 1));
+                    diag_mark(uint32_t(unit), uint32_t(k), 3);
                 }
                 for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
             }
@@ -650,7 +659,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                             for (int i = 0; i < CPL; ++i) Sa[i] = Sp[i] + agg[i];
                             if (crank + 1 < CL) send_chain();
-                            else if (pubc) publish_words<T, CPL>(myc, ctag | 1u, Sa);
+                            else if (pubc && cb > 0) publish_words<T, CPL>(myc, ctag | 1u, Sa);
+                            // (cluster-band 0 publishes only its inclusive: a walk
+                            // must never pass row 0 on an aggregate)
                             mbar_wait_cluster(&ctopb[x], ph);
                             lds_cols<T, CPL>(ctop + size_t(x) * TW + cl, top);
                             mbar_arrive_remote(mapa(smem_u32(&ctopfree[x]), 0));
@@ -692,6 +703,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         for (int i = 0; i < CPL; ++i) top[i] += b[i];
                     }
                     mbar_arrive(&topr[it % XS]);
+                    diag_mark(uint32_t(unit), uint32_t(k), 4);
                 }
             }
         } else {
@@ -714,11 +726,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 }
             }
         }
+        diag_mark(uint32_t(unit), uint32_t(nch), 5);
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
         if constexpr (CL > 1) cluster_sync_all();      // before rank 0 overwrites s_unit
         else __syncthreads();
     }
+    diag_mark(0xFFFFFFFFu, 0, 6);
     if (HOLD) {
         tmem_fence_before();
         __syncthreads();

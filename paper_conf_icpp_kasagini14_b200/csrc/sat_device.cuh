@@ -53,9 +53,18 @@ constexpr unsigned long long kSpinLimitNs = 4000000000ull;   // 4 s
 // a protocol deadlock can be read back after the launch fails.
 __device__ unsigned int* g_sat_diag = nullptr;
 
+// progress marks (debug): per (block, warp) the last {unit, step, mark}
+__device__ __forceinline__ void diag_mark(uint32_t unit, uint32_t step, uint32_t mark) {
+    if (g_sat_diag != nullptr && (threadIdx.x & 31) == 0) {
+        volatile unsigned int* d = g_sat_diag + 4096u * 32u * 4u + (blockIdx.x * 32u + (threadIdx.x >> 5)) * 4u;
+        d[0] = unit; d[1] = step; d[2] = 0xC0DE0000u | mark; d[3] = blockIdx.x;
+    }
+}
+
 struct SpinGuard {
     unsigned long long t0 = 0;
     unsigned n = 0;
+    bool logged = false;
     uint32_t what = 0, extra = 0;
     __device__ __forceinline__ SpinGuard() {}
     __device__ __forceinline__ SpinGuard(uint32_t w, uint32_t e) : what(w), extra(e) {}
@@ -66,7 +75,8 @@ struct SpinGuard {
                 t0 = t;
             } else if (t - t0 > kSpinLimitNs) {
                 __trap();
-            } else if (t - t0 > kSpinLimitNs / 2 && g_sat_diag != nullptr && (n & 0xFFFFFu) == 0) {
+            } else if (t - t0 > kSpinLimitNs / 2 && g_sat_diag != nullptr && !logged) {
+                logged = true;
                 volatile unsigned int* d = g_sat_diag + (blockIdx.x * 32u + (threadIdx.x >> 5)) * 4u;
                 d[0] = what; d[1] = extra; d[2] = 0xC0DE0000u | blockIdx.x; d[3] = threadIdx.x;
                 __threadfence_system();
