@@ -384,7 +384,10 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
                 ? launch_band_d<uint32_t>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid)
                 : launch_band_d<float>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid);
     if (s != SAT_OK) return s;
-    ws.next_base += units + (unsigned long long)grid;
+    // every persistent ticket taker (a CTA, or a cluster) makes exactly one
+    // failing fetch, so the counter ends at base + units + takers
+    const unsigned long long takers = (unsigned long long)(p.cluster > 1 ? grid / p.cluster : grid);
+    ws.next_base += units + takers;
     return SAT_OK;
 }
 

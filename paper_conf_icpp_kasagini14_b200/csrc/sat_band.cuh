@@ -341,6 +341,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         }
         const long long unit = *s_unit;
         diag_mark(uint32_t(unit), 0, 1);
+        if (unit < 0) __trap();                       // ticket accounting out of sync: never silently
         if (g_sat_diag != nullptr && threadIdx.x == 0) {
             // per-block history of units (debug)
             volatile unsigned int* h = g_sat_diag + 4096u * 32u * 4u + 4096u * 32u * 2u + blockIdx.x * 16u;

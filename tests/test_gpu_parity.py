@@ -308,3 +308,51 @@ def test_cfg4_65536_properties(libsat):
         with np.errstate(over="ignore"):
             rec = w[1, 1] - w[0, 1] - w[1, 0] + w[0, 0]
         assert rec == np.uint32(int(x[i, j]) & 0xFFFFFFFF)
+
+
+# ------------------------------------------------------------------ clusters (DSMEM carry chain)
+@pytest.mark.parametrize("shape,th", [((1024, 1024), 64), ((512, 700), 64), ((2048, 4096), 64),
+                                      ((9 * 64, 1280), 64), ((170 * 64, 256), 64),
+                                      ((8 * 48, 2000), 48), ((160 * 48 + 5, 384), 48)])
+def test_cluster_path(libsat, shape, th):
+    """Shapes that take the 8-CTA cluster path (nb % 8 == 0 or nb >= 160,
+    including padded virtual bands) -- several clusters run concurrently and
+    look back over each other's cluster-band descriptors."""
+    for dtype in ("int32", "float32"):
+        a = gen(*shape, dtype, seed=shape[0] + th)
+        check(libsat.sat(dev(a), tile_rows=th), oracle.sat(a), dtype)
+
+
+def test_cluster_repeat_and_jitter(libsat):
+    a = gen(4096, 2048, "int32", seed=41)
+    ref = oracle.sat(a)
+    x = dev(a)
+    for _ in range(5):
+        check(libsat.sat(x, tile_rows=64), ref, "int32")
+    check(libsat.sat(x, tile_rows=64, jitter=20000), ref, "int32")
+
+
+def test_cluster_batched_and_seeded(libsat):
+    a = make_np(512, 640, "int32", "u32", seed=42, batch=3)       # 8 bands per image
+    y = libsat.sat_batched(dev(a), tile_rows=64).cpu().numpy()
+    for b in range(3):
+        check(y[b], oracle.sat(a[b]), "int32")
+    full = gen(64 * 40, 900, "int32", seed=43)
+    ref = oracle.sat(full)
+    r0 = 64 * 8
+    carry = oracle.column_totals(full[:r0])
+    check(libsat.sat_seeded(dev(full[r0:]), carry_row=dev(carry)), ref[r0:], "int32")
+
+
+def test_debug_trace_records_events(libsat):
+    a = gen(640, 1024, "int32", seed=44)
+    x = dev(a)
+    nb, nc = 10, 8
+    buf = torch.zeros(nb * nc * 8, dtype=torch.int64, device="cuda")
+    libsat.debug_trace(buf)
+    y = libsat.sat(x, tile_rows=64)
+    torch.cuda.synchronize()
+    check(y, oracle.sat(a), "int32")
+    t = buf.view(nb, nc, 8).cpu().numpy()
+    assert (t[:, :, 0] != 0).all() and (t[:, :, 2] != 0).all()
+    assert libsat.last_grid() >= 1
