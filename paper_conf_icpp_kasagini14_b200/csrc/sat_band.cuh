@@ -270,20 +270,21 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     extern __shared__ __align__(1024) uint8_t smem[];
     T* tiles = reinterpret_cast<T*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
-    T* chain = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);        // [XS][TW] (CL > 1)
-    T* ctop = chain + size_t(XS) * TW;                                    // [XS][TW] (CL > 1)
+    T* cagg = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);         // [XS][TW] own aggregate (CL > 1)
+    T* ctop = cagg + size_t(XS) * TW;                                     // [XS][TW] top from rank 0 (CL > 1)
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf + SM::cbuf);
     uint64_t* full = bars;              // [S]  TMA load landed (tx count)
     uint64_t* empty = bars + S;         // [S]  every compute warp read the slot
     uint64_t* colr = bars + 2 * S;      // [XS] every compute warp published its bottom row
     uint64_t* topr = bars + 2 * S + XS; // [XS] the control warp wrote the add vectors
-    // clusters (CL > 1), per carry slot: chainb = partial aggregate from rank-1
-    // arrived; chainfree = rank+1 consumed ours; ctopb = cluster top row from
-    // rank 0 arrived; ctopfree (rank 0) = every other rank consumed it
-    uint64_t* chainb = bars + 2 * S + 2 * XS;
-    uint64_t* chainfree = chainb + XS;
-    uint64_t* ctopb = chainb + 2 * XS;
-    uint64_t* ctopfree = chainb + 3 * XS;
+    // clusters (CL > 1), per carry slot: aggb = the aggregates of every lower
+    // rank are readable; aggfree = every higher rank has read ours; ctopb =
+    // the cluster's top row from rank 0 arrived; ctopfree (rank 0) = every
+    // other rank read it
+    uint64_t* aggb = bars + 2 * S + 2 * XS;
+    uint64_t* aggfree = aggb + XS;
+    uint64_t* ctopb = aggb + 2 * XS;
+    uint64_t* ctopfree = aggb + 3 * XS;
     long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
     uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 1);
     const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
@@ -300,8 +301,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             mbar_init(&colr[x], W * 32);
             mbar_init(&topr[x], 32 * NS);
             if constexpr (CL > 1) {
-                mbar_init(&chainb[x], 32);
-                mbar_init(&chainfree[x], 32);
+                const uint32_t rk = cluster_ctarank();
+                mbar_init(&aggb[x], rk > 0 ? 32 * rk : 1);
+                mbar_init(&aggfree[x], rk + 1 < CL ? 32 * (CL - 1 - rk) : 1);
                 mbar_init(&ctopb[x], 32);
                 mbar_init(&ctopfree[x], 32 * (CL - 1));
             }
@@ -622,29 +624,37 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         }
                     };
                     if constexpr (CL > 1) {
-                        // Cluster of CL bands (DSMEM): the
-                        // partial aggregates S_r = agg_0 + .. + agg_r run down a
-                        // chain rank 0 -> 1 -> .. -> CL-1; rank 0 looks back over
-                        // the cluster-band descriptors and broadcasts the SAT row
-                        // T above the cluster; rank r's top = T + S_{r-1}; rank
-                        // CL-1 publishes the cluster's aggregate S_{CL-1} and
-                        // inclusive T + S_{CL-1}.
+                        // Cluster of CL bands (DSMEM): every
+                        // rank leaves its chunk aggregate in its own smem and
+                        // signals the higher ranks; rank r sums the aggregates
+                        // of ranks < r straight from their smem (one DSMEM round
+                        // trip); rank 0 looks back over the cluster-band
+                        // descriptors and broadcasts the SAT row T above the
+                        // cluster; rank r's top = T + S_{r-1}; the last rank
+                        // publishes the cluster's aggregate and inclusive.
                         const uint32_t x = it % XS, ph = (it / XS) & 1u;
                         const int upi = (p.nb + CL - 1) / CL;
                         const bool pubc = cb + 1 < upi;
                         uint64_t* myc = p.desc + int64_t(gcb) * desc_w + c0;
                         const uint32_t ctag = band_tag(p.base, gcb);
-                        T Sa[CPL] = {}, Sp[CPL] = {};
-                        auto send_chain = [&]() {
-                            if (it >= uint32_t(XS)) mbar_wait_cluster(&chainfree[x], ph ^ 1u);
-                            st_cluster_v4(mapa(smem_u32(chain + size_t(x) * TW + cl), crank + 1),
-                                          to_bits(Sa[0]), to_bits(Sa[1]), to_bits(Sa[2]), to_bits(Sa[3]));
-                            mbar_arrive_remote(mapa(smem_u32(&chainb[x]), crank + 1));
-                        };
+                        T Sp[CPL] = {};
+                        if (crank + 1 < CL) {
+                            if (it >= uint32_t(XS)) mbar_wait_cluster(&aggfree[x], ph ^ 1u);
+                            sts_cols<T, CPL>(cagg + size_t(x) * TW + cl, agg);
+                            for (uint32_t r2 = crank + 1; r2 < CL; ++r2)
+                                mbar_arrive_remote(mapa(smem_u32(&aggb[x]), r2));
+                        }
+                        if (crank > 0) {
+                            mbar_wait_cluster(&aggb[x], ph);
+                            for (uint32_t r2 = 0; r2 < crank; ++r2) {
+                                const uint4 u = ld_cluster_v4(mapa(smem_u32(cagg + size_t(x) * TW + cl), r2));
+                                Sp[0] += from_bits<T>(u.x); Sp[1] += from_bits<T>(u.y);
+                                Sp[2] += from_bits<T>(u.z); Sp[3] += from_bits<T>(u.w);
+                            }
+                            for (uint32_t r2 = 0; r2 < crank; ++r2)
+                                mbar_arrive_remote(mapa(smem_u32(&aggfree[x]), r2));
+                        }
                         if (crank == 0) {
-#pragma unroll
-                            for (int i = 0; i < CPL; ++i) { Sa[i] = agg[i]; Sp[i] = T(0); }
-                            send_chain();
                             if (cb == 0) seed_row(top);
                             else walk(gcb, cb, top);
                             if (it >= uint32_t(XS)) mbar_wait_cluster(&ctopfree[x], ph ^ 1u);
@@ -654,15 +664,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                 mbar_arrive_remote(mapa(smem_u32(&ctopb[x]), r2));
                             }
                         } else {
-                            mbar_wait_cluster(&chainb[x], ph);
-                            lds_cols<T, CPL>(chain + size_t(x) * TW + cl, Sp);
-                            mbar_arrive_remote(mapa(smem_u32(&chainfree[x]), crank - 1));
+                            T Sa[CPL];
 #pragma unroll
                             for (int i = 0; i < CPL; ++i) Sa[i] = Sp[i] + agg[i];
-                            if (crank + 1 < CL) send_chain();
-                            else if (pubc && cb > 0) publish_words<T, CPL>(myc, ctag | 1u, Sa);
                             // (cluster-band 0 publishes only its inclusive: a walk
                             // must never pass row 0 on an aggregate)
+                            if (crank + 1 == CL && pubc && cb > 0) publish_words<T, CPL>(myc, ctag | 1u, Sa);
                             mbar_wait_cluster(&ctopb[x], ph);
                             lds_cols<T, CPL>(ctop + size_t(x) * TW + cl, top);
                             mbar_arrive_remote(mapa(smem_u32(&ctopfree[x]), 0));
