@@ -339,15 +339,14 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.nc = int((j.cols + TW - 1) / TW);
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * p.nc : p.total_bands;
-    // Clusters of 8 bands pass the vertical carry through DSMEM (DESIGN.md
-    // Sec. 4.5): plain 1R1W on the TMA path, when few virtual bands pad the
-    // last cluster of each image.
+    // Clusters of 8 bands that pass the vertical carry through DSMEM (DESIGN.md
+    // Sec. 4.5) are correct but measured slower than the plain look-back, so
+    // they are opt-in (SAT_CLUSTER=8) for plain 1R1W on the TMA path.
     p.cluster = 1;
-    if (mode == MODE_SAT && j.tma && p.region == REG_ALL && p.top_src == TOP_LOOKBACK &&
-        !p.tile_units && (j.th == 64 || j.th == 48) && (p.nb % 8 == 0 || p.nb >= 160))
-        p.cluster = 8;
-    if (const char* e = getenv("SAT_DEBUG_CL")) {
-        if (atoi(e) <= 1) p.cluster = 1;
+    if (const char* e = getenv("SAT_CLUSTER")) {
+        if (atoi(e) == 8 && mode == MODE_SAT && j.tma && p.region == REG_ALL &&
+            p.top_src == TOP_LOOKBACK && !p.tile_units && (j.th == 64 || j.th == 48))
+            p.cluster = 8;
     }
     if (p.cluster > 1)
         p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);

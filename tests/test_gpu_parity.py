@@ -314,16 +314,18 @@ def test_cfg4_65536_properties(libsat):
 @pytest.mark.parametrize("shape,th", [((1024, 1024), 64), ((512, 700), 64), ((2048, 4096), 64),
                                       ((9 * 64, 1280), 64), ((170 * 64, 256), 64),
                                       ((8 * 48, 2000), 48), ((160 * 48 + 5, 384), 48)])
-def test_cluster_path(libsat, shape, th):
-    """Shapes that take the 8-CTA cluster path (nb % 8 == 0 or nb >= 160,
-    including padded virtual bands) -- several clusters run concurrently and
-    look back over each other's cluster-band descriptors."""
+def test_cluster_path(libsat, shape, th, monkeypatch):
+    """The opt-in 8-CTA cluster path (SAT_CLUSTER=8), including padded virtual
+    bands -- several clusters run concurrently and look back over each other's
+    cluster-band descriptors."""
+    monkeypatch.setenv("SAT_CLUSTER", "8")
     for dtype in ("int32", "float32"):
         a = gen(*shape, dtype, seed=shape[0] + th)
         check(libsat.sat(dev(a), tile_rows=th), oracle.sat(a), dtype)
 
 
-def test_cluster_repeat_and_jitter(libsat):
+def test_cluster_repeat_and_jitter(libsat, monkeypatch):
+    monkeypatch.setenv("SAT_CLUSTER", "8")
     a = gen(4096, 2048, "int32", seed=41)
     ref = oracle.sat(a)
     x = dev(a)
@@ -332,7 +334,8 @@ def test_cluster_repeat_and_jitter(libsat):
     check(libsat.sat(x, tile_rows=64, jitter=20000), ref, "int32")
 
 
-def test_cluster_batched_and_seeded(libsat):
+def test_cluster_batched_and_seeded(libsat, monkeypatch):
+    monkeypatch.setenv("SAT_CLUSTER", "8")
     a = make_np(512, 640, "int32", "u32", seed=42, batch=3)       # 8 bands per image
     y = libsat.sat_batched(dev(a), tile_rows=64).cpu().numpy()
     for b in range(3):

@@ -18,3 +18,4 @@ done
 for th in 64; do
   timeout 120 python tools/trace_lookback.py 16384 16384 $th gpurun_out/trace16k_$th.npz >> gpurun_out/trace.log 2>&1
 done
+python tools/trace_lookback.py 16384 16384 64 gpurun_out/trace16k_cl.npz >> gpurun_out/trace.log 2>&1
