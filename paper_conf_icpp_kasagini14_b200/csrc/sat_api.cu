@@ -271,6 +271,8 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         }
     }
     if constexpr (MODE == MODE_SAT && TMA) {
+        if (p.big && th == 64)   // 192 KB ring of 64 x 256 slots, 6 chunks parked in TMEM
+            return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1>(p, ti, to, di, st, grid);
         if (p.cluster == 8 && th == 64)
             return launch_band_t<T, 8, 8, 3, 3, 1, 3, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
         if (p.cluster == 8 && th == 48)
@@ -348,6 +350,12 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
             p.top_src == TOP_LOOKBACK && !p.tile_units && (j.th == 64 || j.th == 48))
             p.cluster = 8;
     }
+    // Many bands (>= 4 waves of one CTA per SM): one CTA per SM with twice the
+    // ring and 1-KB row segments per TMA load.
+    p.big = (mode == MODE_SAT && j.tma && p.cluster == 1 && j.th == 64 &&
+             p.total_bands >= 4 * j.di->sms) ? 1 : 0;
+    if (const char* e = getenv("SAT_BIG")) p.big = (atoi(e) != 0 && mode == MODE_SAT && j.tma &&
+                                                    p.cluster == 1 && j.th == 64) ? 1 : 0;
     if (p.cluster > 1)
         p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
     p.jitter = j.jitter;

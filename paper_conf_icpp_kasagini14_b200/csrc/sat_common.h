@@ -46,6 +46,7 @@ struct BandParams {
     long long total_units;     // bands (band units) or bands*nc (tile units)
     int tile_units;            // 1: one ticket = one tile (external carries)
     int cluster;               // CTAs per cluster (1, or 8: one ticket = 8 bands)
+    int big;                   // 1: one CTA per SM with a 2x ring of 1-KB row segments (TH 64)
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)

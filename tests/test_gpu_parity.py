@@ -359,3 +359,13 @@ def test_debug_trace_records_events(libsat):
     t = buf.view(nb, nc, 8).cpu().numpy()
     assert (t[:, :, 0] != 0).all() and (t[:, :, 2] != 0).all()
     assert libsat.last_grid() >= 1
+
+
+@pytest.mark.parametrize("shape", [(1000, 1300), (64 * 40 + 7, 2048), (4096, 777 * 4)])
+def test_big_ring_config(libsat, shape, monkeypatch):
+    """TH=64 with one CTA per SM and 1-KB row segments per TMA load (the
+    configuration chosen automatically for >= 4 waves of bands)."""
+    monkeypatch.setenv("SAT_BIG", "1")
+    for dtype in ("int32", "float32"):
+        a = gen(*shape, dtype, seed=shape[0])
+        check(libsat.sat(dev(a), tile_rows=64), oracle.sat(a), dtype)
