@@ -33,6 +33,7 @@ thread_local int t_th = 0;
 thread_local int t_grid = 0;
 thread_local double t_r = 0.0;
 thread_local unsigned long long* t_trace = nullptr;
+static unsigned int* g_diag_dev = nullptr;   // sat_debug_diag_enable (device view)
 
 int fail(int code, const std::string& msg) {
     t_err = msg;
@@ -192,13 +193,16 @@ constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 1, 2};
 constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
 constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 1, 2};
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
+// TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
+// all 512 columns); half the descriptor bytes and look-back hops per element
+constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int CL = 1>
+          int CL = 1, int LBW = 0>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
     (void)to;
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB>;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB, LBW>;
     const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
@@ -271,8 +275,15 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         }
     }
     if constexpr (MODE == MODE_SAT && TMA) {
-        if (p.big && th == 64)   // 192 KB ring of 64 x 256 slots, 6 chunks parked in TMEM
+        if (p.big && th == 64) {  // 192 KB ring of 64 x 256 slots, 6 chunks parked in TMEM
+            if (const char* e = getenv("SAT_DEBUG_LBW")) {
+                const int lbw = atoi(e);
+                if (lbw == 8) return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
+                if (lbw == 12) return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1, 1, 12>(p, ti, to, di, st, grid);
+                if (lbw == 83) return launch_band_t<T, 8, 8, 3, 6, 2, 8, 2, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
+            }
             return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1>(p, ti, to, di, st, grid);
+        }
         if (p.cluster == 8 && th == 64)
             return launch_band_t<T, 8, 8, 3, 3, 1, 3, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
         if (p.cluster == 8 && th == 48)
@@ -283,8 +294,9 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
         case 48: return launch_band_t<T, SAT_CFG(kCfg48), MODE, TMA, kCfg48.MINB>(p, ti, to, di, st, grid);
         case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
+        case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
     }
-    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48 or 64");
+    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64 or 128");
 }
 
 template <typename T, int MODE>
@@ -308,7 +320,15 @@ int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtenso
 // Automatic band height: the tallest band that still gives roughly one band
 // per resident CTA slot (the look-back chain is per band; more, shorter bands
 // raise parallelism, taller bands cut descriptor traffic).
-int auto_th(int64_t rows, int64_t batch, const DevInfo& di) {
+int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant) {
+    // 1R1W: TH = 128 (one CTA per SM) when its bands fill one wave (16K^2,
+    // 18432^2: measured 5.3-5.4 TB/s vs 5.0 for TH = 64); with several waves
+    // the fractional last wave of 128-row bands costs more than the extra
+    // descriptor traffic of TH = 64 (65536^2: 6.40 ms vs 6.51 ms).
+    if (variant == SAT_1R1W) {
+        const long long b128 = batch * ((rows + 127) / 128);
+        if (b128 * 5 >= 4LL * di.sms && b128 <= di.sms) return 128;
+    }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
     for (int th : {64, 32}) {
         const long long bands = batch * ((rows + th - 1) / th);
@@ -359,6 +379,8 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     if (p.cluster > 1)
         p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
     p.jitter = j.jitter;
+    p.diag = g_diag_dev;
+    if (const char* e = getenv("SAT_DEBUG_NOLB")) p.dbg = atoi(e);   // 1: no look-back, 2: publish only
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
         p.trace = t_trace;
         t_trace = nullptr;
@@ -505,8 +527,8 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     sat_options_init(&o);
     if (opt) o = *opt;
     if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 48 &&
-        o.tile_rows != 64)
-        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48 or 64");
+        o.tile_rows != 64 && o.tile_rows != 128)
+        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48, 64 or 128");
     if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     int dev;
@@ -516,7 +538,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     SAT_TRY(get_ws(dev, st, ws));
     Job j;
     j.in = in; j.out = out; j.batch = batch; j.rows = rows; j.cols = cols; j.dtype = dtype;
-    j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di);
+    j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant);
     j.tma = !o.force_generic && tma_ok(in, out, cols);
     j.jitter = o.jitter;
     j.di = &di;
@@ -859,6 +881,7 @@ int sat_debug_diag_enable(void) {
     unsigned int* dptr = nullptr;
     CUDA_TRY(cudaHostGetDevicePointer(&dptr, g_diag_host, 0));
     CUDA_TRY(cudaMemcpyToSymbol(sat::g_sat_diag, &dptr, sizeof(dptr)));
+    g_diag_dev = static_cast<unsigned int*>(dptr);
     return SAT_OK;
 }
 

@@ -247,7 +247,8 @@ struct TmemCols {
     static_assert(need <= 512, "TMEM holds at most 512 columns");
 };
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int CL, int MODE, bool TMA, int MINB>
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int CL, int MODE, bool TMA, int MINB,
+          int LBW_ = 0>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -342,11 +343,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             __syncthreads();
         }
         const long long unit = *s_unit;
-        diag_mark(uint32_t(unit), 0, 1);
+        diag_mark(p.diag, uint32_t(unit), 0, 1);
         if (unit < 0) __trap();                       // ticket accounting out of sync: never silently
-        if (g_sat_diag != nullptr && threadIdx.x == 0) {
+        if (p.diag != nullptr && threadIdx.x == 0) {
             // per-block history of units (debug)
-            volatile unsigned int* h = g_sat_diag + 4096u * 32u * 4u + 4096u * 32u * 2u + blockIdx.x * 16u;
+            volatile unsigned int* h = p.diag + 4096u * 32u * 4u + 4096u * 32u * 2u + blockIdx.x * 16u;
             const unsigned int n = h[15];
             if (n < 15) { h[n] = uint32_t(unit); h[15] = n + 1; }
         }
@@ -501,9 +502,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             } else {
                 for (int k = 0; k < nch; ++k) {
                     local(k);
-                    diag_mark(uint32_t(unit), uint32_t(k), 2);
+                    diag_mark(p.diag, uint32_t(unit), uint32_t(k), 2);
                     if (k >= DT - 1) finish(k - (DT - 1));
-                    diag_mark(uint32_t(unit), uint32_t(k), 3);
+                    diag_mark(p.diag, uint32_t(unit), uint32_t(k), 3);
                 }
                 for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
             }
@@ -521,7 +522,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if constexpr (HOLD) {
                 constexpr int CPL = 4 / NS;
                 constexpr int G = NCW / NS;
-                constexpr int LBW = 16 / CPL;
+                constexpr int LBW = LBW_ > 0 ? LBW_ : 16 / CPL;   // bands per look-back round trip
                 const int cw = warp - CW;
                 const int grp = cw / NS;
                 const int cl = (cw % NS) * (TW / NS) + lane * CPL;   // column within the chunk
@@ -683,15 +684,18 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             for (int i = 0; i < CPL; ++i) top[i] += Sp[i];
                         }
                     } else {
-                        if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
-                        if (!lookback) {
+                        if (p.dbg & 1) {
+                            // timing probe only: no vertical carry
+                        } else if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                        if (p.dbg & 1) {
+                        } else if (!lookback) {
                             lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
                         } else if (band == 0) {
                             seed_row(top);
-                        } else {
+                        } else if (!(p.dbg & 2)) {
                             walk(gb, band, top);
                         }
-                        if (publish) {
+                        if (publish && !(p.dbg & 1)) {
                             T inc[CPL];
 #pragma unroll
                             for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
@@ -711,7 +715,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         for (int i = 0; i < CPL; ++i) top[i] += b[i];
                     }
                     mbar_arrive(&topr[it % XS]);
-                    diag_mark(uint32_t(unit), uint32_t(k), 4);
+                    diag_mark(p.diag, uint32_t(unit), uint32_t(k), 4);
                 }
             }
         } else {
@@ -734,13 +738,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 }
             }
         }
-        diag_mark(uint32_t(unit), uint32_t(nch), 5);
+        diag_mark(p.diag, uint32_t(unit), uint32_t(nch), 5);
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
         if constexpr (CL > 1) cluster_sync_all();      // before rank 0 overwrites s_unit
         else __syncthreads();
     }
-    diag_mark(0xFFFFFFFFu, 0, 6);
+    diag_mark(p.diag, 0xFFFFFFFFu, 0, 6);
     if (HOLD) {
         tmem_fence_before();
         __syncthreads();

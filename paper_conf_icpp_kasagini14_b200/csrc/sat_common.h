@@ -59,7 +59,9 @@ struct BandParams {
     const void* TopX;          // [total_bands][nc*TW] external SAT row above, nullable
     void* Lb;                  // [total_bands*TH] band-final row carry out, nullable
     int jitter;                // debug: random publish delay (ns scale), 0 = off
+    int dbg;                   // debug: bit 0 = skip look-back and publication (top = 0; WRONG results, timing only)
     unsigned long long* trace; // debug: [total_bands*nc][4] event times (ns), nullable
+    unsigned int* diag;        // debug: host-mapped progress marks (sat_debug_diag_enable), nullable
 };
 
 }  // namespace sat
