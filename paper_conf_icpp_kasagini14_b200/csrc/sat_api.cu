@@ -115,6 +115,7 @@ constexpr unsigned long long kTagSpace = 1ull << 30;
 
 struct Workspace {
     Buf desc;                 // look-back descriptors (zeroed when (re)allocated)
+    Buf lseg;                 // band-segment row carries (zeroed when (re)allocated)
     Buf ticket;               // unsigned long long counter
     unsigned long long next_base = 0;
     Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
@@ -321,13 +322,12 @@ int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtenso
 // per resident CTA slot (the look-back chain is per band; more, shorter bands
 // raise parallelism, taller bands cut descriptor traffic).
 int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant) {
-    // 1R1W: TH = 128 (one CTA per SM) when its bands fill one wave (16K^2,
-    // 18432^2: measured 5.3-5.4 TB/s vs 5.0 for TH = 64); with several waves
-    // the fractional last wave of 128-row bands costs more than the extra
-    // descriptor traffic of TH = 64 (65536^2: 6.40 ms vs 6.51 ms).
+    // 1R1W: TH = 128 (one CTA per SM) once its bands fill a wave (16K^2,
+    // 18432^2: measured 5.3-5.4 TB/s vs 5.0 for TH = 64; 65536^2 with band
+    // segments: 5.97 ms vs 6.27 ms for TH = 64).
     if (variant == SAT_1R1W) {
         const long long b128 = batch * ((rows + 127) / 128);
-        if (b128 * 5 >= 4LL * di.sms && b128 <= di.sms) return 128;
+        if (b128 * 5 >= 4LL * di.sms) return 128;
     }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
     for (int th : {64, 32}) {
@@ -378,6 +378,24 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
                                                     p.cluster == 1 && j.th == 64) ? 1 : 0;
     if (p.cluster > 1)
         p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
+    // Band segments: short units for the last wave when
+    // bands are many waves deep
+    p.nseg = 1;
+    p.segc = p.nc;
+    if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && p.region == REG_ALL && !p.tile_units &&
+        p.cluster == 1 && p.Lx == nullptr && p.Lb == nullptr) {
+        // >= 2 waves of bands: ~16 segments of >= 32 chunks (65536^2, TH 128:
+        // 5.97 ms with 16 segments vs 6.34 ms whole bands); one wave: whole
+        // bands (a segment would wait for the band's previous segment)
+        const int slots = j.di->sms * ((j.th == 128 || p.big) ? 1 : 2);
+        int want = p.total_bands >= 2 * slots ? std::min(16, p.nc / 32) : 1;
+        if (const char* e = getenv("SAT_SEG")) want = std::max(1, atoi(e));
+        if (want > 1 && p.nc > 1) {
+            p.segc = (p.nc + want - 1) / want;
+            p.nseg = (p.nc + p.segc - 1) / p.segc;
+            p.total_units = (long long)p.total_bands * p.nseg;
+        }
+    }
     p.jitter = j.jitter;
     p.diag = g_diag_dev;
     if (const char* e = getenv("SAT_DEBUG_NOLB")) p.dbg = atoi(e);   // 1: no look-back, 2: publish only
@@ -391,15 +409,18 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         SAT_TRY(ensure(ws.desc, need, true));
     }
     SAT_TRY(ensure(ws.ticket, sizeof(unsigned long long), true));
+    if (p.nseg > 1) SAT_TRY(ensure(ws.lseg, size_t(p.total_bands) * j.th * sizeof(uint64_t), true));
     const unsigned long long units = (unsigned long long)p.total_units;
     const unsigned long long worst = units + 4096ull * 64ull;   // units + max grid
     if (ws.next_base + worst >= kTagSpace) {
         // tag space exhausted: clear descriptors and the counter (rare)
         if (ws.desc.p) CUDA_TRY(cudaMemsetAsync(ws.desc.p, 0, ws.desc.bytes, j.st));
+        if (ws.lseg.p) CUDA_TRY(cudaMemsetAsync(ws.lseg.p, 0, ws.lseg.bytes, j.st));
         CUDA_TRY(cudaMemsetAsync(ws.ticket.p, 0, sizeof(unsigned long long), j.st));
         ws.next_base = 0;
     }
     p.desc = static_cast<uint64_t*>(ws.desc.p);
+    p.Lseg = static_cast<uint64_t*>(ws.lseg.p);
     p.ticket = static_cast<unsigned long long*>(ws.ticket.p);
     p.base = ws.next_base;
     CUtensorMap ti, to;

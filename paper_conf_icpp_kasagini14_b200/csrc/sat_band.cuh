@@ -355,6 +355,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 
         int gb, j0, j1;
         int gcb = 0, cb = 0;                           // cluster-band (CL > 1)
+        int seg = 0;                                   // band segment (p.nseg > 1)
         if constexpr (CL > 1) {
             const int upi = (p.nb + CL - 1) / CL;       // cluster-bands per image
             gcb = int(unit);
@@ -368,6 +369,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             int r0, r1;
             region_range(p.region, p.tA, p.nb, p.nc, gb % p.nb, r0, r1);
             j0 = J; j1 = (J >= r0 && J < r1) ? J + 1 : J;
+        } else if (p.nseg > 1) {
+            seg = int(unit / p.total_bands);
+            gb = int(unit - (long long)seg * p.total_bands);
+            j0 = seg * p.segc;
+            j1 = min(p.nc, j0 + p.segc);
         } else {
             gb = int(unit);
             region_range(p.region, p.tA, p.nb, p.nc, gb % p.nb, j0, j1);
@@ -389,6 +395,24 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                               + int64_t(gb) * TH + rbase;
 #pragma unroll
                 for (int r = 0; r < R; ++r) L[r] = lx[r];
+            }
+            if (seg > 0) {
+                // row carry from segment seg-1 of this band (an earlier ticket,
+                // normally long finished): lane r < R polls row rbase + r
+                const uint32_t want = band_tag(p.base, (seg - 1) * p.total_bands + gb) | 3u;
+                const uint64_t* q = p.Lseg + int64_t(gb) * TH + rbase + (lane < R ? lane : 0);
+                uint64_t wv;
+                asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(wv) : "l"(q) : "memory");
+                if (__any_sync(0xffffffffu, lane < R && uint32_t(wv >> 32) != want)) {
+                    SpinGuard guard(0x20000000u | uint32_t(gb), uint32_t(seg));
+                    while (__any_sync(0xffffffffu, lane < R && uint32_t(wv >> 32) != want)) {
+                        __nanosleep(64);
+                        guard.tick();
+                        asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(wv) : "l"(q) : "memory");
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < R; ++r) L[r] = from_bits<T>(__shfl_sync(0xffffffffu, uint32_t(wv), r));
             }
             const T* gin = reinterpret_cast<const T*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
@@ -507,6 +531,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     diag_mark(p.diag, uint32_t(unit), uint32_t(k), 3);
                 }
                 for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
+            }
+            if (p.nseg > 1 && seg + 1 < p.nseg && lane < R) {
+                // hand the row carry to segment seg+1 of this band
+                T mine = L[0];
+#pragma unroll
+                for (int r = 1; r < R; ++r) if (lane == r) mine = L[r];
+                const uint64_t w = (uint64_t(band_tag(p.base, seg * p.total_bands + gb) | 3u) << 32) | to_bits(mine);
+                asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" :: "l"(p.Lseg + int64_t(gb) * TH + rbase + lane), "l"(w) : "memory");
             }
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;

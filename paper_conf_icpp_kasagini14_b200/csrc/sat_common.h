@@ -62,6 +62,13 @@ struct BandParams {
     int dbg;                   // debug: bit 0 = skip look-back and publication (top = 0; WRONG results, timing only)
     unsigned long long* trace; // debug: [total_bands*nc][4] event times (ns), nullable
     unsigned int* diag;        // debug: host-mapped progress marks (sat_debug_diag_enable), nullable
+    // Band segments (plain 1R1W, many waves): a ticket is (segment s, band b),
+    // segment-major, so the last wave holds short units.  Segment s covers
+    // chunks [s*segc, (s+1)*segc); the row carry L of band b crosses from
+    // segment s-1 to s through Lseg (tagged 64-bit words).
+    int nseg;                  // 1 = whole bands
+    int segc;                  // chunks per segment
+    uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
 };
 
 }  // namespace sat
