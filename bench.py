@@ -375,6 +375,12 @@ def main():
         alg_bytes = 4 * eb * my_elems
     elif variant == "2r1w":
         alg_bytes = 3 * eb * my_elems
+    elif variant == "1+rr1w":                          # (2 + r_eff) eb, Theorem 7
+        alg_bytes = int((2 + libsat.last_r_effective()) * eb * my_elems)
+    elif variant == "4r4w":                            # four read+write passes, Lemma 3
+        alg_bytes = 8 * eb * my_elems
+    elif variant == "4r1w":                            # Formula (1): 4 reads + 1 write, Lemma 5
+        alg_bytes = 5 * eb * my_elems
     achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9
     traffic = ncu_traffic(f"{cfg_key}:{variant}:n{world}")
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",

@@ -66,8 +66,17 @@ typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1 } sat_dtype;
  *                   band C, 2R1W on the bottom-right triangle B (Sec. VII,
  *                   P:L2289-L2355, Theorem 7); r from sat_options (0.25 =
  *                   the paper's 1.25R1W).
+ *   SAT_4R4W        column-wise prefix pass, transpose, column-wise prefix
+ *                   pass, transpose: four coalesced read+write passes (Sec. IV,
+ *                   P:L1081-L1085, Lemma 3).  Needs a rows*cols*4-byte
+ *                   workspace (allocated on first use per stream).
+ *   SAT_4R1W        Formula (1) b[i][j] = a[i][j] + b[i-1][j] + b[i][j-1]
+ *                   - b[i-1][j-1] one anti-diagonal per launch, rows+cols-1
+ *                   launches (Sec. VI, Lemma 5).  Float32 loses
+ *                   accuracy to the subtraction (R16); batch <= 65535.
  */
-typedef enum { SAT_2R2W = 0, SAT_2R1W = 1, SAT_1R1W = 2, SAT_1PLUSR_R1W = 3 } sat_variant;
+typedef enum { SAT_2R2W = 0, SAT_2R1W = 1, SAT_1R1W = 2, SAT_1PLUSR_R1W = 3,
+               SAT_4R4W = 4, SAT_4R1W = 5 } sat_variant;
 
 typedef enum {
     SAT_OK = 0,

@@ -22,7 +22,7 @@ if not os.path.exists(_LIB_PATH):
 _lib = ctypes.CDLL(_LIB_PATH)
 
 SAT_INT32, SAT_FLOAT32 = 0, 1
-VARIANTS = {"2r2w": 0, "2r1w": 1, "1r1w": 2, "1+rr1w": 3}
+VARIANTS = {"2r2w": 0, "2r1w": 1, "1r1w": 2, "1+rr1w": 3, "4r4w": 4, "4r1w": 5}
 SAT_OK = 0
 
 

@@ -22,6 +22,7 @@
 #include "../../include/sat.h"
 #include "sat_aux.cuh"
 #include "sat_band.cuh"
+#include "sat_paper.cuh"
 
 using namespace sat;
 
@@ -119,6 +120,7 @@ struct Workspace {
     Buf ticket;               // unsigned long long counter
     unsigned long long next_base = 0;
     Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
+    Buf tr;                   // 4R4W transposed copy
     Buf part;                 // column totals partials
     Buf seedrow;              // seeded mode: SAT row above the strip
     Buf shard;                // sharded default workspace
@@ -537,13 +539,63 @@ int choose_tA(int nb, int nc, double r, double& r_eff) {
     return best;
 }
 
+// ------------------------------------------------------------------ 4R4W / 4R1W (Table II columns)
+template <typename T>
+int transpose_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols, cudaStream_t st) {
+    const int64_t ntr = (rows + 31) / 32;
+    const dim3 grid(unsigned((cols + 31) / 32), unsigned(std::min<int64_t>(ntr, 65535)), unsigned(batch));
+    sat_transpose_kernel<T><<<grid, dim3(32, 8), 0, st>>>(static_cast<const T*>(in), static_cast<T*>(out),
+                                                          rows, cols);
+    CUDA_TRY(cudaGetLastError());
+    ++t_launches;
+    return SAT_OK;
+}
+
+// 4R4W (Sec. IV, Lemma 3): column prefix, transpose, column prefix, transpose.
+int run_4r4w(const Job& j, const sat_options& o) {
+    Workspace& ws = *j.ws;
+    SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * 4, false));
+    SAT_TRY(run_band(j, MODE_COL, j.in, j.out, base_params()));
+    auto tp = [&](const void* a, void* b, int64_t r, int64_t c) {
+        return j.dtype == SAT_INT32 ? transpose_t<uint32_t>(a, b, j.batch, r, c, j.st)
+                                    : transpose_t<float>(a, b, j.batch, r, c, j.st);
+    };
+    SAT_TRY(tp(j.out, ws.tr.p, j.rows, j.cols));
+    Job jt = j;
+    jt.rows = j.cols;
+    jt.cols = j.rows;
+    jt.in = ws.tr.p;
+    jt.out = ws.tr.p;
+    jt.th = o.tile_rows ? o.tile_rows : auto_th(jt.rows, jt.batch, *j.di, SAT_4R4W);
+    jt.tma = !o.force_generic && tma_ok(ws.tr.p, ws.tr.p, jt.cols);
+    SAT_TRY(run_band(jt, MODE_COL, ws.tr.p, ws.tr.p, base_params()));
+    return tp(ws.tr.p, j.out, jt.rows, jt.cols);
+}
+
+// 4R1W (Sec. VI, Formula (1)): rows + cols - 1 anti-diagonal stage launches.
+template <typename T>
+int run_4r1w_t(const Job& j) {
+    const int64_t stages = j.rows + j.cols - 1;
+    for (int64_t t = 0; t < stages; ++t) {
+        const int64_t i0 = std::max<int64_t>(0, t - (j.cols - 1));
+        const int64_t i1 = std::min<int64_t>(j.rows - 1, t);
+        const int64_t cnt = i1 - i0 + 1;
+        const unsigned blocks = unsigned(std::min<int64_t>((cnt + 255) / 256, 8LL * j.di->sms));
+        sat_4r1w_stage_kernel<T><<<dim3(blocks, unsigned(j.batch)), 256, 0, j.st>>>(
+            static_cast<const T*>(j.in), static_cast<T*>(j.out), j.rows, j.cols, t, i0, cnt);
+        CUDA_TRY(cudaGetLastError());
+        ++t_launches;
+    }
+    return SAT_OK;
+}
+
 // ------------------------------------------------------------------ core driver
 int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
                  int dtype, int variant, const sat_options* opt, const void* seed,
                  int seed_kind, cudaStream_t st) {
     t_launches = 0;
     SAT_TRY(validate(in, out, batch, rows, cols, dtype));
-    if (variant < SAT_2R2W || variant > SAT_1PLUSR_R1W) return fail(SAT_ERR_INVALID, "bad variant");
+    if (variant < SAT_2R2W || variant > SAT_4R1W) return fail(SAT_ERR_INVALID, "bad variant");
     sat_options o;
     sat_options_init(&o);
     if (opt) o = *opt;
@@ -620,6 +672,11 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             // (B) 2R1W on the bottom-right triangle, seeded from (C).
             return run_2r1w_region(j, c, REG_B, tA, in, out, ws->lb.p);
         }
+        case SAT_4R4W:
+            return run_4r4w(j, o);
+        case SAT_4R1W:
+            if (batch > 65535) return fail(SAT_ERR_UNSUPPORTED, "4R1W: batch must be <= 65535");
+            return dtype == SAT_INT32 ? run_4r1w_t<uint32_t>(j) : run_4r1w_t<float>(j);
     }
     return fail(SAT_ERR_INVALID, "bad variant");
 }

@@ -391,3 +391,63 @@ def test_band_segments(libsat, nseg, tile_rows, monkeypatch):
     for _ in range(3):
         check(libsat.sat(x, tile_rows=tile_rows), ref, "int32")
     check(libsat.sat(x, tile_rows=tile_rows, jitter=20000), ref, "int32")
+
+
+# ------------------------------------------------------------------ 4R4W / 4R1W
+PAPER_VARIANTS = ["4r4w", "4r1w"]
+
+
+def check_4r1w_f32(got, a):
+    """4R1W in float32: Formula (1) subtracts, so rounding errors do not stay
+    relative.  The computed b-hat satisfies b-hat = a + b-hat_up + b-hat_left
+    - b-hat_diag + delta with |delta_ij| <= 3u (2 b_ij + 1) for inputs in
+    [0, 1) (three roundings of partial sums <= 2 b_ij + 1, u = 2^-24), and the
+    error e = b-hat - b obeys the same recurrence, so e = SAT(delta) and
+    |e_ij| <= 3u SAT(2b + 1)_ij (R16).  Checked element by element
+    (with 1 % slack for second-order terms)."""
+    ref = oracle.sat(a)
+    bound = 3 * 2.0 ** -24 * np.cumsum(np.cumsum(2 * ref + 1, axis=0), axis=1) * 1.01
+    err = np.abs(got.astype(np.float64) - ref)
+    assert (err <= bound).all(), f"max err/bound {(err / bound).max()}"
+
+
+@pytest.mark.parametrize("variant", PAPER_VARIANTS)
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_fig3_paper_variants(libsat, fig3, variant, dtype):
+    a, _, b = fig3
+    y = libsat.sat(dev(a.astype(dtype)), variant=variant)
+    assert np.array_equal(y.cpu().numpy(), b.astype(dtype))
+
+
+@pytest.mark.parametrize("variant", PAPER_VARIANTS)
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: f"{s[0]}x{s[1]}")
+def test_shapes_paper_variants(libsat, variant, shape):
+    a = gen(*shape, "int32", seed=shape[0] * 3 + shape[1])
+    check(libsat.sat(dev(a), variant=variant), oracle.sat(a), "int32")
+    af = gen(*shape, "float32", seed=shape[0] * 3 + shape[1])
+    got = libsat.sat(dev(af), variant=variant).cpu().numpy()
+    if variant == "4r4w":
+        check(got, oracle.sat(af), "float32")
+    else:
+        check_4r1w_f32(got, af)
+
+
+@pytest.mark.parametrize("variant", PAPER_VARIANTS)
+def test_paper_variants_inplace_batched(libsat, variant):
+    a = gen(3 * 129, 200, "int32", seed=9).reshape(3, 129, 200)
+    got = libsat.sat_batched(dev(a), variant=variant).cpu().numpy()
+    for i in range(3):
+        assert np.array_equal(got[i], oracle.sat(a[i]))
+    b = gen(257, 300, "int32", seed=10)
+    x = dev(b)
+    y = libsat.sat(x, variant=variant, out=x)
+    assert y.data_ptr() == x.data_ptr()
+    assert np.array_equal(x.cpu().numpy(), oracle.sat(b))
+
+
+def test_4r4w_cfg2_and_4r1w_4096(libsat):
+    af = gen(4096, 4096, "float32", seed=2)
+    check(libsat.sat(dev(af), variant="4r4w"), oracle.sat(af), "float32")
+    a = gen(4096, 4096, "int32", seed=2)
+    check(libsat.sat(dev(a), variant="4r1w"), oracle.sat(a), "int32")
+    assert libsat.last_launch_count() == 4096 + 4096 - 1
