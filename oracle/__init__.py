@@ -12,7 +12,8 @@ Definition followed (Kasagi, Nakano, Ito, ICPP 2014 -- /root/reference/PAPER.md)
     sequential baselines.
 
 Element types (reading R3): int32 input is summed in uint32 (wraps
-mod 2^32); float32 input is summed in float64.  The heavy loops are plain C
+mod 2^32); float32 input is summed in float64; float64 input (the paper's own
+precision) is summed in float64.  The heavy loops are plain C
 (``sat_oracle.c``, single-threaded, gcc -O2) loaded with ctypes; small helpers
 are numpy.  Every pin lives in ``tests/test_oracle.py``.
 """
@@ -49,19 +50,32 @@ def _load():
     if _lib is None:
         build()
         lib = ctypes.CDLL(_LIB_PATH)
-        for name in ("oracle_sat_u32", "oracle_sat_f64"):
-            getattr(lib, name).argtypes = [_P, _P, _I64, _I64, _P]
-        for name in ("oracle_sat_u32_eq1", "oracle_sat_f64_eq1"):
-            getattr(lib, name).argtypes = [_P, _P, _I64, _I64, _P]
-        for name in ("oracle_sat_u32_2pass", "oracle_sat_f64_2pass",
-                     "oracle_sat_u32_brute", "oracle_sat_f64_brute"):
-            getattr(lib, name).argtypes = [_P, _P, _I64, _I64]
-        lib.oracle_sat_u32_at.argtypes = [_P, _I64, _I64, _I64, _I64]
+        for k in _KINDS:
+            getattr(lib, f"oracle_sat_{k}").argtypes = [_P, _P, _I64, _I64, _P]
+            getattr(lib, f"oracle_sat_{k}_eq1").argtypes = [_P, _P, _I64, _I64, _P]
+            getattr(lib, f"oracle_sat_{k}_2pass").argtypes = [_P, _P, _I64, _I64]
+            getattr(lib, f"oracle_sat_{k}_brute").argtypes = [_P, _P, _I64, _I64]
+            getattr(lib, f"oracle_sat_{k}_at").argtypes = [_P, _I64, _I64, _I64, _I64]
         lib.oracle_sat_u32_at.restype = ctypes.c_uint32
-        lib.oracle_sat_f64_at.argtypes = [_P, _I64, _I64, _I64, _I64]
         lib.oracle_sat_f64_at.restype = ctypes.c_double
+        lib.oracle_sat_d64_at.restype = ctypes.c_double
         _lib = lib
     return _lib
+
+
+# C function families by input kind: u32 (int32/uint32 input, uint32 sums),
+# f64 (float32 input, float64 sums), d64 (float64 input, float64 sums)
+_KINDS = ("u32", "f64", "d64")
+
+
+def _kind(a: np.ndarray) -> str:
+    if a.dtype in (np.int32, np.uint32):
+        return "u32"
+    if a.dtype == np.float32:
+        return "f64"
+    if a.dtype == np.float64:
+        return "d64"
+    raise TypeError(f"oracle supports int32/uint32/float32/float64 inputs, got {a.dtype}")
 
 
 def _prep(a: np.ndarray):
@@ -69,11 +83,14 @@ def _prep(a: np.ndarray):
     a = np.ascontiguousarray(a)
     if a.ndim != 2:
         raise ValueError("oracle expects a 2-D matrix")
-    if a.dtype in (np.int32, np.uint32):
+    k = _kind(a)
+    if k == "u32":
         return a.view(np.uint32), True, np.uint32
-    if a.dtype == np.float32:
-        return a, False, np.float64
-    raise TypeError(f"oracle supports int32/uint32/float32 inputs, got {a.dtype}")
+    return a, False, np.float64
+
+
+def _fn(lib, a: np.ndarray, suffix: str = ""):
+    return getattr(lib, f"oracle_sat_{_kind(a)}{suffix}")
 
 
 def _ptr(x: np.ndarray):
@@ -102,7 +119,7 @@ class Stream:
             raise ValueError("strip does not match stream")
         out = np.empty(a.shape, dtype=odt)
         lib = _load()
-        fn = lib.oracle_sat_u32 if is_int else lib.oracle_sat_f64
+        fn = _fn(lib, a)
         if a.size:
             fn(_ptr(a), _ptr(out), a.shape[0], a.shape[1], _ptr(self.colsum))
         return _ret(out, strip.dtype)
@@ -119,7 +136,7 @@ def sat_eq1(a: np.ndarray, prev_row: np.ndarray | None = None) -> np.ndarray:
     a_c, is_int, odt = _prep(a)
     out = np.empty(a_c.shape, dtype=odt)
     lib = _load()
-    fn = lib.oracle_sat_u32_eq1 if is_int else lib.oracle_sat_f64_eq1
+    fn = _fn(lib, a_c, "_eq1")
     pr = None
     if prev_row is not None:
         pr = np.ascontiguousarray(prev_row)
@@ -135,7 +152,7 @@ def sat_2pass(a: np.ndarray) -> np.ndarray:
     a_c, is_int, odt = _prep(a)
     out = np.empty(a_c.shape, dtype=odt)
     lib = _load()
-    fn = lib.oracle_sat_u32_2pass if is_int else lib.oracle_sat_f64_2pass
+    fn = _fn(lib, a_c, "_2pass")
     if a_c.size:
         fn(_ptr(a_c), _ptr(out), a_c.shape[0], a_c.shape[1])
     return _ret(out, a.dtype)
@@ -148,7 +165,7 @@ def sat_brute(a: np.ndarray) -> np.ndarray:
         raise ValueError("sat_brute is for tiny inputs")
     out = np.empty(a_c.shape, dtype=odt)
     lib = _load()
-    fn = lib.oracle_sat_u32_brute if is_int else lib.oracle_sat_f64_brute
+    fn = _fn(lib, a_c, "_brute")
     if a_c.size:
         fn(_ptr(a_c), _ptr(out), a_c.shape[0], a_c.shape[1])
     return _ret(out, a.dtype)
@@ -161,7 +178,7 @@ def sat_at(a: np.ndarray, i: int, j: int):
     if is_int:
         v = lib.oracle_sat_u32_at(_ptr(a_c), a_c.shape[0], a_c.shape[1], int(i), int(j))
         return np.uint32(v).view(np.int32) if a.dtype == np.int32 else np.uint32(v)
-    return float(lib.oracle_sat_f64_at(_ptr(a_c), a_c.shape[0], a_c.shape[1], int(i), int(j)))
+    return float(_fn(lib, a_c, "_at")(_ptr(a_c), a_c.shape[0], a_c.shape[1], int(i), int(j)))
 
 
 def rect_sum(b: np.ndarray, r0: int, c0: int, r1: int, c1: int):
@@ -182,7 +199,7 @@ def rect_sum(b: np.ndarray, r0: int, c0: int, r1: int, c1: int):
 def column_totals(a: np.ndarray) -> np.ndarray:
     """Column sums of a strip (the sharded mode's exchanged vector).
 
-    int32 -> uint32 (mod 2^32, returned as int32), float32 -> float64.
+    int32 -> uint32 (mod 2^32, returned as int32), float32/float64 -> float64.
     """
     a_c, is_int, _ = _prep(a)
     if is_int:

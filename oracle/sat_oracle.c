@@ -151,3 +151,62 @@ void oracle_sat_f64_brute(const float *a, double *b, int64_t rows, int64_t cols)
         for (int64_t j = 0; j < cols; ++j)
             b[i * cols + j] = oracle_sat_f64_at(a, rows, cols, i, j);
 }
+
+/* ---------------- float64 input, float64 arithmetic (the paper's precision,
+ * "double (64-bit) numbers") ---------------- */
+
+void oracle_sat_d64(const double *a, double *b, int64_t rows, int64_t cols,
+                    double *colsum)
+{
+    for (int64_t i = 0; i < rows; ++i) {
+        double s = 0.0;
+        for (int64_t j = 0; j < cols; ++j) {
+            colsum[j] += a[i * cols + j];   /* column-wise prefix-sum */
+            s += colsum[j];                 /* row-wise prefix-sum of it */
+            b[i * cols + j] = s;
+        }
+    }
+}
+
+void oracle_sat_d64_eq1(const double *a, double *b, int64_t rows, int64_t cols,
+                        const double *prev_row)
+{
+    for (int64_t i = 0; i < rows; ++i) {
+        const double *up = (i > 0) ? b + (i - 1) * cols : prev_row;
+        for (int64_t j = 0; j < cols; ++j) {
+            double v = a[i * cols + j];
+            double b_up = up ? up[j] : 0.0;
+            double b_left = (j > 0) ? b[i * cols + j - 1] : 0.0;
+            double b_diag = (up && j > 0) ? up[j - 1] : 0.0;
+            b[i * cols + j] = v + b_up + b_left - b_diag;
+        }
+    }
+}
+
+void oracle_sat_d64_2pass(const double *a, double *b, int64_t rows, int64_t cols)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 0; j < cols; ++j)
+            b[i * cols + j] = a[i * cols + j] + (i > 0 ? b[(i - 1) * cols + j] : 0.0);
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 1; j < cols; ++j)
+            b[i * cols + j] += b[i * cols + j - 1];
+}
+
+double oracle_sat_d64_at(const double *a, int64_t rows, int64_t cols,
+                         int64_t i, int64_t j)
+{
+    (void)rows;
+    double s = 0.0;
+    for (int64_t k = 0; k <= i; ++k)
+        for (int64_t l = 0; l <= j; ++l)
+            s += a[k * cols + l];
+    return s;
+}
+
+void oracle_sat_d64_brute(const double *a, double *b, int64_t rows, int64_t cols)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 0; j < cols; ++j)
+            b[i * cols + j] = oracle_sat_d64_at(a, rows, cols, i, j);
+}

@@ -14,6 +14,12 @@ Distributions (DESIGN.md "input recipe"):
   int32 "ones" : all ones (closed form (i+1)(j+1))
   float32 "unit": (hash >> 40) * 2^-24, dyadic uniform in [0, 1)
   float32 "ones": all ones (exact in float32 while the SAT stays <= 2^24)
+  float64 "unit": (hash >> 40) * 2^-24 -- the float32 "unit" values held in
+                  double: every partial sum is exact while the SAT stays
+                  below 2^29, so float64 results are unique (up to ~23K^2)
+  float64 "unit53": (hash >> 11) * 2^-53, uniform [0, 1) with full 53-bit
+                  mantissas (rounding-sensitive)
+  float64 "ones": all ones
 """
 from __future__ import annotations
 
@@ -25,6 +31,7 @@ _M2 = np.uint64(0x94D049BB133111EB)
 
 INT_DISTS = ("u32", "u8", "ones")
 FLOAT_DISTS = ("unit", "ones")
+DOUBLE_DISTS = ("unit", "unit53", "ones")
 
 
 def _splitmix_np(ctr: np.ndarray, seed: int) -> np.ndarray:
@@ -61,6 +68,13 @@ def _finish_np(h: np.ndarray, dtype: str, dist: str) -> np.ndarray:
             return ((h >> np.uint64(40)).astype(np.float64) * 2.0 ** -24).astype(np.float32)
         if dist == "ones":
             return np.ones(h.shape, dtype=np.float32)
+    elif dtype == "float64":
+        if dist == "unit":
+            return (h >> np.uint64(40)).astype(np.float64) * 2.0 ** -24
+        if dist == "unit53":
+            return (h >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+        if dist == "ones":
+            return np.ones(h.shape, dtype=np.float64)
     raise ValueError(f"unknown dtype/dist {dtype}/{dist}")
 
 
@@ -109,7 +123,7 @@ def make_torch(rows: int, cols: int, dtype: str = "int32", dist: str | None = No
     """
     import torch
     dist = dist or ("u32" if dtype == "int32" else "unit")
-    tdt = torch.int32 if dtype == "int32" else torch.float32
+    tdt = {"int32": torch.int32, "float32": torch.float32, "float64": torch.float64}[dtype]
     shape = (rows, cols) if batch is None else (batch, rows, cols)
     if out is None:
         out = torch.empty(shape, dtype=tdt, device=device)
@@ -130,6 +144,13 @@ def make_torch(rows: int, cols: int, dtype: str = "int32", dist: str | None = No
                 v = torch.where(v >= (1 << 31), v - (1 << 32), v).to(torch.int32)
             elif dist == "u8":
                 v = torch.bitwise_and(h, 0xFF).to(torch.int32)
+            else:
+                raise ValueError(dist)
+        elif dtype == "float64":
+            if dist == "unit":
+                v = _lsr(h, 40).to(torch.float64) * 2.0 ** -24
+            elif dist == "unit53":
+                v = _lsr(h, 11).to(torch.float64) * 2.0 ** -53
             else:
                 raise ValueError(dist)
         else:

@@ -8,7 +8,9 @@ from sat_inputs import make_np, make_torch
 
 
 @pytest.mark.parametrize("dtype,dist", [("int32", "u32"), ("int32", "u8"), ("int32", "ones"),
-                                        ("float32", "unit"), ("float32", "ones")])
+                                        ("float32", "unit"), ("float32", "ones"),
+                                        ("float64", "unit"), ("float64", "unit53"),
+                                        ("float64", "ones")])
 def test_numpy_torch_twins(dtype, dist):
     a = make_np(37, 53, dtype, dist, seed=123)
     t = make_torch(37, 53, dtype, dist, seed=123, chunk_rows=5).numpy()
@@ -34,3 +36,12 @@ def test_ranges():
     u = make_np(64, 64, "int32", "u32", seed=1)
     assert u.min() < -2**30 and u.max() > 2**30
     assert not np.array_equal(make_np(8, 8, seed=1), make_np(8, 8, seed=2))
+
+
+def test_float64_ranges():
+    d = make_np(64, 64, "float64", "unit", seed=1)
+    assert np.array_equal(d, make_np(64, 64, "float32", "unit", seed=1).astype(np.float64))
+    e = make_np(64, 64, "float64", "unit53", seed=1)
+    assert e.min() >= 0.0 and e.max() < 1.0
+    assert np.array_equal(np.floor(e * 2**53), e * 2**53)
+    assert (np.floor(e * 2**24) != e * 2**24).any()       # genuinely finer than 2^-24

@@ -251,3 +251,72 @@ def test_sharding_invariant():
 def test_max_rel_err():
     assert oracle.max_rel_err(np.array([1.0, 2.0]), np.array([1.0, 2.0])) == 0.0
     assert abs(oracle.max_rel_err(np.array([1.0, 2.2]), np.array([1.0, 2.0])) - 0.1) < 1e-12
+
+
+# ---------------------------------------------------------------- float64 input
+# The paper computes in double.  Pins for the d64 family.
+@pytest.mark.parametrize("form", FORMS + [oracle.sat_brute])
+def test_fig3_float64(fig3, form):
+    a, cp, b = fig3
+    got = form(a.astype(np.float64))
+    assert got.dtype == np.float64 and np.array_equal(got, b.astype(np.float64))
+
+
+@pytest.mark.parametrize("n,m", [(1, 1), (2, 7), (7, 2), (9, 13)])
+def test_brute_small_float64(n, m):
+    """Pure-Python double sum of exact dyadic values (no oracle code)."""
+    a = make_np(n, m, "float64", "unit", seed=n * 31 + m)
+    ref = np.array(py_brute(a.tolist()), dtype=np.float64)
+    for form in FORMS + [oracle.sat_brute]:
+        assert np.array_equal(form(a), ref)
+
+
+def test_float64_dyadic_exact():
+    """float64 "unit" inputs are k 2^-24: every partial sum below 2^29 is exact,
+    so each formulation equals integer arithmetic on k exactly."""
+    a = make_np(211, 173, "float64", "unit", seed=12)
+    k = (a * 2.0**24).astype(np.int64)
+    assert np.array_equal(k.astype(np.float64) * 2.0**-24, a)
+    ref = np.cumsum(np.cumsum(k, axis=0), axis=1).astype(np.float64) * 2.0**-24
+    for form in FORMS:
+        assert np.array_equal(form(a), ref)
+    # inclusion-exclusion recovers the input exactly (all values exact)
+    b = oracle.sat(a)
+    pad = np.zeros((212, 174))
+    pad[1:, 1:] = b
+    assert np.array_equal(pad[1:, 1:] - pad[:-1, 1:] - pad[1:, :-1] + pad[:-1, :-1], a)
+
+
+def test_float64_unit53_vs_exact_rationals():
+    """Full-mantissa inputs: the float64 oracle is within the recursive-summation
+    bound (i + j + 2) u b[i][j] of the exact rational SAT (fractions)."""
+    from fractions import Fraction
+    a = make_np(12, 17, "float64", "unit53", seed=3)
+    fa = [[Fraction(x) for x in row] for row in a.tolist()]
+    exact = py_brute(fa)
+    u = 2.0 ** -53
+    for form in FORMS:
+        got = form(a)
+        for i in range(12):
+            for j in range(17):
+                err = abs(Fraction(got[i, j]) - exact[i][j])
+                assert err <= (i + j + 2) * u * exact[i][j] * Fraction(101, 100)
+
+
+@pytest.mark.parametrize("n,m", [(17, 29), (29, 17)])
+def test_separable_closed_form_float64(n, m):
+    f = (np.arange(n, dtype=np.int64) * 5 + 2)
+    g = (np.arange(m, dtype=np.int64) % 11 + 1)
+    a = (f[:, None] * g[None, :]).astype(np.float64)
+    ref = (np.cumsum(f)[:, None] * np.cumsum(g)[None, :]).astype(np.float64)
+    for form in FORMS:
+        assert np.array_equal(form(a), ref)
+
+
+@pytest.mark.parametrize("shape", [(1, 999), (999, 1)])
+def test_1d_is_cumsum_float64(shape):
+    """One row / one column: both are sequential left-to-right sums, bit-equal
+    to numpy's cumsum (a library routine)."""
+    a = make_np(*shape, "float64", "unit53", seed=4)
+    for form in FORMS:
+        assert np.array_equal(form(a).ravel(), np.cumsum(a.ravel()))
