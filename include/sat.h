@@ -23,7 +23,12 @@
  *     nearest, no FTZ); its summation order differs between variants and may
  *     differ between runs (the look-back takes whichever predecessor state it
  *     finds first); every order stays within the documented 1e-5 max relative
- *     error for inputs in [0, 1).
+ *     error for inputs in [0, 1).  SAT_FLOAT64 (the
+ *     paper's "double (64-bit)" precision) uses IEEE fp64 adds with
+ *     the same ordering caveats; for inputs k*2^-24 every partial sum below
+ *     2^29 is exact, so those results are unique.  Float64 takes tile_rows
+ *     16, 32, 48 or 64 and needs 8-byte aligned pointers; the TMA path needs
+ *     16-byte aligned pointers and cols % 4 == 0 (as for 4-byte types).
  *   - in == out (exact aliasing) is allowed for every entry point that takes
  *     both; a partial overlap returns SAT_ERR_INVALID.
  *   - rows == 0 or cols == 0 (or batch == 0) is a no-op returning SAT_OK.
@@ -49,7 +54,7 @@ extern "C" {
 
 #define SAT_ABI_VERSION 1
 
-typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1 } sat_dtype;
+typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1, SAT_FLOAT64 = 2 } sat_dtype;
 
 /* Variants (Table I / Secs. IV-VII):
  *   SAT_2R2W        column-wise prefix pass then row-wise prefix pass, each a

@@ -21,7 +21,7 @@ if not os.path.exists(_LIB_PATH):
 
 _lib = ctypes.CDLL(_LIB_PATH)
 
-SAT_INT32, SAT_FLOAT32 = 0, 1
+SAT_INT32, SAT_FLOAT32, SAT_FLOAT64 = 0, 1, 2
 VARIANTS = {"2r2w": 0, "2r1w": 1, "1r1w": 2, "1+rr1w": 3, "4r4w": 4, "4r1w": 5}
 SAT_OK = 0
 
@@ -92,7 +92,9 @@ def _dtype_code(t) -> int:
         return SAT_INT32
     if t.dtype == torch.float32:
         return SAT_FLOAT32
-    raise TypeError(f"libsat supports int32 and float32, got {t.dtype}")
+    if t.dtype == torch.float64:
+        return SAT_FLOAT64
+    raise TypeError(f"libsat supports int32, float32 and float64, got {t.dtype}")
 
 
 def _stream(stream) -> int:
@@ -125,7 +127,7 @@ def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
 
 def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
         force_generic: bool = False, jitter: int = 0, stream=None):
-    """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32 IEEE).
+    """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32/float64 IEEE).
 
     ``out`` may be ``x`` itself (in place).  ``variant`` in
     {"1r1w", "2r2w", "2r1w", "1+rr1w"}.
@@ -228,14 +230,15 @@ def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=N
     cols = strip.shape[1]
     nbytes = _lib.sat_sharded_workspace_bytes(cols, nranks, _dtype_code(strip))
     ws = torch.empty(max(nbytes, 1), dtype=torch.uint8, device=strip.device)
-    row = ((cols * 4) + 255) // 256 * 256
-    send = ws[:cols * 4].view(strip.dtype)
-    recv = ws[2 * row:2 * row + nranks * cols * 4].view(strip.dtype).view(nranks, cols)
+    eb = strip.element_size()
+    row = ((cols * eb) + 255) // 256 * 256
+    send = ws[:cols * eb].view(strip.dtype)
+    recv = ws[2 * row:2 * row + nranks * cols * eb].view(strip.dtype).view(nranks, cols)
     err = []
 
     def cb(ctx, send_p, recv_p, nb, st):
         try:
-            assert send_p == send.data_ptr() and recv_p == recv.data_ptr() and nb == cols * 4
+            assert send_p == send.data_ptr() and recv_p == recv.data_ptr() and nb == cols * eb
             allgather(send, recv)
             return 0
         except Exception as e:  # reported through SAT_ERR_COMM

@@ -140,16 +140,24 @@ int get_ws(int dev, cudaStream_t st, Workspace*& ws) {
 
 // ------------------------------------------------------------------ helpers
 
+bool dtype_ok(int dtype) { return dtype == SAT_INT32 || dtype == SAT_FLOAT32 || dtype == SAT_FLOAT64; }
+size_t esize(int dtype) { return dtype == SAT_FLOAT64 ? 8 : 4; }
+// Element type of a sat_dtype: uint32 (int32, wrapping), float, double.
+#define SAT_DISPATCH(dtype, T, ...)                                             \
+    ((dtype) == SAT_INT32     ? [&] { using T = uint32_t; return __VA_ARGS__; }() \
+     : (dtype) == SAT_FLOAT32 ? [&] { using T = float; return __VA_ARGS__; }()    \
+                              : [&] { using T = double; return __VA_ARGS__; }())
+
 int validate(const void* in, const void* out, int64_t batch, int64_t rows, int64_t cols,
              int dtype, bool need_in = true) {
-    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32)
-        return fail(SAT_ERR_INVALID, "dtype must be SAT_INT32 or SAT_FLOAT32");
+    if (!dtype_ok(dtype))
+        return fail(SAT_ERR_INVALID, "dtype must be SAT_INT32, SAT_FLOAT32 or SAT_FLOAT64");
     if (rows < 0 || cols < 0 || batch < 0) return fail(SAT_ERR_INVALID, "negative size");
     if (rows > INT32_MAX || cols > INT32_MAX || batch > INT32_MAX)
         return fail(SAT_ERR_INVALID, "rows, cols and batch must each be < 2^31");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     const double n = double(rows) * double(cols) * double(batch);
-    if (n * 4.0 > 9.0e18) return fail(SAT_ERR_INVALID, "matrix byte size overflows");
+    if (n * double(esize(dtype)) > 9.0e18) return fail(SAT_ERR_INVALID, "matrix byte size overflows");
     if ((need_in && !in) || !out) return fail(SAT_ERR_INVALID, "null pointer with nonzero size");
     if (need_in && in != out) {
         const uintptr_t a0 = reinterpret_cast<uintptr_t>(in), b0 = reinterpret_cast<uintptr_t>(out);
@@ -157,8 +165,9 @@ int validate(const void* in, const void* out, int64_t batch, int64_t rows, int64
         if (a0 < b0 + len && b0 < a0 + len)
             return fail(SAT_ERR_INVALID, "in and out partially overlap");
     }
-    if ((reinterpret_cast<uintptr_t>(out) & 3) || (need_in && (reinterpret_cast<uintptr_t>(in) & 3)))
-        return fail(SAT_ERR_INVALID, "pointers must be 4-byte aligned");
+    const uintptr_t am = esize(dtype) - 1;
+    if ((reinterpret_cast<uintptr_t>(out) & am) || (need_in && (reinterpret_cast<uintptr_t>(in) & am)))
+        return fail(SAT_ERR_INVALID, "pointers must be aligned to the element size");
     return SAT_OK;
 }
 
@@ -170,11 +179,13 @@ bool tma_ok(const void* in, const void* out, int64_t cols) {
 int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_t rows,
               int64_t cols, int th) {
     cuuint64_t dims[3] = {cuuint64_t(cols), cuuint64_t(rows), cuuint64_t(batch)};
-    cuuint64_t strides[2] = {cuuint64_t(cols) * 4, cuuint64_t(cols) * cuuint64_t(rows) * 4};
+    const cuuint64_t eb = esize(dtype);
+    cuuint64_t strides[2] = {cuuint64_t(cols) * eb, cuuint64_t(cols) * cuuint64_t(rows) * eb};
     cuuint32_t box[3] = {cuuint32_t(TW), cuuint32_t(th), 1};
     cuuint32_t es[3] = {1, 1, 1};
-    CUresult r = g_encode(m, dtype == SAT_INT32 ? CU_TENSOR_MAP_DATA_TYPE_UINT32
-                                                : CU_TENSOR_MAP_DATA_TYPE_FLOAT32,
+    CUresult r = g_encode(m, dtype == SAT_INT32     ? CU_TENSOR_MAP_DATA_TYPE_UINT32
+                             : dtype == SAT_FLOAT32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                                    : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
                           3, const_cast<void*>(base), dims, strides, box, es,
                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -199,6 +210,17 @@ constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
+// float64 (8-byte elements: 1 KB chunk rows, two TMEM words per element)
+constexpr BandCfg kCfgD16{2, 8, 4, 4, 1, 3, 1, 2};   //  96 KB smem, 128 TMEM cols: 2 CTAs/SM
+constexpr BandCfg kCfgD32{4, 8, 4, 8, 1, 4, 1, 1};   // 192 KB smem, 512 TMEM cols
+constexpr BandCfg kCfgD48{8, 6, 3, 4, 1, 4, 1, 1};   // 168 KB smem, 512 TMEM cols
+constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 3, 1, 1};   // 224 KB smem, 512 TMEM cols
+
+// CTAs per SM of a configuration (for wave counts before launch)
+int ctas_per_sm(int dtype, int th, bool big) {
+    if (dtype == SAT_FLOAT64) return th == 16 ? 2 : 1;
+    return (th == 128 || big) ? 1 : 2;
+}
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
           int CL = 1, int LBW = 0>
@@ -224,7 +246,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
     int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
                         di.smem_sm / int(smem + fa.sharedSizeBytes + 1024),
-                        MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT>::alloc, 32});
+                        MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT, int(sizeof(T) / 4)>::alloc, 32});
     if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
     if (const char* e = getenv("SAT_DEBUG_OCC")) occ = atoi(e);
     if constexpr (CL > 1) {
@@ -277,6 +299,15 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
             if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
         }
     }
+    if constexpr (sizeof(T) == 8) {
+        switch (th) {
+            case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, to, di, st, grid);
+            case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, to, di, st, grid);
+            case 48: return launch_band_t<T, SAT_CFG(kCfgD48), MODE, TMA, kCfgD48.MINB>(p, ti, to, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, to, di, st, grid);
+        }
+        return fail(SAT_ERR_INVALID, "float64: tile_rows must be 16, 32, 48 or 64");
+    } else {
     if constexpr (MODE == MODE_SAT && TMA) {
         if (p.big && th == 64) {  // 192 KB ring of 64 x 256 slots, 6 chunks parked in TMEM
             if (const char* e = getenv("SAT_DEBUG_LBW")) {
@@ -300,6 +331,7 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
     }
     return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64 or 128");
+    }
 }
 
 template <typename T, int MODE>
@@ -323,7 +355,15 @@ int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtenso
 // Automatic band height: the tallest band that still gives roughly one band
 // per resident CTA slot (the look-back chain is per band; more, shorter bands
 // raise parallelism, taller bands cut descriptor traffic).
-int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant) {
+int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dtype) {
+    if (dtype == SAT_FLOAT64) {
+        // one CTA per SM for TH 32/64 (1-KB rows): the tallest band with a wave
+        for (int th : {64, 32}) {
+            const long long bands = batch * ((rows + th - 1) / th);
+            if (bands * 5 >= 4LL * di.sms) return th;
+        }
+        return 16;
+    }
     // 1R1W: TH = 128 (one CTA per SM) once its bands fill a wave (16K^2,
     // 18432^2: measured 5.3-5.4 TB/s vs 5.0 for TH = 64; 65536^2 with band
     // segments: 5.97 ms vs 6.27 ms for TH = 64).
@@ -368,16 +408,16 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     // they are opt-in (SAT_CLUSTER=8) for plain 1R1W on the TMA path.
     p.cluster = 1;
     if (const char* e = getenv("SAT_CLUSTER")) {
-        if (atoi(e) == 8 && mode == MODE_SAT && j.tma && p.region == REG_ALL &&
+        if (atoi(e) == 8 && mode == MODE_SAT && j.tma && p.region == REG_ALL && j.dtype != SAT_FLOAT64 &&
             p.top_src == TOP_LOOKBACK && !p.tile_units && (j.th == 64 || j.th == 48))
             p.cluster = 8;
     }
     // Many bands (>= 4 waves of one CTA per SM): one CTA per SM with twice the
     // ring and 1-KB row segments per TMA load.
-    p.big = (mode == MODE_SAT && j.tma && p.cluster == 1 && j.th == 64 &&
+    p.big = (mode == MODE_SAT && j.tma && p.cluster == 1 && j.th == 64 && j.dtype != SAT_FLOAT64 &&
              p.total_bands >= 4 * j.di->sms) ? 1 : 0;
     if (const char* e = getenv("SAT_BIG")) p.big = (atoi(e) != 0 && mode == MODE_SAT && j.tma &&
-                                                    p.cluster == 1 && j.th == 64) ? 1 : 0;
+                                                    p.cluster == 1 && j.th == 64 && j.dtype != SAT_FLOAT64) ? 1 : 0;
     if (p.cluster > 1)
         p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
     // Band segments: short units for the last wave when
@@ -389,7 +429,7 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         // >= 2 waves of bands: ~16 segments of >= 32 chunks (65536^2, TH 128:
         // 5.97 ms with 16 segments vs 6.34 ms whole bands); one wave: whole
         // bands (a segment would wait for the band's previous segment)
-        const int slots = j.di->sms * ((j.th == 128 || p.big) ? 1 : 2);
+        const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0);
         int want = p.total_bands >= 2 * slots ? std::min(16, p.nc / 32) : 1;
         if (const char* e = getenv("SAT_SEG")) want = std::max(1, atoi(e));
         if (want > 1 && p.nc > 1) {
@@ -407,11 +447,12 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     }
     Workspace& ws = *j.ws;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
-        const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t);
+        const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t) * (esize(j.dtype) / 4);
         SAT_TRY(ensure(ws.desc, need, true));
     }
     SAT_TRY(ensure(ws.ticket, sizeof(unsigned long long), true));
-    if (p.nseg > 1) SAT_TRY(ensure(ws.lseg, size_t(p.total_bands) * j.th * sizeof(uint64_t), true));
+    if (p.nseg > 1)
+        SAT_TRY(ensure(ws.lseg, size_t(p.total_bands) * j.th * sizeof(uint64_t) * (esize(j.dtype) / 4), true));
     const unsigned long long units = (unsigned long long)p.total_units;
     const unsigned long long worst = units + 4096ull * 64ull;   // units + max grid
     if (ws.next_base + worst >= kTagSpace) {
@@ -432,9 +473,7 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         SAT_TRY(make_tmap(&ti, in, j.dtype, j.batch, j.rows, j.cols, j.th));
     }
     int grid = 0;
-    int s = (j.dtype == SAT_INT32)
-                ? launch_band_d<uint32_t>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid)
-                : launch_band_d<float>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid);
+    int s = SAT_DISPATCH(j.dtype, T, launch_band_d<T>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid));
     if (s != SAT_OK) return s;
     // every persistent ticket taker (a CTA, or a cluster) makes exactly one
     // failing fetch, so the counter ends at base + units + takers
@@ -462,7 +501,7 @@ int prep_2r1w(const Job& j, Carry2r1w& c) {
     c.nc = int((j.cols + TW - 1) / TW);
     c.total_bands = int(j.batch * c.nb);
     Workspace& ws = *j.ws;
-    const size_t eb = 4;
+    const size_t eb = esize(j.dtype);
     const size_t wide = size_t(c.total_bands) * c.nc * TW * eb;
     const size_t rowsp = size_t(c.total_bands) * j.th * eb;
     SAT_TRY(ensure(ws.bt, wide, false));
@@ -513,8 +552,7 @@ int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, cons
 
 int run_2r1w_region(const Job& j, const Carry2r1w& c, int region, int tA, const void* in,
                     void* out, const void* Lb) {
-    return j.dtype == SAT_INT32 ? run_2r1w_region_t<uint32_t>(j, c, region, tA, in, out, Lb)
-                                : run_2r1w_region_t<float>(j, c, region, tA, in, out, Lb);
+    return SAT_DISPATCH(j.dtype, T, run_2r1w_region_t<T>(j, c, region, tA, in, out, Lb));
 }
 
 // Choose the triangle threshold tA whose tile fraction (|A|+|B|)/(nb*nc) is
@@ -554,11 +592,10 @@ int transpose_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t 
 // 4R4W (Sec. IV, Lemma 3): column prefix, transpose, column prefix, transpose.
 int run_4r4w(const Job& j, const sat_options& o) {
     Workspace& ws = *j.ws;
-    SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * 4, false));
+    SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * esize(j.dtype), false));
     SAT_TRY(run_band(j, MODE_COL, j.in, j.out, base_params()));
     auto tp = [&](const void* a, void* b, int64_t r, int64_t c) {
-        return j.dtype == SAT_INT32 ? transpose_t<uint32_t>(a, b, j.batch, r, c, j.st)
-                                    : transpose_t<float>(a, b, j.batch, r, c, j.st);
+        return SAT_DISPATCH(j.dtype, T, transpose_t<T>(a, b, j.batch, r, c, j.st));
     };
     SAT_TRY(tp(j.out, ws.tr.p, j.rows, j.cols));
     Job jt = j;
@@ -566,7 +603,7 @@ int run_4r4w(const Job& j, const sat_options& o) {
     jt.cols = j.rows;
     jt.in = ws.tr.p;
     jt.out = ws.tr.p;
-    jt.th = o.tile_rows ? o.tile_rows : auto_th(jt.rows, jt.batch, *j.di, SAT_4R4W);
+    jt.th = o.tile_rows ? o.tile_rows : auto_th(jt.rows, jt.batch, *j.di, SAT_4R4W, j.dtype);
     jt.tma = !o.force_generic && tma_ok(ws.tr.p, ws.tr.p, jt.cols);
     SAT_TRY(run_band(jt, MODE_COL, ws.tr.p, ws.tr.p, base_params()));
     return tp(ws.tr.p, j.out, jt.rows, jt.cols);
@@ -611,7 +648,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     SAT_TRY(get_ws(dev, st, ws));
     Job j;
     j.in = in; j.out = out; j.batch = batch; j.rows = rows; j.cols = cols; j.dtype = dtype;
-    j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant);
+    j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
     j.tma = !o.force_generic && tma_ok(in, out, cols);
     j.jitter = o.jitter;
     j.di = &di;
@@ -623,13 +660,10 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             BandParams p = base_params();
             if (seed && seed_kind == SEED_COLSUM) {
                 // column sums above the strip -> the SAT row just above it
-                SAT_TRY(ensure(ws->seedrow, size_t(cols) * 4, false));
-                if (dtype == SAT_INT32)
-                    sat_row_prefix_kernel<uint32_t><<<1, 1024, 0, st>>>(
-                        static_cast<const uint32_t*>(seed), static_cast<uint32_t*>(ws->seedrow.p), cols);
-                else
-                    sat_row_prefix_kernel<float><<<1, 1024, 0, st>>>(
-                        static_cast<const float*>(seed), static_cast<float*>(ws->seedrow.p), cols);
+                SAT_TRY(ensure(ws->seedrow, size_t(cols) * esize(dtype), false));
+                SAT_DISPATCH(dtype, T, (sat_row_prefix_kernel<T><<<1, 1024, 0, st>>>(
+                                            static_cast<const T*>(seed), static_cast<T*>(ws->seedrow.p), cols),
+                                        0));
                 CUDA_TRY(cudaGetLastError());
                 ++t_launches;
                 seed = ws->seedrow.p;
@@ -676,7 +710,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             return run_4r4w(j, o);
         case SAT_4R1W:
             if (batch > 65535) return fail(SAT_ERR_UNSUPPORTED, "4R1W: batch must be <= 65535");
-            return dtype == SAT_INT32 ? run_4r1w_t<uint32_t>(j) : run_4r1w_t<float>(j);
+            return SAT_DISPATCH(dtype, T, run_4r1w_t<T>(j));
     }
     return fail(SAT_ERR_INVALID, "bad variant");
 }
@@ -709,19 +743,15 @@ int column_totals_core(const void* in, void* totals, int64_t rows, int64_t cols,
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
-    return dtype == SAT_INT32 ? column_totals_t<uint32_t>(in, totals, rows, cols, di, *ws, st)
-                              : column_totals_t<float>(in, totals, rows, cols, di, *ws, st);
+    return SAT_DISPATCH(dtype, T, column_totals_t<T>(in, totals, rows, cols, di, *ws, st));
 }
 
 int exscan_core(const void* gathered, void* carry, int64_t nranks, int64_t cols, int rank,
                 int dtype, cudaStream_t st) {
     const unsigned blocks = unsigned((cols + 255) / 256);
-    if (dtype == SAT_INT32)
-        sat_rank_exscan_kernel<uint32_t><<<blocks, 256, 0, st>>>(
-            static_cast<const uint32_t*>(gathered), static_cast<uint32_t*>(carry), cols, rank);
-    else
-        sat_rank_exscan_kernel<float><<<blocks, 256, 0, st>>>(
-            static_cast<const float*>(gathered), static_cast<float*>(carry), cols, rank);
+    SAT_DISPATCH(dtype, T, (sat_rank_exscan_kernel<T><<<blocks, 256, 0, st>>>(
+                                static_cast<const T*>(gathered), static_cast<T*>(carry), cols, rank),
+                            0));
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     return SAT_OK;
@@ -776,7 +806,7 @@ int sat_column_totals(const void* in, void* totals, int64_t rows, int64_t cols, 
     SAT_TRY(validate(in, totals, 1, rows, cols, dtype, true));
     if (rows == 0 || cols == 0) {
         if (cols > 0 && totals)
-            CUDA_TRY(cudaMemsetAsync(totals, 0, size_t(cols) * 4, static_cast<cudaStream_t>(stream)));
+            CUDA_TRY(cudaMemsetAsync(totals, 0, size_t(cols) * esize(dtype), static_cast<cudaStream_t>(stream)));
         return SAT_OK;
     }
     return column_totals_core(in, totals, rows, cols, dtype, static_cast<cudaStream_t>(stream));
@@ -785,7 +815,7 @@ int sat_column_totals(const void* in, void* totals, int64_t rows, int64_t cols, 
 int sat_rank_exscan(const void* gathered, void* carry_row, int64_t nranks, int64_t cols, int rank,
                     int dtype, void* stream) {
     t_launches = 0;
-    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (!dtype_ok(dtype)) return fail(SAT_ERR_INVALID, "bad dtype");
     if (nranks < 1 || rank < 0 || rank >= nranks || cols < 0)
         return fail(SAT_ERR_INVALID, "bad rank / nranks / cols");
     if (cols == 0) return SAT_OK;
@@ -795,9 +825,8 @@ int sat_rank_exscan(const void* gathered, void* carry_row, int64_t nranks, int64
 }
 
 size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype) {
-    (void)dtype;
     if (cols <= 0 || nranks <= 0) return 0;
-    const size_t row = align256(size_t(cols) * 4);
+    const size_t row = align256(size_t(cols) * (dtype == SAT_FLOAT64 ? 8 : 4));
     return row * size_t(nranks + 2);
 }
 
@@ -811,7 +840,8 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
     if (nranks > 1 && !allgather) return fail(SAT_ERR_INVALID, "allgather callback required");
     if (stats) std::memset(stats, 0, sizeof(*stats));
     if (cols == 0) return SAT_OK;
-    const size_t row = align256(size_t(cols) * 4);
+    const size_t eb = esize(dtype);
+    const size_t row = align256(size_t(cols) * eb);
     uint8_t* wsp = static_cast<uint8_t*>(workspace);
     if (!wsp) {
         int dev;
@@ -834,10 +864,10 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
             SAT_TRY(column_totals_core(in_strip, send, strip_rows, cols, dtype, st));
             launches += t_launches;
         } else {
-            CUDA_TRY(cudaMemsetAsync(send, 0, size_t(cols) * 4, st));
+            CUDA_TRY(cudaMemsetAsync(send, 0, size_t(cols) * eb, st));
         }
         // 2. all-gather of the m-vectors (NCCL over NVLink in the Python binding)
-        if (allgather(comm_ctx, send, recv, size_t(cols) * 4, stream) != 0)
+        if (allgather(comm_ctx, send, recv, size_t(cols) * eb, stream) != 0)
             return fail(SAT_ERR_COMM, "allgather callback failed");
         // 3. exclusive scan over ranks
         if (rank > 0) {
@@ -855,11 +885,11 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
     }
     t_launches = launches;
     if (stats) {
-        const int64_t b = strip_rows * cols * 4;
+        const int64_t b = strip_rows * cols * int64_t(eb);
         stats->strip_bytes_read = b;
         stats->strip_bytes_written = b;
         stats->extra_bytes_read = (nranks > 1 && rank < nranks - 1) ? b : 0;
-        stats->allgather_bytes = nranks > 1 ? int64_t(nranks) * cols * 4 : 0;
+        stats->allgather_bytes = nranks > 1 ? int64_t(nranks) * cols * int64_t(eb) : 0;
     }
     return SAT_OK;
 }
@@ -868,7 +898,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
                      int variant, void* stream) {
     t_launches = 0;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
-    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (!dtype_ok(dtype)) return fail(SAT_ERR_INVALID, "bad dtype");
     if (rows < 0 || cols < 0) return fail(SAT_ERR_INVALID, "negative size");
     if (rows == 0 || cols == 0) return SAT_OK;
     if (!in_host || !out_host) return fail(SAT_ERR_INVALID, "null pointer");
@@ -877,7 +907,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
-    const size_t bytes = size_t(rows) * size_t(cols) * 4;
+    const size_t bytes = size_t(rows) * size_t(cols) * esize(dtype);
     SAT_TRY(ensure(ws->din, bytes, false));
     SAT_TRY(ensure(ws->dout, bytes, false));
     cudaPointerAttributes ai, ao;
@@ -917,7 +947,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     uint8_t* hout = static_cast<uint8_t*>(out_host);
     uint8_t* din = static_cast<uint8_t*>(ws->din.p);
     uint8_t* dout = static_cast<uint8_t*>(ws->dout.p);
-    const size_t rowb = size_t(cols) * 4;
+    const size_t rowb = size_t(cols) * esize(dtype);
     for (int k = 0; k < nstrips; ++k) {
         const int64_t r0 = k * srows, r1 = std::min<int64_t>(rows, r0 + srows);
         if (r1 <= r0) { CUDA_TRY(cudaEventRecord(ev_in[k], ws->cstream_in)); continue; }

@@ -46,9 +46,7 @@ sat_reduce_kernel(const TileParams p)
         T e[4] = {T(0), T(0), T(0), T(0)};
         if (row < p.rows) {
             if (vec && c + 3 < p.cols) {
-                uint4 u = __ldg(reinterpret_cast<const uint4*>(gin + row * p.cols + c));
-                e[0] = from_bits<T>(u.x); e[1] = from_bits<T>(u.y);
-                e[2] = from_bits<T>(u.z); e[3] = from_bits<T>(u.w);
+                ldg4<T>(gin + row * p.cols + c, e);
             } else {
 #pragma unroll
                 for (int i = 0; i < 4; ++i) if (c + i < p.cols) e[i] = gin[row * p.cols + c + i];
@@ -179,9 +177,10 @@ sat_colsum_partial_kernel(const T* __restrict__ in, T* __restrict__ part,
     T cs[4] = {T(0), T(0), T(0), T(0)};
     for (int64_t r = r0 + warp; r < r1; r += 8) {
         if (vec) {
-            uint4 u = __ldg(reinterpret_cast<const uint4*>(in + r * cols + c));
-            cs[0] += from_bits<T>(u.x); cs[1] += from_bits<T>(u.y);
-            cs[2] += from_bits<T>(u.z); cs[3] += from_bits<T>(u.w);
+            T e[4];
+            ldg4<T>(in + r * cols + c, e);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) cs[i] += e[i];
         } else {
 #pragma unroll
             for (int i = 0; i < 4; ++i) if (c + i < cols) cs[i] += in[r * cols + c + i];

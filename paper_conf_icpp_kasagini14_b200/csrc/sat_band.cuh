@@ -45,19 +45,32 @@ namespace sat {
 template <typename T>
 struct V4 { T x, y, z, w; };
 
+// 4 consecutive elements (16 B, or 32 B for float64) as vector accesses
+template <typename T>
+__device__ __forceinline__ void v4_words(const V4<T>& v, uint32_t (&w)[4 * Words<T>::N]) {
+    const T e[4] = {v.x, v.y, v.z, v.w};
+    pack<T, 4>(e, w);
+}
 template <typename T>
 __device__ __forceinline__ V4<T> lds4(const T* p) {
-    uint4 u = *reinterpret_cast<const uint4*>(p);
-    return V4<T>{from_bits<T>(u.x), from_bits<T>(u.y), from_bits<T>(u.z), from_bits<T>(u.w)};
+    uint32_t w[4 * Words<T>::N];
+    ld_words<4 * Words<T>::N>(p, w);
+    T e[4];
+    unpack<T, 4>(w, e);
+    return V4<T>{e[0], e[1], e[2], e[3]};
 }
 template <typename T>
 __device__ __forceinline__ void sts4(T* p, const V4<T>& v) {
-    *reinterpret_cast<uint4*>(p) = make_uint4(to_bits(v.x), to_bits(v.y), to_bits(v.z), to_bits(v.w));
+    uint32_t w[4 * Words<T>::N];
+    v4_words(v, w);
+    st_words<4 * Words<T>::N>(p, w);
 }
-// 16-B streaming store (evict-first: the SAT is not re-read by this kernel)
+// streaming store (evict-first: the SAT is not re-read by this kernel)
 template <typename T>
 __device__ __forceinline__ void st_global_v4(T* p, const V4<T>& v) {
-    __stcs(reinterpret_cast<uint4*>(p), make_uint4(to_bits(v.x), to_bits(v.y), to_bits(v.z), to_bits(v.w)));
+    uint32_t w[4 * Words<T>::N];
+    v4_words(v, w);
+    stcs_words<4 * Words<T>::N>(p, w);
 }
 template <typename T>
 __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
@@ -87,49 +100,40 @@ __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
 // CPL consecutive columns (4, 2 or 1) as one shared-memory vector access.
 template <typename T, int CPL>
 __device__ __forceinline__ void lds_cols(const T* p, T (&v)[CPL]) {
-    if constexpr (CPL == 4) {
-        const uint4 u = *reinterpret_cast<const uint4*>(p);
-        v[0] = from_bits<T>(u.x); v[1] = from_bits<T>(u.y); v[2] = from_bits<T>(u.z); v[3] = from_bits<T>(u.w);
-    } else if constexpr (CPL == 2) {
-        const uint2 u = *reinterpret_cast<const uint2*>(p);
-        v[0] = from_bits<T>(u.x); v[1] = from_bits<T>(u.y);
-    } else {
-        v[0] = *p;
-    }
+    uint32_t w[CPL * Words<T>::N];
+    ld_words<CPL * Words<T>::N>(p, w);
+    unpack<T, CPL>(w, v);
 }
 template <typename T, int CPL>
 __device__ __forceinline__ void sts_cols(T* p, const T (&v)[CPL]) {
-    if constexpr (CPL == 4) {
-        *reinterpret_cast<uint4*>(p) = make_uint4(to_bits(v[0]), to_bits(v[1]), to_bits(v[2]), to_bits(v[3]));
-    } else if constexpr (CPL == 2) {
-        *reinterpret_cast<uint2*>(p) = make_uint2(to_bits(v[0]), to_bits(v[1]));
-    } else {
-        *p = v[0];
-    }
+    uint32_t w[CPL * Words<T>::N];
+    pack<T, CPL>(v, w);
+    st_words<CPL * Words<T>::N>(p, w);
 }
 
-// Descriptor words (tag << 32 | value bits) of CPL consecutive columns.
-template <int CPL>
-__device__ __forceinline__ void load_words(const uint64_t* q, uint64_t (&w)[CPL]) {
-    if constexpr (CPL == 4) {
-        ld_relaxed_v2(q, w[0], w[1]);
-        ld_relaxed_v2(q + 2, w[2], w[3]);
-    } else if constexpr (CPL == 2) {
-        ld_relaxed_v2(q, w[0], w[1]);
+// Descriptor words (tag << 32 | 32 value bits): NW consecutive words, each
+// single-copy atomic at gpu scope (a float64 value is two words, low first).
+template <int NW>
+__device__ __forceinline__ void load_words(const uint64_t* q, uint64_t (&w)[NW]) {
+    if constexpr (NW % 2 == 0) {
+#pragma unroll
+        for (int k = 0; k < NW; k += 2) ld_relaxed_v2(q + k, w[k], w[k + 1]);
     } else {
+        static_assert(NW == 1, "1 or 2k words");
         asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w[0]) : "l"(q) : "memory");
     }
 }
 template <typename T, int CPL>
 __device__ __forceinline__ void publish_words(uint64_t* my, uint32_t tag, const T (&v)[CPL]) {
+    constexpr int NW = CPL * Words<T>::N;
     const uint64_t hi = uint64_t(tag) << 32;
-    if constexpr (CPL == 4) {
-        st_relaxed_v2(my, hi | to_bits(v[0]), hi | to_bits(v[1]));
-        st_relaxed_v2(my + 2, hi | to_bits(v[2]), hi | to_bits(v[3]));
-    } else if constexpr (CPL == 2) {
-        st_relaxed_v2(my, hi | to_bits(v[0]), hi | to_bits(v[1]));
+    uint32_t w[NW];
+    pack<T, CPL>(v, w);
+    if constexpr (NW % 2 == 0) {
+#pragma unroll
+        for (int k = 0; k < NW; k += 2) st_relaxed_v2(my + k, hi | w[k], hi | w[k + 1]);
     } else {
-        asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" :: "l"(my), "l"(hi | to_bits(v[0])) : "memory");
+        asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" :: "l"(my), "l"(hi | w[0]) : "memory");
     }
 }
 
@@ -232,15 +236,34 @@ __device__ __forceinline__ void tmem_ld<32>(uint32_t t, uint32_t (&r)[32]) {
                    "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]),
                    "=r"(r[30]), "=r"(r[31]) : "r"(t) : "memory");
 }
+template <>
+__device__ __forceinline__ void tmem_st<64>(uint32_t t, const uint32_t (&r)[64]) {
+    // two x32 stores into adjacent column ranges
+    uint32_t a[32], b[32];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) { a[i] = r[i]; b[i] = r[32 + i]; }
+    tmem_st<32>(t, a);
+    tmem_st<32>(t + 32, b);
+}
+template <>
+__device__ __forceinline__ void tmem_ld<64>(uint32_t t, uint32_t (&r)[64]) {
+    uint32_t a[32], b[32];
+    tmem_ld<32>(t, a);
+    tmem_ld<32>(t + 32, b);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) { r[i] = a[i]; r[32 + i] = b[i]; }
+}
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tmem_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// TMEM columns per CTA for W compute warps holding DT chunks of R x 4 words.
-template <int R, int W, int DT>
+// TMEM columns per CTA for W compute warps holding DT chunks of R x 4
+// elements of NWE 32-bit words each.
+template <int R, int W, int DT, int NWE = 1>
 struct TmemCols {
-    static constexpr int per_warp = DT * 4 * R;
+    static constexpr int per_chunk = 4 * R * NWE;
+    static constexpr int per_warp = DT * per_chunk;
     static constexpr int need = per_warp * ((W + 3) / 4);       // warps w, w+4, .. share lanes
     static constexpr int alloc = need <= 32 ? 32 : need <= 64 ? 64 : need <= 128 ? 128
                                  : need <= 256 ? 256 : 512;
@@ -258,8 +281,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
     using SM = BandSmem<T, R, W, S, DT, SUB, CL>;
-    static_assert(CL == 1 || (MODE == MODE_SAT && NS == 1), "clusters: 1R1W band kernel only");
-    using TC = TmemCols<R, W, DT>;
+    static_assert(CL == 1 || (MODE == MODE_SAT && NS == 1 && sizeof(T) == 4), "clusters: 1R1W band kernel only");
+    constexpr int NWE = Words<T>::N;             // 32-bit words per element
+    using TC = TmemCols<R, W, DT, NWE>;
     constexpr int XS = SM::XS;
     constexpr bool HOLD = (MODE != MODE_ROW);    // chunks wait for a vertical carry
     // A control warp waits on colr[] of chunk k only after finishing chunk
@@ -400,19 +424,25 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 // row carry from segment seg-1 of this band (an earlier ticket,
                 // normally long finished): lane r < R polls row rbase + r
                 const uint32_t want = band_tag(p.base, (seg - 1) * p.total_bands + gb) | 3u;
-                const uint64_t* q = p.Lseg + int64_t(gb) * TH + rbase + (lane < R ? lane : 0);
+                const bool mine = lane < R * NWE;        // word `lane` of this warp's rows
+                const uint64_t* q = p.Lseg + (int64_t(gb) * TH + rbase) * NWE + (mine ? lane : 0);
                 uint64_t wv;
                 asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(wv) : "l"(q) : "memory");
-                if (__any_sync(0xffffffffu, lane < R && uint32_t(wv >> 32) != want)) {
+                if (__any_sync(0xffffffffu, mine && uint32_t(wv >> 32) != want)) {
                     SpinGuard guard(0x20000000u | uint32_t(gb), uint32_t(seg));
-                    while (__any_sync(0xffffffffu, lane < R && uint32_t(wv >> 32) != want)) {
+                    while (__any_sync(0xffffffffu, mine && uint32_t(wv >> 32) != want)) {
                         __nanosleep(64);
                         guard.tick();
                         asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(wv) : "l"(q) : "memory");
                     }
                 }
 #pragma unroll
-                for (int r = 0; r < R; ++r) L[r] = from_bits<T>(__shfl_sync(0xffffffffu, uint32_t(wv), r));
+                for (int r = 0; r < R; ++r) {
+                    uint32_t w[NWE];
+#pragma unroll
+                    for (int k = 0; k < NWE; ++k) w[k] = __shfl_sync(0xffffffffu, uint32_t(wv), r * NWE + k);
+                    L[r] = from_words<T>(w);
+                }
             }
             const T* gin = reinterpret_cast<const T*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
@@ -462,9 +492,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         // proxy: without this, a quick refill overtook the LDS
                         // (seen as corrupted rows with 4 compute warps)
 #pragma unroll
-                        for (int r = 0; r < R; ++r)
-                            asm volatile("" :: "r"(to_bits(v[r].x)), "r"(to_bits(v[r].y)),
-                                         "r"(to_bits(v[r].z)), "r"(to_bits(v[r].w)));
+                        for (int r = 0; r < R; ++r) {
+                            uint32_t w[4 * NWE];
+                            v4_words(v[r], w);
+#pragma unroll
+                            for (int k = 0; k < 4 * NWE; ++k) asm volatile("" :: "r"(w[k]));
+                        }
                         fence_proxy_async_smem();
                         mbar_arrive(&empty[s]);
                     }
@@ -486,13 +519,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 } else {
 #pragma unroll
                     for (int r = 1; r < R; ++r) add4(v[r], v[r - 1]);
-                    uint32_t u[4 * R];
+                    uint32_t u[TC::per_chunk];
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
-                        u[4 * r + 0] = to_bits(v[r].x); u[4 * r + 1] = to_bits(v[r].y);
-                        u[4 * r + 2] = to_bits(v[r].z); u[4 * r + 3] = to_bits(v[r].w);
+                        const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) to_words<T>(e[i], u + (4 * r + i) * NWE);
                     }
-                    tmem_st<4 * R>(tm_warp + uint32_t((it % DT) * 4 * R), u);
+                    tmem_st<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
                     sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
                     mbar_arrive(&colr[it % XS]);
                 }
@@ -505,15 +539,16 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 if (traced && warp == 0 && lane == 0)
                     p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
                 const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
-                uint32_t u[4 * R];
+                uint32_t u[TC::per_chunk];
                 tmem_wait_st();
-                tmem_ld<4 * R>(tm_warp + uint32_t((it % DT) * 4 * R), u);
+                tmem_ld<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
                 tmem_wait_ld();
                 V4<T> v[R];
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
-                    v[r] = V4<T>{from_bits<T>(u[4 * r]), from_bits<T>(u[4 * r + 1]),
-                                 from_bits<T>(u[4 * r + 2]), from_bits<T>(u[4 * r + 3])};
+                    const uint32_t* q = u + 4 * r * NWE;
+                    v[r] = V4<T>{from_words<T>(q), from_words<T>(q + NWE), from_words<T>(q + 2 * NWE),
+                                 from_words<T>(q + 3 * NWE)};
                     add4(v[r], add);
                 }
                 store_rows(v, k);
@@ -532,13 +567,16 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 }
                 for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
             }
-            if (p.nseg > 1 && seg + 1 < p.nseg && lane < R) {
-                // hand the row carry to segment seg+1 of this band
-                T mine = L[0];
+            if (p.nseg > 1 && seg + 1 < p.nseg && lane < R * NWE) {
+                // hand the row carry to segment seg+1 of this band (word `lane`)
+                uint32_t wl[R * NWE];
+                pack<T, R>(L, wl);
+                uint32_t mine = wl[0];
 #pragma unroll
-                for (int r = 1; r < R; ++r) if (lane == r) mine = L[r];
-                const uint64_t w = (uint64_t(band_tag(p.base, seg * p.total_bands + gb) | 3u) << 32) | to_bits(mine);
-                asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" :: "l"(p.Lseg + int64_t(gb) * TH + rbase + lane), "l"(w) : "memory");
+                for (int k = 1; k < R * NWE; ++k) if (lane == k) mine = wl[k];
+                const uint64_t w = (uint64_t(band_tag(p.base, seg * p.total_bands + gb) | 3u) << 32) | mine;
+                asm volatile("st.relaxed.gpu.global.b64 [%0], %1;"
+                             :: "l"(p.Lseg + (int64_t(gb) * TH + rbase) * NWE + lane), "l"(w) : "memory");
             }
             if (p.Lb != nullptr && !p.tile_units && lane == 0) {
                 T* lb = reinterpret_cast<T*>(p.Lb) + int64_t(gb) * TH + rbase;
@@ -554,7 +592,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if constexpr (HOLD) {
                 constexpr int CPL = 4 / NS;
                 constexpr int G = NCW / NS;
-                constexpr int LBW = LBW_ > 0 ? LBW_ : 16 / CPL;   // bands per look-back round trip
+                constexpr int NW = CPL * NWE;                  // descriptor words per band
+                constexpr int LBW = LBW_ > 0 ? LBW_ : (16 / NW > 0 ? 16 / NW : 1);   // bands per round trip
                 const int cw = warp - CW;
                 const int grp = cw / NS;
                 const int cl = (cw % NS) * (TW / NS) + lane * CPL;   // column within the chunk
@@ -579,7 +618,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) agg[i] += b[i];
                     }
-                    uint64_t* my = p.desc + int64_t(gb) * desc_w + c0;
+                    uint64_t* my = p.desc + (int64_t(gb) * desc_w + c0) * NWE;
                     if (p.jitter && lookback) {
                         uint32_t h = (uint32_t(gb) * 2654435761u) ^ (uint32_t(J) * 40503u) ^ (uint32_t(cl) * 97u);
                         h ^= h >> 13; h *= 0x5bd1e995u; h ^= h >> 15;
@@ -600,15 +639,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     int kb = idx - 1;
                     SpinGuard guard(0x80000000u | uint32_t(J), uint32_t(gidx));
                     while (pend) {
-                        uint64_t wv[LBW][CPL];
+                        uint64_t wv[LBW][NW];
 #pragma unroll
                         for (int q = 0; q < LBW; ++q) {
                             const int b2 = kb - q;
                             if (b2 >= 0) {
-                                load_words<CPL>(p.desc + (int64_t(gidx) - (idx - b2)) * desc_w + c0, wv[q]);
+                                load_words<NW>(p.desc + ((int64_t(gidx) - (idx - b2)) * desc_w + c0) * NWE, wv[q]);
                             } else {
 #pragma unroll
-                                for (int i = 0; i < CPL; ++i) wv[q][i] = 0;
+                                for (int i = 0; i < NW; ++i) wv[q][i] = 0;
                             }
                         }
                         bool stalled = false;
@@ -629,16 +668,26 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             const uint32_t tk = band_tag(p.base, gidx - (idx - b2));
                             bool ready = true;
 #pragma unroll
-                            for (int i = 0; i < CPL; ++i) {
+                            for (int i = 0; i < NW; ++i) {
                                 const uint32_t t = uint32_t(wv[q][i] >> 32);
                                 ready = ready && ((t & ~3u) == tk) && (t & 3u);
                             }
+                            // the words of one float64 value must come from the
+                            // same publication (aggregate and inclusive share a slot)
+#pragma unroll
+                            for (int i = 0; i < CPL; ++i)
+#pragma unroll
+                                for (int k = 1; k < NWE; ++k)
+                                    ready = ready && (uint32_t(wv[q][i * NWE + k] >> 32) == uint32_t(wv[q][i * NWE] >> 32));
                             if (!ready) { stalled = true; kb = b2; break; }
 #pragma unroll
                             for (int i = 0; i < CPL; ++i) {
                                 if ((pend >> i) & 1u) {
-                                    top[i] += from_bits<T>(uint32_t(wv[q][i]));
-                                    if ((uint32_t(wv[q][i] >> 32) & 3u) == 2u) pend &= ~(1u << i);
+                                    uint32_t w[NWE];
+#pragma unroll
+                                    for (int k = 0; k < NWE; ++k) w[k] = uint32_t(wv[q][i * NWE + k]);
+                                    top[i] += from_words<T>(w);
+                                    if ((uint32_t(wv[q][i * NWE] >> 32) & 3u) == 2u) pend &= ~(1u << i);
                                 }
                             }
                             ++hops;

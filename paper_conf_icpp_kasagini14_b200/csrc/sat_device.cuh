@@ -201,13 +201,100 @@ __device__ __forceinline__ unsigned long long globaltimer() {
 }
 
 // ------------------------------------------------------------- arithmetic
-// int32 SATs are computed in uint32 (mod 2^32); float32 in IEEE fp32 adds.
+// int32 SATs are computed in uint32 (mod 2^32); float32 in IEEE fp32 adds;
+// float64 (the paper's precision) in IEEE fp64 adds.
 template <typename T> __device__ __forceinline__ uint32_t to_bits(T v);
 template <> __device__ __forceinline__ uint32_t to_bits<uint32_t>(uint32_t v) { return v; }
 template <> __device__ __forceinline__ uint32_t to_bits<float>(float v) { return __float_as_uint(v); }
 template <typename T> __device__ __forceinline__ T from_bits(uint32_t v);
 template <> __device__ __forceinline__ uint32_t from_bits<uint32_t>(uint32_t v) { return v; }
 template <> __device__ __forceinline__ float from_bits<float>(uint32_t v) { return __uint_as_float(v); }
+
+// 32-bit words per element (1 for int32/float32, 2 for float64) and the
+// conversions between an element and its words (low word first).
+template <typename T> struct Words { static constexpr int N = int(sizeof(T) / 4); };
+template <typename T>
+__device__ __forceinline__ void to_words(T v, uint32_t* w) {
+    if constexpr (sizeof(T) == 8) {
+        w[0] = uint32_t(__double2loint(v));
+        w[1] = uint32_t(__double2hiint(v));
+    } else {
+        w[0] = to_bits<T>(v);
+    }
+}
+template <typename T>
+__device__ __forceinline__ T from_words(const uint32_t* w) {
+    if constexpr (sizeof(T) == 8) return __hiloint2double(int(w[1]), int(w[0]));
+    else return from_bits<T>(w[0]);
+}
+
+// N consecutive 32-bit words (N*4 B, naturally aligned) with the widest
+// vector accesses: generic (shared or global) load / store, read-only global
+// load, streaming (evict-first) global store.
+template <int N>
+__device__ __forceinline__ void ld_words(const void* p, uint32_t (&w)[N]) {
+    if constexpr (N % 4 == 0) {
+#pragma unroll
+        for (int k = 0; k < N / 4; ++k) {
+            const uint4 u = reinterpret_cast<const uint4*>(p)[k];
+            w[4 * k] = u.x; w[4 * k + 1] = u.y; w[4 * k + 2] = u.z; w[4 * k + 3] = u.w;
+        }
+    } else if constexpr (N == 2) {
+        const uint2 u = *reinterpret_cast<const uint2*>(p);
+        w[0] = u.x; w[1] = u.y;
+    } else {
+        static_assert(N == 1, "1, 2 or 4k words");
+        w[0] = *reinterpret_cast<const uint32_t*>(p);
+    }
+}
+template <int N>
+__device__ __forceinline__ void st_words(void* p, const uint32_t (&w)[N]) {
+    if constexpr (N % 4 == 0) {
+#pragma unroll
+        for (int k = 0; k < N / 4; ++k)
+            reinterpret_cast<uint4*>(p)[k] = make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]);
+    } else if constexpr (N == 2) {
+        *reinterpret_cast<uint2*>(p) = make_uint2(w[0], w[1]);
+    } else {
+        static_assert(N == 1, "1, 2 or 4k words");
+        *reinterpret_cast<uint32_t*>(p) = w[0];
+    }
+}
+template <int N>
+__device__ __forceinline__ void ldg_words(const void* p, uint32_t (&w)[N]) {
+    static_assert(N % 4 == 0, "16-B vectors");
+#pragma unroll
+    for (int k = 0; k < N / 4; ++k) {
+        const uint4 u = __ldg(reinterpret_cast<const uint4*>(p) + k);
+        w[4 * k] = u.x; w[4 * k + 1] = u.y; w[4 * k + 2] = u.z; w[4 * k + 3] = u.w;
+    }
+}
+template <int N>
+__device__ __forceinline__ void stcs_words(void* p, const uint32_t (&w)[N]) {
+    static_assert(N % 4 == 0, "16-B vectors");
+#pragma unroll
+    for (int k = 0; k < N / 4; ++k)
+        __stcs(reinterpret_cast<uint4*>(p) + k, make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]));
+}
+
+// K consecutive elements <-> their words
+template <typename T, int K>
+__device__ __forceinline__ void pack(const T (&v)[K], uint32_t (&w)[K * Words<T>::N]) {
+#pragma unroll
+    for (int i = 0; i < K; ++i) to_words<T>(v[i], w + i * Words<T>::N);
+}
+template <typename T, int K>
+__device__ __forceinline__ void unpack(const uint32_t (&w)[K * Words<T>::N], T (&v)[K]) {
+#pragma unroll
+    for (int i = 0; i < K; ++i) v[i] = from_words<T>(w + i * Words<T>::N);
+}
+// 4 consecutive elements by 16-B vector loads (read-only path)
+template <typename T>
+__device__ __forceinline__ void ldg4(const T* p, T (&e)[4]) {
+    uint32_t w[4 * Words<T>::N];
+    ldg_words<4 * Words<T>::N>(p, w);
+    unpack<T, 4>(w, e);
+}
 
 // Inclusive warp scan of x (lane order).  Kogge-Stone with shfl.up.
 template <typename T>
