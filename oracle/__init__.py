@@ -56,6 +56,8 @@ def _load():
             getattr(lib, f"oracle_sat_{k}_2pass").argtypes = [_P, _P, _I64, _I64]
             getattr(lib, f"oracle_sat_{k}_brute").argtypes = [_P, _P, _I64, _I64]
             getattr(lib, f"oracle_sat_{k}_at").argtypes = [_P, _I64, _I64, _I64, _I64]
+        for k in _KINDS:
+            getattr(lib, f"oracle_box_{k}").argtypes = [_P, _P, _I64, _I64, _I64, _I64]
         lib.oracle_sat_u32_at.restype = ctypes.c_uint32
         lib.oracle_sat_f64_at.restype = ctypes.c_double
         lib.oracle_sat_d64_at.restype = ctypes.c_double
@@ -194,6 +196,29 @@ def rect_sum(b: np.ndarray, r0: int, c0: int, r1: int, c1: int):
         return bb[i, j]
     with np.errstate(over="ignore"):
         return at(r1, c1) - at(r0 - 1, c1) - at(r1, c0 - 1) + at(r0 - 1, c0 - 1)
+
+
+def box_filter(a: np.ndarray, rr: int, rc: int, normalize: bool = False) -> np.ndarray:
+    """Box filter by its plain definition (the SAT's use case,
+    P:L193, L221): out[i][j] = sum of a over rows |k - i| <= rr and columns
+    |l - j| <= rc, clipped to the matrix.  int32 -> uint32 sums (returned as
+    int32), float -> float64.  ``normalize`` divides by the clipped window's
+    element count (a box mean; float inputs only).  O(n m rr rc): small inputs."""
+    a_c, is_int, odt = _prep(a)
+    out = np.empty(a_c.shape, dtype=odt)
+    if a_c.size:
+        getattr(_load(), f"oracle_box_{_kind(a_c)}")(_ptr(a_c), _ptr(out), a_c.shape[0],
+                                                      a_c.shape[1], int(rr), int(rc))
+    if normalize:
+        if is_int:
+            raise ValueError("normalize is for float inputs")
+        n, m = a_c.shape
+        i = np.arange(n)
+        j = np.arange(m)
+        ci = np.minimum(n - 1, i + rr) - np.maximum(0, i - rr) + 1
+        cj = np.minimum(m - 1, j + rc) - np.maximum(0, j - rc) + 1
+        out = out / (ci[:, None] * cj[None, :]).astype(np.float64)
+    return _ret(out, a.dtype)
 
 
 def column_totals(a: np.ndarray) -> np.ndarray:

@@ -210,3 +210,51 @@ void oracle_sat_d64_brute(const double *a, double *b, int64_t rows, int64_t cols
         for (int64_t j = 0; j < cols; ++j)
             b[i * cols + j] = oracle_sat_d64_at(a, rows, cols, i, j);
 }
+
+/* ---------------- box filter (the SAT's motivating use, P:L193, L221;
+ * SURVEY 8(f2)) written as its plain definition: the sum of the input over
+ * the (2*rr+1) x (2*rc+1) window centred on (i, j), clipped to the matrix.
+ * O(rows * cols * window): test sizes only. ---------------- */
+
+static int64_t lo_clip(int64_t x) { return x < 0 ? 0 : x; }
+static int64_t hi_clip(int64_t x, int64_t n) { return x > n - 1 ? n - 1 : x; }
+
+void oracle_box_u32(const uint32_t *a, uint32_t *out, int64_t rows, int64_t cols,
+                    int64_t rr, int64_t rc)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 0; j < cols; ++j) {
+            uint32_t s = 0;
+            for (int64_t k = lo_clip(i - rr); k <= hi_clip(i + rr, rows); ++k)
+                for (int64_t l = lo_clip(j - rc); l <= hi_clip(j + rc, cols); ++l)
+                    s += a[k * cols + l];
+            out[i * cols + j] = s;
+        }
+}
+
+/* float32 input summed in float64 */
+void oracle_box_f64(const float *a, double *out, int64_t rows, int64_t cols,
+                    int64_t rr, int64_t rc)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 0; j < cols; ++j) {
+            double s = 0.0;
+            for (int64_t k = lo_clip(i - rr); k <= hi_clip(i + rr, rows); ++k)
+                for (int64_t l = lo_clip(j - rc); l <= hi_clip(j + rc, cols); ++l)
+                    s += (double)a[k * cols + l];
+            out[i * cols + j] = s;
+        }
+}
+
+void oracle_box_d64(const double *a, double *out, int64_t rows, int64_t cols,
+                    int64_t rr, int64_t rc)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        for (int64_t j = 0; j < cols; ++j) {
+            double s = 0.0;
+            for (int64_t k = lo_clip(i - rr); k <= hi_clip(i + rr, rows); ++k)
+                for (int64_t l = lo_clip(j - rc); l <= hi_clip(j + rc, cols); ++l)
+                    s += a[k * cols + l];
+            out[i * cols + j] = s;
+        }
+}

@@ -320,3 +320,62 @@ def test_1d_is_cumsum_float64(shape):
     a = make_np(*shape, "float64", "unit53", seed=4)
     for form in FORMS:
         assert np.array_equal(form(a).ravel(), np.cumsum(a.ravel()))
+
+
+# ---------------------------------------------------------------- box filter
+def py_box(a, rr, rc):
+    """Pure-Python windowed sum (independent of the oracle's C code)."""
+    n, m = len(a), len(a[0])
+    return [[sum(a[k][l] for k in range(max(0, i - rr), min(n - 1, i + rr) + 1)
+                 for l in range(max(0, j - rc), min(m - 1, j + rc) + 1))
+             for j in range(m)] for i in range(n)]
+
+
+@pytest.mark.parametrize("n,m,rr,rc", [(1, 1, 0, 0), (3, 4, 1, 1), (5, 7, 2, 1), (7, 5, 0, 3),
+                                       (6, 6, 9, 9), (9, 13, 1, 4)])
+def test_box_brute(n, m, rr, rc):
+    a = make_np(n, m, "int32", "u8", seed=n * m)
+    assert np.array_equal(oracle.box_filter(a, rr, rc), np.array(py_box(a.tolist(), rr, rc)))
+    f = make_np(n, m, "float64", "unit", seed=n + m)
+    assert np.array_equal(oracle.box_filter(f, rr, rc), np.array(py_box(f.tolist(), rr, rc)))
+
+
+def test_box_worked_3x4():
+    a = np.arange(12, dtype=np.int32).reshape(3, 4)
+    assert oracle.box_filter(a, 1, 1).tolist() == [[10, 18, 24, 18], [27, 45, 54, 39],
+                                                   [26, 42, 48, 34]]
+
+
+def test_box_closed_forms():
+    n, m, rr, rc = 37, 53, 3, 5
+    ones = np.ones((n, m), dtype=np.int32)
+    i, j = np.arange(n), np.arange(m)
+    ci = np.minimum(n - 1, i + rr) - np.maximum(0, i - rr) + 1
+    cj = np.minimum(m - 1, j + rc) - np.maximum(0, j - rc) + 1
+    assert np.array_equal(oracle.box_filter(ones, rr, rc), ci[:, None] * cj[None, :])
+    # separable a = f(i) g(j): window sums factor (f != g catches a swap of rr/rc)
+    f = np.arange(n, dtype=np.int64) % 5 + 1
+    g = np.arange(m, dtype=np.int64) % 3 + 2
+    a = (f[:, None] * g[None, :]).astype(np.int32)
+    wf = np.array([f[max(0, k - rr):k + rr + 1].sum() for k in range(n)])
+    wg = np.array([g[max(0, k - rc):k + rc + 1].sum() for k in range(m)])
+    assert np.array_equal(oracle.box_filter(a, rr, rc), wf[:, None] * wg[None, :])
+    # radius 0 is the identity; a radius covering everything is the total
+    b = make_np(20, 30, "int32", "u32", seed=3)
+    assert np.array_equal(oracle.box_filter(b, 0, 0), b)
+    tot = b.view(np.uint32).sum(dtype=np.uint64) % 2**32
+    assert (oracle.box_filter(b, 40, 40).view(np.uint32) == tot).all()
+    # the box mean of a constant is the constant
+    c = np.full((9, 11), 0.75, dtype=np.float32)
+    assert np.allclose(oracle.box_filter(c, 2, 3, normalize=True), 0.75, rtol=0, atol=1e-15)
+
+
+def test_box_equals_four_sat_reads():
+    """Inclusion-exclusion over the oracle SAT equals the direct
+    windowed sum: the same quantity two ways."""
+    a = make_np(40, 50, "int32", "u32", seed=11)
+    b = oracle.sat(a)
+    box = oracle.box_filter(a, 2, 3)
+    for (i, j) in [(0, 0), (39, 49), (10, 3), (2, 47), (20, 25)]:
+        r0, r1, c0, c1 = max(0, i - 2), min(39, i + 2), max(0, j - 3), min(49, j + 3)
+        assert np.uint32(oracle.rect_sum(b, r0, c0, r1, c1)) == box.view(np.uint32)[i, j]
