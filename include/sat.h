@@ -54,7 +54,8 @@ extern "C" {
 
 #define SAT_ABI_VERSION 1
 
-typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1, SAT_FLOAT64 = 2 } sat_dtype;
+typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1, SAT_FLOAT64 = 2,
+               SAT_UINT8 = 3 /* input only: sat_compute_widening, sat_box_filter */ } sat_dtype;
 
 /* Variants (Table I / Secs. IV-VII):
  *   SAT_2R2W        column-wise prefix pass then row-wise prefix pass, each a
@@ -120,6 +121,43 @@ int sat_compute_ex(const void *in, void *out, int64_t rows, int64_t cols,
 int sat_compute_batched(const void *in, void *out, int64_t batch, int64_t rows,
                         int64_t cols, int dtype, int variant, const sat_options *opt,
                         void *stream);
+
+/* Widening 1R1W: in holds in_dtype elements, out gets
+ * the SAT in `dtype`, the input widened on load inside the kernel (no extra
+ * pass).  Pairs: (SAT_UINT8 -> SAT_INT32) = the classic integral image of
+ * 8-bit pixels, exact in uint32 arithmetic (1 + 4 bytes per pixel moved);
+ * (SAT_FLOAT32 -> SAT_FLOAT64) = a float integral image in the paper's
+ * precision (4 + 8 bytes); same-type pairs behave as sat_compute_batched with
+ * SAT_1R1W.  batch x rows x cols, back to back.  in == out is invalid for a
+ * widening pair.  TMA path needs 16-B aligned pointers and cols % 16 == 0
+ * (uint8) or cols % 4 == 0; otherwise the generic path runs.  tile_rows: 64 or
+ * 128 for uint8 input, 16/32/64 for float32 -> float64. */
+int sat_compute_widening(const void *in, int in_dtype, void *out, int dtype,
+                         int64_t batch, int64_t rows, int64_t cols,
+                         const sat_options *opt, void *stream);
+
+/* Box filter (the SAT's use, "the sum of any rectangular area
+ * in O(1)"): out[b][i][j] = sum of in[b][k][l] over
+ * |k - i| <= rr, |l - j| <= rc, clipped to the image.  Computed as a widening
+ * 1R1W SAT into a library workspace (uint32 sums for SAT_UINT8/SAT_INT32
+ * input, float64 sums for SAT_FLOAT32/SAT_FLOAT64 input) followed by one
+ * kernel doing four SAT reads per output element.  out_dtype: SAT_INT32 for
+ * integer input (sums mod 2^32), SAT_FLOAT32 or SAT_FLOAT64 for float input.
+ * normalize != 0 divides by the clipped window's element count (box mean;
+ * float input only).  rr, rc >= 0; batch <= 65535.  Bytes moved per pixel:
+ * in + 2 x sum (SAT write + read) + out. */
+int sat_box_filter(const void *in, int in_dtype, void *out, int out_dtype,
+                   int64_t batch, int64_t rows, int64_t cols, int rr, int rc,
+                   int normalize, void *stream);
+
+/* Rectangle sums from a SAT: for q < nrects, with
+ * rects[5q .. 5q+4] = (image, r0, c0, r1, c1) (device int32, inclusive
+ * bounds), out[q] = sum of the rectangle = S[r1][c1] - S[r0-1][c1]
+ * - S[r1][c0-1] + S[r0-1][c0-1].  Bounds are clipped to the matrix; an empty
+ * rectangle or an image index outside [0, batch) gives 0.  sat, out: device,
+ * `dtype` elements (uint32 arithmetic for SAT_INT32). */
+int sat_rect_sums(const void *sat, int dtype, int64_t batch, int64_t rows, int64_t cols,
+                  const int32_t *rects, int64_t nrects, void *out, void *stream);
 
 /* Seeded 1R1W: the rows x cols matrix is a strip of a taller matrix and
  * carry_row[j] (device, cols entries, same dtype) is the column sum of

@@ -21,7 +21,7 @@ if not os.path.exists(_LIB_PATH):
 
 _lib = ctypes.CDLL(_LIB_PATH)
 
-SAT_INT32, SAT_FLOAT32, SAT_FLOAT64 = 0, 1, 2
+SAT_INT32, SAT_FLOAT32, SAT_FLOAT64, SAT_UINT8 = 0, 1, 2, 3
 VARIANTS = {"2r2w": 0, "2r1w": 1, "1r1w": 2, "1+rr1w": 3, "4r4w": 4, "4r1w": 5}
 SAT_OK = 0
 
@@ -46,6 +46,9 @@ _SIGS = {
     "sat_compute": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
     "sat_compute_ex": ([_P, _P, _I64, _I64, _I, _I, ctypes.POINTER(SatOptions), _P], _I),
     "sat_compute_batched": ([_P, _P, _I64, _I64, _I64, _I, _I, ctypes.POINTER(SatOptions), _P], _I),
+    "sat_compute_widening": ([_P, _I, _P, _I, _I64, _I64, _I64, ctypes.POINTER(SatOptions), _P], _I),
+    "sat_box_filter": ([_P, _I, _P, _I, _I64, _I64, _I64, _I, _I, _I, _P], _I),
+    "sat_rect_sums": ([_P, _I, _I64, _I64, _I64, _P, _I64, _P, _P], _I),
     "sat_compute_seeded": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
     "sat_compute_seeded_satrow": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
     "sat_column_totals": ([_P, _P, _I64, _I64, _I, _P], _I),
@@ -94,6 +97,8 @@ def _dtype_code(t) -> int:
         return SAT_FLOAT32
     if t.dtype == torch.float64:
         return SAT_FLOAT64
+    if t.dtype == torch.uint8:
+        return SAT_UINT8
     raise TypeError(f"libsat supports int32, float32 and float64, got {t.dtype}")
 
 
@@ -159,6 +164,57 @@ def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: 
     _check(_lib.sat_compute_batched(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                     x.shape[2], _dtype_code(x), VARIANTS[variant],
                                     ctypes.byref(o), _stream(stream)))
+    return out
+
+
+def _as3(x):
+    return x if x.dim() == 3 else x.unsqueeze(0)
+
+
+def sat_widening(x, dtype, out=None, tile_rows: int = 0, force_generic: bool = False, stream=None):
+    """1R1W SAT of a uint8 (-> int32 sums) or float32 (-> float64 sums) CUDA
+    tensor, 2-D or (batch, rows, cols), widened on load (no extra pass)."""
+    import torch
+    x3 = _as3(x)
+    if out is None:
+        out = torch.empty(x.shape, dtype=dtype, device=x.device)
+    _check_dev(x, out)
+    o = options(0.25, tile_rows, force_generic)
+    _check(_lib.sat_compute_widening(x.data_ptr(), _dtype_code(x), out.data_ptr(), _dtype_code(out),
+                                     x3.shape[0], x3.shape[1], x3.shape[2], ctypes.byref(o),
+                                     _stream(stream)))
+    return out
+
+
+def box_filter(x, rr: int, rc: int, normalize: bool = False, out_dtype=None, out=None, stream=None):
+    """Box filter through a SAT: window (2rr+1) x (2rc+1),
+    clipped.  uint8/int32 input -> int32 sums; float32/float64 input -> float
+    (``out_dtype``, default the input's), SAT in float64."""
+    import torch
+    x3 = _as3(x)
+    if out is None:
+        if out_dtype is None:
+            out_dtype = torch.int32 if x.dtype in (torch.uint8, torch.int32) else x.dtype
+        out = torch.empty(x.shape, dtype=out_dtype, device=x.device)
+    _check_dev(x, out)
+    _check(_lib.sat_box_filter(x.data_ptr(), _dtype_code(x), out.data_ptr(), _dtype_code(out),
+                               x3.shape[0], x3.shape[1], x3.shape[2], int(rr), int(rc),
+                               int(bool(normalize)), _stream(stream)))
+    return out
+
+
+def rect_sums(sat_t, rects, out=None, stream=None):
+    """Rectangle sums from a SAT: ``rects`` (K, 5) int32 CUDA tensor of
+    (image, r0, c0, r1, c1), inclusive, clipped."""
+    import torch
+    s3 = _as3(sat_t)
+    rects = rects.to(torch.int32).contiguous()
+    if out is None:
+        out = torch.empty(rects.shape[0], dtype=sat_t.dtype, device=sat_t.device)
+    _check_dev(sat_t, rects, out)
+    _check(_lib.sat_rect_sums(sat_t.data_ptr(), _dtype_code(sat_t), s3.shape[0], s3.shape[1],
+                              s3.shape[2], rects.data_ptr(), rects.shape[0], out.data_ptr(),
+                              _stream(stream)))
     return out
 
 

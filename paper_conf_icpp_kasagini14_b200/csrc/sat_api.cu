@@ -23,6 +23,7 @@
 #include "sat_aux.cuh"
 #include "sat_band.cuh"
 #include "sat_paper.cuh"
+#include "sat_box.cuh"
 
 using namespace sat;
 
@@ -121,6 +122,7 @@ struct Workspace {
     unsigned long long next_base = 0;
     Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
     Buf tr;                   // 4R4W transposed copy
+    Buf box;                  // box filter: the SAT it reads
     Buf part;                 // column totals partials
     Buf seedrow;              // seeded mode: SAT row above the strip
     Buf shard;                // sharded default workspace
@@ -141,7 +143,12 @@ int get_ws(int dev, cudaStream_t st, Workspace*& ws) {
 // ------------------------------------------------------------------ helpers
 
 bool dtype_ok(int dtype) { return dtype == SAT_INT32 || dtype == SAT_FLOAT32 || dtype == SAT_FLOAT64; }
-size_t esize(int dtype) { return dtype == SAT_FLOAT64 ? 8 : 4; }
+size_t esize(int dtype) { return dtype == SAT_FLOAT64 ? 8 : dtype == SAT_UINT8 ? 1 : 4; }
+// widening input -> sum pairs of sat_compute_widening (besides same-type pairs)
+bool widen_ok(int in_dtype, int dtype) {
+    return in_dtype == dtype || (in_dtype == SAT_UINT8 && dtype == SAT_INT32) ||
+           (in_dtype == SAT_FLOAT32 && dtype == SAT_FLOAT64);
+}
 // Element type of a sat_dtype: uint32 (int32, wrapping), float, double.
 #define SAT_DISPATCH(dtype, T, ...)                                             \
     ((dtype) == SAT_INT32     ? [&] { using T = uint32_t; return __VA_ARGS__; }() \
@@ -149,9 +156,12 @@ size_t esize(int dtype) { return dtype == SAT_FLOAT64 ? 8 : 4; }
                               : [&] { using T = double; return __VA_ARGS__; }())
 
 int validate(const void* in, const void* out, int64_t batch, int64_t rows, int64_t cols,
-             int dtype, bool need_in = true) {
+             int dtype, bool need_in = true, int in_dtype = -1) {
+    if (in_dtype < 0) in_dtype = dtype;
     if (!dtype_ok(dtype))
         return fail(SAT_ERR_INVALID, "dtype must be SAT_INT32, SAT_FLOAT32 or SAT_FLOAT64");
+    if (!widen_ok(in_dtype, dtype))
+        return fail(SAT_ERR_INVALID, "input/sum dtype pair must be equal, UINT8->INT32 or FLOAT32->FLOAT64");
     if (rows < 0 || cols < 0 || batch < 0) return fail(SAT_ERR_INVALID, "negative size");
     if (rows > INT32_MAX || cols > INT32_MAX || batch > INT32_MAX)
         return fail(SAT_ERR_INVALID, "rows, cols and batch must each be < 2^31");
@@ -159,20 +169,25 @@ int validate(const void* in, const void* out, int64_t batch, int64_t rows, int64
     const double n = double(rows) * double(cols) * double(batch);
     if (n * double(esize(dtype)) > 9.0e18) return fail(SAT_ERR_INVALID, "matrix byte size overflows");
     if ((need_in && !in) || !out) return fail(SAT_ERR_INVALID, "null pointer with nonzero size");
+    if (need_in && in_dtype != dtype && in == out)
+        return fail(SAT_ERR_INVALID, "a widening SAT cannot run in place");
     if (need_in && in != out) {
         const uintptr_t a0 = reinterpret_cast<uintptr_t>(in), b0 = reinterpret_cast<uintptr_t>(out);
-        const uintptr_t len = uintptr_t(rows) * uintptr_t(cols) * uintptr_t(batch) * 4u;
-        if (a0 < b0 + len && b0 < a0 + len)
+        const uintptr_t n_el = uintptr_t(rows) * uintptr_t(cols) * uintptr_t(batch);
+        const uintptr_t la = n_el * esize(in_dtype), lb = n_el * esize(dtype);
+        if (a0 < b0 + lb && b0 < a0 + la)
             return fail(SAT_ERR_INVALID, "in and out partially overlap");
     }
-    const uintptr_t am = esize(dtype) - 1;
-    if ((reinterpret_cast<uintptr_t>(out) & am) || (need_in && (reinterpret_cast<uintptr_t>(in) & am)))
+    const uintptr_t am = esize(dtype) - 1, ai = esize(in_dtype) - 1;
+    if ((reinterpret_cast<uintptr_t>(out) & am) || (need_in && (reinterpret_cast<uintptr_t>(in) & ai)))
         return fail(SAT_ERR_INVALID, "pointers must be aligned to the element size");
     return SAT_OK;
 }
 
-bool tma_ok(const void* in, const void* out, int64_t cols) {
-    return (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) &&
+bool tma_ok(const void* in, const void* out, int64_t cols, int in_dtype = -1) {
+    // 16-B aligned rows for the TMA box and the 4-per-lane vector stores
+    const int64_t q = in_dtype == SAT_UINT8 ? 16 : 4;
+    return (cols % q == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) &&
            ((reinterpret_cast<uintptr_t>(out) & 15) == 0);
 }
 
@@ -185,6 +200,7 @@ int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_
     cuuint32_t es[3] = {1, 1, 1};
     CUresult r = g_encode(m, dtype == SAT_INT32     ? CU_TENSOR_MAP_DATA_TYPE_UINT32
                              : dtype == SAT_FLOAT32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                             : dtype == SAT_UINT8   ? CU_TENSOR_MAP_DATA_TYPE_UINT8
                                                     : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
                           3, const_cast<void*>(base), dims, strides, box, es,
                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -223,12 +239,12 @@ int ctas_per_sm(int dtype, int th, bool big) {
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int CL = 1, int LBW = 0>
+          int CL = 1, int LBW = 0, typename TI = T>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                   const DevInfo& di, cudaStream_t st, int& grid_out) {
     (void)to;
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB, LBW>;
-    const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL>::total;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB, LBW, TI>;
+    const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL, TI>::total;
     const int threads = (W + NCW + 1) * 32;
     static int configured = 0;   // per instantiation (per process; devices share the attribute)
     if (!configured) {
@@ -334,6 +350,24 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
     }
 }
 
+// Widening 1R1W: uint8 -> uint32 and float32 -> float64.
+template <typename T, typename TI, bool TMA>
+int launch_band_widen(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
+                      const DevInfo& di, cudaStream_t st, int& grid) {
+    if constexpr (sizeof(TI) == 1) {
+        if (th == 128) return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, 0, TI>(p, ti, to, di, st, grid);
+        if (th == 64) return launch_band_t<T, 8, 8, 6, 4, 1, 4, 1, MODE_SAT, TMA, 2, 1, 0, TI>(p, ti, to, di, st, grid);
+        return fail(SAT_ERR_INVALID, "uint8 input: tile_rows must be 64 or 128");
+    } else {
+        switch (th) {
+            case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE_SAT, TMA, kCfgD16.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
+            case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE_SAT, TMA, kCfgD32.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE_SAT, TMA, kCfgD64.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
+        }
+        return fail(SAT_ERR_INVALID, "float32 -> float64: tile_rows must be 16, 32 or 64");
+    }
+}
+
 template <typename T, int MODE>
 int launch_band_m(bool tma, int th, const BandParams& p, const CUtensorMap& ti,
                   const CUtensorMap& to, const DevInfo& di, cudaStream_t st, int& grid) {
@@ -384,6 +418,7 @@ struct Job {
     void* out;
     int64_t batch, rows, cols;
     int dtype;
+    int in_dtype;     // == dtype, or a narrower input widened on load (1R1W only)
     int th;
     bool tma;
     int jitter;
@@ -470,10 +505,18 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     std::memset(&ti, 0, sizeof(ti));
     std::memset(&to, 0, sizeof(to));
     if (j.tma) {
-        SAT_TRY(make_tmap(&ti, in, j.dtype, j.batch, j.rows, j.cols, j.th));
+        SAT_TRY(make_tmap(&ti, in, j.in_dtype, j.batch, j.rows, j.cols, j.th));
     }
     int grid = 0;
-    int s = SAT_DISPATCH(j.dtype, T, launch_band_d<T>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid));
+    int s;
+    if (j.in_dtype == SAT_UINT8)
+        s = j.tma ? launch_band_widen<uint32_t, uint8_t, true>(j.th, p, ti, to, *j.di, j.st, grid)
+                  : launch_band_widen<uint32_t, uint8_t, false>(j.th, p, ti, to, *j.di, j.st, grid);
+    else if (j.in_dtype != j.dtype)
+        s = j.tma ? launch_band_widen<double, float, true>(j.th, p, ti, to, *j.di, j.st, grid)
+                  : launch_band_widen<double, float, false>(j.th, p, ti, to, *j.di, j.st, grid);
+    else
+        s = SAT_DISPATCH(j.dtype, T, launch_band_d<T>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid));
     if (s != SAT_OK) return s;
     // every persistent ticket taker (a CTA, or a cluster) makes exactly one
     // failing fetch, so the counter ends at base + units + takers
@@ -629,10 +672,13 @@ int run_4r1w_t(const Job& j) {
 // ------------------------------------------------------------------ core driver
 int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
                  int dtype, int variant, const sat_options* opt, const void* seed,
-                 int seed_kind, cudaStream_t st) {
+                 int seed_kind, cudaStream_t st, int in_dtype = -1) {
     t_launches = 0;
-    SAT_TRY(validate(in, out, batch, rows, cols, dtype));
+    if (in_dtype < 0) in_dtype = dtype;
+    SAT_TRY(validate(in, out, batch, rows, cols, dtype, true, in_dtype));
     if (variant < SAT_2R2W || variant > SAT_4R1W) return fail(SAT_ERR_INVALID, "bad variant");
+    if (in_dtype != dtype && (variant != SAT_1R1W || seed))
+        return fail(SAT_ERR_UNSUPPORTED, "widening input: unseeded 1R1W only");
     sat_options o;
     sat_options_init(&o);
     if (opt) o = *opt;
@@ -648,8 +694,10 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     SAT_TRY(get_ws(dev, st, ws));
     Job j;
     j.in = in; j.out = out; j.batch = batch; j.rows = rows; j.cols = cols; j.dtype = dtype;
+    j.in_dtype = in_dtype;
     j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
-    j.tma = !o.force_generic && tma_ok(in, out, cols);
+    if (in_dtype == SAT_UINT8 && !o.tile_rows) j.th = j.th == 128 ? 128 : 64;
+    j.tma = !o.force_generic && tma_ok(in, out, cols, in_dtype);
     j.jitter = o.jitter;
     j.di = &di;
     j.ws = ws;
@@ -786,6 +834,85 @@ int sat_compute_batched(const void* in, void* out, int64_t batch, int64_t rows, 
                         int dtype, int variant, const sat_options* opt, void* stream) {
     return compute_core(in, out, batch, rows, cols, dtype, variant, opt, nullptr, SEED_NONE,
                         static_cast<cudaStream_t>(stream));
+}
+
+int sat_compute_widening(const void* in, int in_dtype, void* out, int dtype, int64_t batch,
+                         int64_t rows, int64_t cols, const sat_options* opt, void* stream) {
+    if (in_dtype != SAT_UINT8 && !dtype_ok(in_dtype)) return fail(SAT_ERR_INVALID, "bad input dtype");
+    return compute_core(in, out, batch, rows, cols, dtype, SAT_1R1W, opt, nullptr, SEED_NONE,
+                        static_cast<cudaStream_t>(stream), in_dtype);
+}
+
+int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64_t batch,
+                   int64_t rows, int64_t cols, int rr, int rc, int normalize, void* stream) {
+    t_launches = 0;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    // the SAT's type: uint32 sums for integer pixels, float64 for float inputs
+    const int sdt = (in_dtype == SAT_UINT8 || in_dtype == SAT_INT32) ? SAT_INT32
+                    : (in_dtype == SAT_FLOAT32 || in_dtype == SAT_FLOAT64) ? SAT_FLOAT64 : -1;
+    if (sdt < 0) return fail(SAT_ERR_INVALID, "box filter input must be UINT8, INT32, FLOAT32 or FLOAT64");
+    if (sdt == SAT_INT32 ? out_dtype != SAT_INT32 : (out_dtype != SAT_FLOAT32 && out_dtype != SAT_FLOAT64))
+        return fail(SAT_ERR_INVALID, "box filter output: INT32 for integer input, FLOAT32/64 for float input");
+    if (rr < 0 || rc < 0) return fail(SAT_ERR_INVALID, "negative radius");
+    if (normalize && sdt == SAT_INT32) return fail(SAT_ERR_INVALID, "normalize needs float input");
+    if (batch > 65535) return fail(SAT_ERR_UNSUPPORTED, "box filter: batch must be <= 65535");
+    SAT_TRY(validate(nullptr, out, batch, rows, cols, out_dtype, false));
+    if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
+    if (!in) return fail(SAT_ERR_INVALID, "null pointer with nonzero size");
+    if (reinterpret_cast<uintptr_t>(in) & (esize(in_dtype) - 1))
+        return fail(SAT_ERR_INVALID, "pointers must be aligned to the element size");
+    {   // the SAT lives in a workspace, so out may alias in exactly, not partially
+        const uintptr_t a0 = reinterpret_cast<uintptr_t>(in), b0 = reinterpret_cast<uintptr_t>(out);
+        const uintptr_t n_el = uintptr_t(rows) * uintptr_t(cols) * uintptr_t(batch);
+        const uintptr_t la = n_el * esize(in_dtype), lb = n_el * esize(out_dtype);
+        if (a0 != b0 && a0 < b0 + lb && b0 < a0 + la)
+            return fail(SAT_ERR_INVALID, "in and out partially overlap");
+        if (a0 == b0 && la != lb) return fail(SAT_ERR_INVALID, "in place needs equal element sizes");
+    }
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    Workspace* ws;
+    SAT_TRY(get_ws(dev, st, ws));
+    SAT_TRY(ensure(ws->box, size_t(batch) * rows * cols * esize(sdt), false));
+    // 1. the SAT (1R1W, widening uint8 -> uint32 and float32 -> float64 on load)
+    SAT_TRY(compute_core(in, ws->box.p, batch, rows, cols, sdt, SAT_1R1W, nullptr, nullptr, SEED_NONE,
+                         st, in_dtype));
+    int launches = t_launches;
+    // 2. four SAT reads per output element
+    const dim3 grid(unsigned((cols + 255) / 256), unsigned(std::min<int64_t>(rows, 65535)), unsigned(batch));
+    if (sdt == SAT_INT32)
+        sat_box_kernel<uint32_t, int32_t><<<grid, 256, 0, st>>>(static_cast<const uint32_t*>(ws->box.p),
+                                                                static_cast<int32_t*>(out), rows, cols, rr, rc, 0);
+    else if (out_dtype == SAT_FLOAT32)
+        sat_box_kernel<double, float><<<grid, 256, 0, st>>>(static_cast<const double*>(ws->box.p),
+                                                           static_cast<float*>(out), rows, cols, rr, rc, normalize);
+    else
+        sat_box_kernel<double, double><<<grid, 256, 0, st>>>(static_cast<const double*>(ws->box.p),
+                                                            static_cast<double*>(out), rows, cols, rr, rc, normalize);
+    CUDA_TRY(cudaGetLastError());
+    t_launches = launches + 1;
+    return SAT_OK;
+}
+
+int sat_rect_sums(const void* sat, int dtype, int64_t batch, int64_t rows, int64_t cols,
+                  const int32_t* rects, int64_t nrects, void* out, void* stream) {
+    t_launches = 0;
+    if (!dtype_ok(dtype)) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (nrects < 0 || batch < 0 || rows < 0 || cols < 0) return fail(SAT_ERR_INVALID, "negative size");
+    if (nrects == 0) return SAT_OK;
+    if (!sat || !rects || !out) return fail(SAT_ERR_INVALID, "null pointer");
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    const unsigned blocks = unsigned(std::min<int64_t>((nrects + 255) / 256, 16LL * di.sms));
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    SAT_DISPATCH(dtype, T, (sat_rect_kernel<T><<<blocks, 256, 0, st>>>(static_cast<const T*>(sat), batch, rows,
+                                                                      cols, rects, nrects, static_cast<T*>(out)),
+                            0));
+    CUDA_TRY(cudaGetLastError());
+    t_launches = 1;
+    return SAT_OK;
 }
 
 int sat_compute_seeded(const void* in, void* out, int64_t rows, int64_t cols, int dtype,

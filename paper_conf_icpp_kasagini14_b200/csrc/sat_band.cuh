@@ -77,14 +77,31 @@ __device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
     a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
 }
 
+// Input element -> arithmetic element for 4 consecutive columns in shared
+// memory: the same type, or a narrower input widened on load (uint8 pixels ->
+// uint32 sums, the classic integral image; float32 -> float64 sums, an
+// accurate float integral image).  DESIGN.md Sec. 4.8.
+template <typename T, typename TI>
+__device__ __forceinline__ V4<T> lds4_in(const TI* p) {
+    if constexpr (std::is_same<T, TI>::value) {
+        return lds4<T>(p);
+    } else if constexpr (sizeof(TI) == 1) {
+        const uint32_t w = *reinterpret_cast<const uint32_t*>(p);
+        return V4<T>{T(w & 255u), T((w >> 8) & 255u), T((w >> 16) & 255u), T(w >> 24)};
+    } else {
+        const V4<TI> a = lds4<TI>(p);
+        return V4<T>{T(a.x), T(a.y), T(a.z), T(a.w)};
+    }
+}
+
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int DT, int SUB, int CL = 1>
+template <typename T, int R, int W, int S, int DT, int SUB, int CL = 1, typename TI = T>
 struct BandSmem {
     static constexpr int TH = R * W;
     static constexpr int XS = DT;                    // carry slots: one per parked chunk
     static constexpr size_t tile_elems = size_t(TH) * TW;            // one 128-column chunk
     static constexpr size_t slot_elems = tile_elems * SUB;           // one ring slot
-    static constexpr size_t tiles = S * slot_elems * sizeof(T);
+    static constexpr size_t tiles = S * slot_elems * sizeof(TI);     // the ring holds input elements
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
     // clusters: incoming partial aggregate (chain) and cluster top row per carry slot
     static constexpr size_t cbuf = CL > 1 ? size_t(2) * XS * TW * sizeof(T) : 0;
@@ -271,7 +288,7 @@ struct TmemCols {
 };
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int CL, int MODE, bool TMA, int MINB,
-          int LBW_ = 0>
+          int LBW_ = 0, typename TI = T>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -279,8 +296,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int TH = R * W;
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
-    constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(T);
-    using SM = BandSmem<T, R, W, S, DT, SUB, CL>;
+    constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(TI);
+    using SM = BandSmem<T, R, W, S, DT, SUB, CL, TI>;
+    static_assert(std::is_same<T, TI>::value || (MODE == MODE_SAT && CL == 1), "widening input: 1R1W only");
     static_assert(CL == 1 || (MODE == MODE_SAT && NS == 1 && sizeof(T) == 4), "clusters: 1R1W band kernel only");
     constexpr int NWE = Words<T>::N;             // 32-bit words per element
     using TC = TmemCols<R, W, DT, NWE>;
@@ -293,7 +311,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     static_assert(NCW / NS <= XS, "more control groups than carry slots");
 
     extern __shared__ __align__(1024) uint8_t smem[];
-    T* tiles = reinterpret_cast<T*>(smem);
+    TI* tiles = reinterpret_cast<TI*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
     T* cagg = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);         // [XS][TW] own aggregate (CL > 1)
     T* ctop = cagg + size_t(XS) * TW;                                     // [XS][TW] top from rank 0 (CL > 1)
@@ -444,7 +462,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     L[r] = from_words<T>(w);
                 }
             }
-            const T* gin = reinterpret_cast<const T*>(p.in) + int64_t(img) * img_elems;
+            const TI* gin = reinterpret_cast<const TI*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
             // this warp's TMEM lanes (32*(warp%4) ..) and column range
             const uint32_t tm_warp = tmem_base + ((uint32_t(32 * (warp & 3))) << 16)
@@ -481,10 +499,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     if (k % SUB == 0) mbar_wait(&full[s], (q / S) & 1);
                     if (traced && warp == 0 && lane == 0)
                         p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
-                    const T* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
-                                 + size_t(rbase) * TW + 4 * lane;
+                    const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
+                                  + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
-                    for (int r = 0; r < R; ++r) v[r] = lds4<T>(t + r * TW);
+                    for (int r = 0; r < R; ++r) v[r] = lds4_in<T, TI>(t + r * TW);
                     if (k % SUB == SUB - 1 || k == nch - 1) {
                         // release the slot to the next TMA write only once the
                         // generic-proxy reads have landed in registers (the
@@ -509,7 +527,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         T e[4];
 #pragma unroll
                         for (int i = 0; i < 4; ++i)
-                            e[i] = (row < p.rows && c + i < p.cols) ? gin[row * p.cols + c + i] : T(0);
+                            e[i] = (row < p.rows && c + i < p.cols) ? T(gin[row * p.cols + c + i]) : T(0);
                         v[r] = V4<T>{e[0], e[1], e[2], e[3]};
                     }
                 }

@@ -1,0 +1,80 @@
+// sat_box.cuh -- consumers of a SAT: the reason the
+// paper computes SATs at all -- "the sum of any rectangular area can be
+// computed in O(1) time" from four SAT reads (Sec. I).
+//
+//  * sat_box_kernel: box filter, out[i][j] = sum of a over rows |k - i| <= rr
+//    and columns |l - j| <= rc, clipped to the matrix, by inclusion-exclusion
+//    over the SAT S:  S[i2][j2] - S[i1-1][j2] - S[i2][j1-1] + S[i1-1][j1-1]
+//    (terms with index -1 are 0), optionally divided by the clipped window's
+//    element count (box mean).  One thread per output element; a warp reads
+//    two SAT rows at two column offsets, all coalesced; the 2rr+1 rows a
+//    block row shares stay in L2.
+//  * sat_rect_kernel: K arbitrary rectangle queries (image, r0, c0, r1, c1),
+//    inclusive and clipped to the matrix, one thread each.
+#pragma once
+#include "sat_common.h"
+
+namespace sat {
+
+template <typename T>
+__device__ __forceinline__ T rect_from_sat(const T* S, int64_t cols, int64_t i1, int64_t j1, int64_t i2,
+                                           int64_t j2) {
+    T v = S[i2 * cols + j2];
+    if (i1 > 0) v -= S[(i1 - 1) * cols + j2];
+    if (j1 > 0) v -= S[i2 * cols + j1 - 1];
+    if (i1 > 0 && j1 > 0) v += S[(i1 - 1) * cols + j1 - 1];
+    return v;
+}
+
+template <typename TO, typename T>
+__device__ __forceinline__ TO box_out(T v) {
+    if constexpr (std::is_same<T, uint32_t>::value) return TO(int32_t(v));   // int32 bits, mod 2^32
+    else return TO(v);
+}
+
+// grid: (ceil(cols / 256), min(rows, 65535), batch); block 256
+template <typename T, typename TO>
+__global__ void __launch_bounds__(256) sat_box_kernel(const T* __restrict__ S, TO* __restrict__ out,
+                                                      int64_t rows, int64_t cols, int rr, int rc,
+                                                      int normalize) {
+    const int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (j >= cols) return;
+    const int64_t img = blockIdx.z;
+    const T* Si = S + img * rows * cols;
+    TO* Oi = out + img * rows * cols;
+    const int64_t j1 = j - rc > 0 ? j - rc : 0;
+    const int64_t j2 = j + rc < cols - 1 ? j + rc : cols - 1;
+    for (int64_t i = blockIdx.y; i < rows; i += gridDim.y) {
+        const int64_t i1 = i - rr > 0 ? i - rr : 0;
+        const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
+        T v = rect_from_sat(Si, cols, i1, j1, i2, j2);
+        if constexpr (!std::is_same<T, uint32_t>::value) {
+            if (normalize) v = v / T((i2 - i1 + 1) * (j2 - j1 + 1));
+        }
+        Oi[i * cols + j] = box_out<TO>(v);
+    }
+}
+
+// rects: [K][5] int32 = (image, r0, c0, r1, c1), inclusive; clipped to the
+// matrix; an empty (clipped) rectangle or a bad image index sums to 0.
+template <typename T>
+__global__ void __launch_bounds__(256) sat_rect_kernel(const T* __restrict__ S, int64_t batch, int64_t rows,
+                                                       int64_t cols, const int32_t* __restrict__ rects,
+                                                       int64_t K, T* __restrict__ out) {
+    for (int64_t q = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; q < K;
+         q += int64_t(gridDim.x) * blockDim.x) {
+        const int32_t* r = rects + q * 5;
+        const int64_t b = r[0];
+        int64_t i1 = r[1], j1 = r[2], i2 = r[3], j2 = r[4];
+        if (i1 < 0) i1 = 0;
+        if (j1 < 0) j1 = 0;
+        if (i2 > rows - 1) i2 = rows - 1;
+        if (j2 > cols - 1) j2 = cols - 1;
+        T v = T(0);
+        if (b >= 0 && b < batch && i1 <= i2 && j1 <= j2)
+            v = rect_from_sat(S + b * rows * cols, cols, i1, j1, i2, j2);
+        out[q] = v;
+    }
+}
+
+}  // namespace sat

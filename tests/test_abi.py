@@ -72,3 +72,36 @@ def test_python_wrapper_rejects_cpu_tensors():
         libsat.sat(torch.zeros(4, 4, dtype=torch.int32))
     with pytest.raises(ValueError):
         libsat.sat(torch.zeros(4, 4, 4, dtype=torch.int32))
+
+
+def test_validation_new_entry_points_without_gpu():
+    """float64 / widening / box filter / rectangle sums: argument checks that
+    return before any CUDA call."""
+    o = libsat.options()
+    # widening pairs: only equal, UINT8->INT32, FLOAT32->FLOAT64
+    assert L.sat_compute_widening(4096, 3, 1 << 20, 1, 1, 4, 4, ctypes.byref(o), None) == -1
+    assert L.sat_compute_widening(4096, 2, 1 << 20, 1, 1, 4, 4, ctypes.byref(o), None) == -1
+    assert b"pair" in L.sat_last_error()
+    # widening cannot run in place
+    assert L.sat_compute_widening(4096, 1, 4096, 2, 1, 4, 4, ctypes.byref(o), None) == -1
+    assert b"in place" in L.sat_last_error()
+    # float64 alignment and overlap use 8-byte elements
+    assert L.sat_compute(4100, 1 << 20, 4, 4, 2, 2, None) == -1
+    assert L.sat_compute(4096, 4096 + 64, 4, 4, 2, 2, None) == -1      # 128-B matrices overlap
+    assert b"overlap" in L.sat_last_error()
+    # box filter: dtype rules, radii, normalize
+    assert L.sat_box_filter(4096, 3, 1 << 20, 1, 1, 4, 4, 1, 1, 0, None) == -1   # uint8 -> float
+    assert L.sat_box_filter(4096, 1, 1 << 20, 0, 1, 4, 4, 1, 1, 0, None) == -1   # float -> int
+    assert L.sat_box_filter(4096, 0, 1 << 20, 0, 1, 4, 4, -1, 1, 0, None) == -1  # radius
+    assert L.sat_box_filter(4096, 0, 1 << 20, 0, 1, 4, 4, 1, 1, 1, None) == -1   # normalize int
+    assert b"normalize" in L.sat_last_error()
+    assert L.sat_box_filter(None, 3, None, 0, 1, 0, 4, 1, 1, 0, None) == 0       # empty
+    # rectangle sums
+    assert L.sat_rect_sums(None, 0, 1, 4, 4, 64, 3, 128, None) == -1
+    assert L.sat_rect_sums(4096, 5, 1, 4, 4, 64, 3, 128, None) == -1
+    assert L.sat_rect_sums(None, 0, 1, 4, 4, None, 0, None, None) == 0
+    # the 4R4W / 4R1W variant codes are accepted by validation (bad options still fail)
+    o = libsat.options(tile_rows=40)
+    assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 5, ctypes.byref(o), None) == -1
+    assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 6, ctypes.byref(o), None) == -1
+    assert b"variant" in L.sat_last_error()

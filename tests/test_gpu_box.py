@@ -1,0 +1,160 @@
+"""GPU parity for the SAT's consumers and widening inputs:
+widening 1R1W (uint8 -> int32 sums, float32 -> float64 sums), the box filter
+and rectangle-sum queries, through the C ABI, against the
+oracle's plain definitions (oracle.sat, oracle.box_filter, oracle.rect_sum).
+
+Integer paths are exact (mod 2^32).  Float32 inputs are dyadic (k 2^-24), so
+their float64 SATs and box sums are exact and the float32 box output is the
+correctly rounded exact value: compared bit for bit.  Full-mantissa float64
+box sums get the SAT-error bound (R17) through four corners.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from sat_inputs import make_np
+
+pytestmark = pytest.mark.gpu
+U = 2.0 ** -53
+
+
+@pytest.fixture(scope="module")
+def libsat():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_icpp_kasagini14_b200 as m
+    return m
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def u8img(n, m, seed, batch=None):
+    return make_np(n, m, "int32", "u8", seed=seed, batch=batch).astype(np.uint8)
+
+
+# ------------------------------------------------------------------ widening 1R1W
+@pytest.mark.parametrize("shape", [(1, 1), (3, 5), (64, 256), (129, 160), (1080, 1920), (333, 1000),
+                                   (2049, 784)], ids=lambda s: f"{s[0]}x{s[1]}")
+@pytest.mark.parametrize("generic", [False, True])
+def test_widening_uint8(libsat, shape, generic):
+    a = u8img(*shape, seed=shape[0])
+    y = libsat.sat_widening(dev(a), torch.int32, force_generic=generic)
+    assert np.array_equal(y.cpu().numpy(), oracle.sat(a.astype(np.int32)))
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (3, 5), (64, 256), (129, 160), (1080, 1920), (2049, 784)],
+                         ids=lambda s: f"{s[0]}x{s[1]}")
+def test_widening_float32_to_float64(libsat, shape):
+    a = make_np(*shape, "float32", "unit", seed=shape[1])
+    y = libsat.sat_widening(dev(a), torch.float64)
+    assert np.array_equal(y.cpu().numpy(), oracle.sat(a))        # exact: dyadic sums in double
+
+
+def test_widening_batched_tiles_segments(libsat, monkeypatch):
+    a = u8img(1080, 1920, seed=4, batch=5)
+    for th in (64, 128):
+        y = libsat.sat_widening(dev(a), torch.int32, tile_rows=th).cpu().numpy()
+        for b in range(5):
+            assert np.array_equal(y[b], oracle.sat(a[b].astype(np.int32)))
+    f = make_np(700, 1300, "float32", "unit", seed=3)
+    for th in (16, 32, 64):
+        assert np.array_equal(libsat.sat_widening(dev(f), torch.float64, tile_rows=th).cpu().numpy(),
+                              oracle.sat(f))
+    monkeypatch.setenv("SAT_SEG", "3")
+    g = u8img(64 * 40 + 7, 2048, seed=5)
+    assert np.array_equal(libsat.sat_widening(dev(g), torch.int32, tile_rows=64).cpu().numpy(),
+                          oracle.sat(g.astype(np.int32)))
+
+
+# ------------------------------------------------------------------ box filter
+@pytest.mark.parametrize("rr,rc", [(0, 0), (1, 1), (4, 4), (2, 7), (40, 3), (2000, 2000)])
+def test_box_uint8_images(libsat, rr, rc):
+    a = u8img(270, 480, seed=rr * 31 + rc, batch=3)
+    y = libsat.box_filter(dev(a), rr, rc).cpu().numpy()
+    assert y.dtype == np.int32
+    for b in range(3):
+        assert np.array_equal(y[b], oracle.box_filter(a[b].astype(np.int32), rr, rc))
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (5, 3), (127, 129), (1080, 1920)], ids=lambda s: f"{s[0]}x{s[1]}")
+def test_box_int32_wrapping(libsat, shape):
+    a = make_np(*shape, "int32", "u32", seed=7)
+    assert np.array_equal(libsat.box_filter(dev(a), 3, 5).cpu().numpy(), oracle.box_filter(a, 3, 5))
+
+
+@pytest.mark.parametrize("normalize", [False, True])
+def test_box_float32_exact(libsat, normalize):
+    """Dyadic float32 input: float64 SAT and box sums are exact, the float32
+    output is the correctly rounded oracle value, bit for bit."""
+    a = make_np(540, 960, "float32", "unit", seed=11, batch=2)
+    for out_dtype in (torch.float32, torch.float64):
+        y = libsat.box_filter(dev(a), 4, 6, normalize=normalize, out_dtype=out_dtype).cpu().numpy()
+        for b in range(2):
+            ref = oracle.box_filter(a[b], 4, 6, normalize=normalize)
+            assert np.array_equal(y[b], ref.astype(y.dtype))
+
+
+def test_box_float64_full_mantissa(libsat):
+    n, m, rr, rc = 300, 500, 3, 9
+    a = make_np(n, m, "float64", "unit53", seed=2)
+    y = libsat.box_filter(dev(a), rr, rc).cpu().numpy()
+    ref = oracle.box_filter(a, rr, rc)
+    S = oracle.sat(a)
+    i = np.arange(n)[:, None]
+    j = np.arange(m)[None, :]
+    i1, i2 = np.maximum(0, i - rr), np.minimum(n - 1, i + rr)
+    j1, j2 = np.maximum(0, j - rc), np.minimum(m - 1, j + rc)
+
+    def corner(r, c):
+        ok = (r >= 0) & (c >= 0)
+        rr_, cc_ = np.clip(r, 0, None), np.clip(c, 0, None)
+        return np.where(ok, S[rr_, cc_] * (rr_ + cc_ + 128), 0.0), np.where(ok, S[rr_, cc_], 0.0)
+    tot_e = np.zeros((n, m))
+    tot_m = np.zeros((n, m))
+    for r, c in [(i2, j2), (i1 - 1, j2), (i2, j1 - 1), (i1 - 1, j1 - 1)]:
+        e, mag = corner(r + 0 * c, c + 0 * r)
+        tot_e += e
+        tot_m += mag
+    bound = 2 * U * tot_e + 4 * U * tot_m + 2 * U * np.abs(ref)
+    assert (np.abs(y - ref) <= bound).all()
+
+
+def test_box_inplace_and_generic(libsat):
+    a = make_np(333, 1001, "int32", "u8", seed=9)           # cols % 4 != 0: generic path
+    x = dev(a)
+    ref = oracle.box_filter(a, 2, 2)
+    y = libsat.box_filter(x, 2, 2, out=x)
+    assert y.data_ptr() == x.data_ptr()
+    assert np.array_equal(x.cpu().numpy(), ref)
+    b = u8img(333, 1001, seed=9)
+    assert np.array_equal(libsat.box_filter(dev(b), 2, 2).cpu().numpy(), oracle.box_filter(b.astype(np.int32), 2, 2))
+
+
+# ------------------------------------------------------------------ rectangle queries
+def test_rect_sums(libsat):
+    rng = np.random.default_rng(0)
+    batch, n, m = 3, 300, 400
+    a = make_np(n, m, "int32", "u32", seed=13, batch=batch)
+    sat = libsat.sat_batched(dev(a))
+    K = 5000
+    rects = np.stack([rng.integers(-1, batch + 1, K), rng.integers(-20, n + 20, K),
+                      rng.integers(-20, m + 20, K), rng.integers(-20, n + 20, K),
+                      rng.integers(-20, m + 20, K)], axis=1).astype(np.int32)
+    got = libsat.rect_sums(sat, dev(rects)).cpu().numpy()
+    refs = [oracle.sat(a[b]) for b in range(batch)]
+    for q in range(K):
+        b, r0, c0, r1, c1 = rects[q].tolist()
+        r0, c0, r1, c1 = max(r0, 0), max(c0, 0), min(r1, n - 1), min(c1, m - 1)
+        want = 0
+        if 0 <= b < batch and r0 <= r1 and c0 <= c1:
+            want = int(np.uint32(oracle.rect_sum(refs[b], r0, c0, r1, c1)).view(np.int32))
+        assert int(got[q]) == want, (q, rects[q])
+    # float64 SAT of dyadic input: exact rectangle sums equal the input block sums
+    f = make_np(200, 300, "float64", "unit", seed=14)
+    sf = libsat.sat(dev(f))
+    rq = np.array([[0, 10, 20, 150, 250], [0, 0, 0, 199, 299], [0, 5, 5, 5, 5]], dtype=np.int32)
+    gf = libsat.rect_sums(sf, dev(rq)).cpu().numpy()
+    for q, (_, r0, c0, r1, c1) in enumerate(rq.tolist()):
+        assert gf[q] == f[r0:r1 + 1, c0:c1 + 1].sum()
