@@ -880,7 +880,8 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
                          st, in_dtype));
     int launches = t_launches;
     // 2. four SAT reads per output element
-    const dim3 grid(unsigned((cols + 255) / 256), unsigned(std::min<int64_t>(rows, 65535)), unsigned(batch));
+    const dim3 grid(unsigned((cols + 255) / 256), unsigned(std::min<int64_t>((rows + BOX_RB - 1) / BOX_RB, 65535)),
+                    unsigned(batch));
     if (sdt == SAT_INT32)
         sat_box_kernel<uint32_t, int32_t><<<grid, 256, 0, st>>>(static_cast<const uint32_t*>(ws->box.p),
                                                                 static_cast<int32_t*>(out), rows, cols, rr, rc, 0);

@@ -32,7 +32,11 @@ __device__ __forceinline__ TO box_out(T v) {
     else return TO(v);
 }
 
-// grid: (ceil(cols / 256), min(rows, 65535), batch); block 256
+// grid: (ceil(cols / 256), min(ceil(rows / BOX_RB), 65535), batch); block 256.
+// A thread owns one column and BOX_RB consecutive rows per iteration and
+// issues all 4*BOX_RB SAT loads before any arithmetic (memory-level
+// parallelism: one row per thread left the kernel latency-bound).
+constexpr int BOX_RB = 8;
 template <typename T, typename TO>
 __global__ void __launch_bounds__(256) sat_box_kernel(const T* __restrict__ S, TO* __restrict__ out,
                                                       int64_t rows, int64_t cols, int rr, int rc,
@@ -44,14 +48,32 @@ __global__ void __launch_bounds__(256) sat_box_kernel(const T* __restrict__ S, T
     TO* Oi = out + img * rows * cols;
     const int64_t j1 = j - rc > 0 ? j - rc : 0;
     const int64_t j2 = j + rc < cols - 1 ? j + rc : cols - 1;
-    for (int64_t i = blockIdx.y; i < rows; i += gridDim.y) {
-        const int64_t i1 = i - rr > 0 ? i - rr : 0;
-        const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
-        T v = rect_from_sat(Si, cols, i1, j1, i2, j2);
-        if constexpr (!std::is_same<T, uint32_t>::value) {
-            if (normalize) v = v / T((i2 - i1 + 1) * (j2 - j1 + 1));
+    for (int64_t i0 = int64_t(blockIdx.y) * BOX_RB; i0 < rows; i0 += int64_t(gridDim.y) * BOX_RB) {
+        T a[BOX_RB], b[BOX_RB], c[BOX_RB], d[BOX_RB];
+#pragma unroll
+        for (int k = 0; k < BOX_RB; ++k) {
+            const int64_t i = i0 + k < rows ? i0 + k : rows - 1;
+            const int64_t i1 = i - rr > 0 ? i - rr : 0;
+            const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
+            a[k] = Si[i2 * cols + j2];
+            b[k] = i1 > 0 ? Si[(i1 - 1) * cols + j2] : T(0);
+            c[k] = j1 > 0 ? Si[i2 * cols + j1 - 1] : T(0);
+            d[k] = (i1 > 0 && j1 > 0) ? Si[(i1 - 1) * cols + j1 - 1] : T(0);
         }
-        Oi[i * cols + j] = box_out<TO>(v);
+#pragma unroll
+        for (int k = 0; k < BOX_RB; ++k) {
+            const int64_t i = i0 + k;
+            if (i >= rows) break;
+            T v = ((a[k] - b[k]) - c[k]) + d[k];
+            if constexpr (!std::is_same<T, uint32_t>::value) {
+                if (normalize) {
+                    const int64_t i1 = i - rr > 0 ? i - rr : 0;
+                    const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
+                    v = v / T((i2 - i1 + 1) * (j2 - j1 + 1));
+                }
+            }
+            Oi[i * cols + j] = box_out<TO>(v);
+        }
     }
 }
 
