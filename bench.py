@@ -230,6 +230,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-sample-rows", type=int, default=None)
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
+                    help="N>1 row strips: NCCL all-gather, or the fused peer exchange (IPC mailboxes)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -286,7 +288,18 @@ def main():
 
     launches = [0]
 
-    if sharded:
+    if sharded and args.exchange == "fused":
+        from paper_conf_icpp_kasagini14_b200.dist import make_peer_exchange
+        xchg, _ = make_peer_exchange(cols, tdt, device=dev)
+
+        def step(ev=None):
+            if ev:
+                ev[0].record(stream)
+            xchg.sat(x, out=y)
+            if ev:
+                ev[1].record(stream)
+            launches[0] += libsat.last_launch_count()
+    elif sharded:
         P = world
         gathered = torch.empty(P * cols, dtype=tdt, device=dev)
         send = torch.empty(cols, dtype=tdt, device=dev)
@@ -420,7 +433,7 @@ def main():
             "data": "synthetic (splitmix64 counter hash: uniform 32-bit int / dyadic [0,1) float)",
             "config": {"workload": desc + (f" [{variant}]" if variant != "1r1w" else ""),
                        "rows": rows, "cols": cols, "batch": batch,
-                       "parallelism": (f"row-strips x{world}" if sharded else
+                       "parallelism": (f"row-strips x{world} ({args.exchange} exchange)" if sharded else
                                        (f"dp{world}" if world > 1 else "1 GPU")),
                        "l2": "inputs > L2, no flush" if my_elems * eb > 4 * 126e6 else
                              "inputs near L2 size: hot-L2 number",

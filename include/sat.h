@@ -171,6 +171,36 @@ int sat_compute_seeded(const void *in, void *out, int64_t rows, int64_t cols,
 int sat_compute_seeded_satrow(const void *in, void *out, int64_t rows, int64_t cols,
                               int dtype, const void *sat_row, void *stream);
 
+/* ---- Fused peer exchange ----
+ * The sharded mode without a collective call: rank p's column-totals kernel
+ * stores its totals straight into slot p of every higher rank's "mailbox"
+ * (peer memory over NVLink, e.g. IPC-mapped) and raises a flag there; rank
+ * p's SAT prologue waits for the flags of ranks < p, sums their slots in rank
+ * order (the exclusive scan) and acknowledges; then the seeded 1R1W runs.
+ * Mailboxes are double-buffered by call parity with acknowledgements, so
+ * consecutive calls need no barrier.  All ranks must make the same sequence of
+ * calls.  Results are bit-identical to sat_compute_sharded (int32).
+ *
+ * sat_exchange_mailbox_bytes: size of one rank's mailbox.
+ * sat_exchange_create: rank of nranks (<= 16); `mailbox` = this rank's own
+ *   mailbox (device, 256-B aligned, zeroed here); peers[q] = rank q's mailbox
+ *   as addressable from this rank's device (peers[rank] == mailbox).  The
+ *   caller owns the memory and keeps it alive until sat_exchange_destroy.
+ * sat_compute_sharded_fused: as sat_compute_sharded for this rank's strip. */
+size_t sat_exchange_mailbox_bytes(int64_t cols, int nranks, int dtype);
+int sat_exchange_create(void **exchange, int rank, int nranks, int64_t cols, int dtype,
+                        void *mailbox, void *const *peers);
+int sat_exchange_destroy(void *exchange);
+int sat_compute_sharded_fused(const void *in_strip, void *out_strip, int64_t strip_rows,
+                              void *exchange, void *stream);
+
+/* CUDA IPC helpers for the mailboxes of other processes: a 64-byte handle of
+ * a device allocation, and its mapping into this process (peer access over
+ * NVLink enabled lazily). */
+int sat_ipc_get_handle(const void *dev_ptr, void *handle64);
+int sat_ipc_open(const void *handle64, void **dev_ptr);
+int sat_ipc_close(void *dev_ptr);
+
 /* totals[j] = sum_i in[i][j] (device, cols entries).  Deterministic order. */
 int sat_column_totals(const void *in, void *totals, int64_t rows, int64_t cols,
                       int dtype, void *stream);

@@ -49,6 +49,14 @@ _SIGS = {
     "sat_compute_widening": ([_P, _I, _P, _I, _I64, _I64, _I64, ctypes.POINTER(SatOptions), _P], _I),
     "sat_box_filter": ([_P, _I, _P, _I, _I64, _I64, _I64, _I, _I, _I, _P], _I),
     "sat_rect_sums": ([_P, _I, _I64, _I64, _I64, _P, _I64, _P, _P], _I),
+    "sat_exchange_mailbox_bytes": ([_I64, _I, _I], ctypes.c_size_t),
+    "sat_exchange_create": ([ctypes.POINTER(ctypes.c_void_p), _I, _I, _I64, _I, _P,
+                             ctypes.POINTER(ctypes.c_void_p)], _I),
+    "sat_exchange_destroy": ([_P], _I),
+    "sat_compute_sharded_fused": ([_P, _P, _I64, _P, _P], _I),
+    "sat_ipc_get_handle": ([_P, _P], _I),
+    "sat_ipc_open": ([_P, ctypes.POINTER(ctypes.c_void_p)], _I),
+    "sat_ipc_close": ([_P], _I),
     "sat_compute_seeded": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
     "sat_compute_seeded_satrow": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
     "sat_column_totals": ([_P, _P, _I64, _I64, _I, _P], _I),
@@ -309,6 +317,70 @@ def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=N
         raise err[0]
     _check(st)
     return out, {f: getattr(stats, f) for f, _ in SatShardStats._fields_}
+
+
+class PeerExchange:
+    """One rank's end of the fused peer exchange (sat_exchange_create).
+
+    ``mailbox``: this rank's mailbox (a CUDA uint8 tensor of
+    ``mailbox_bytes`` bytes); ``peer_ptrs``: integer device pointers of every
+    rank's mailbox as seen from this rank (IPC-mapped for other processes).
+    Keep the tensors alive as long as the exchange.
+    """
+
+    def __init__(self, rank: int, nranks: int, cols: int, dtype, mailbox, peer_ptrs):
+        import torch
+        self.dtype = dtype
+        self.cols = int(cols)
+        self.mailbox = mailbox
+        code = {torch.int32: SAT_INT32, torch.float32: SAT_FLOAT32, torch.float64: SAT_FLOAT64}[dtype]
+        arr = (ctypes.c_void_p * nranks)(*[int(p) for p in peer_ptrs])
+        h = ctypes.c_void_p()
+        _check(_lib.sat_exchange_create(ctypes.byref(h), int(rank), int(nranks), self.cols, code,
+                                        mailbox.data_ptr(), arr))
+        self._h = h
+
+    @staticmethod
+    def mailbox_bytes(cols: int, nranks: int, dtype) -> int:
+        import torch
+        code = {torch.int32: SAT_INT32, torch.float32: SAT_FLOAT32, torch.float64: SAT_FLOAT64}[dtype]
+        return int(_lib.sat_exchange_mailbox_bytes(int(cols), int(nranks), code))
+
+    def sat(self, strip, out=None, stream=None):
+        import torch
+        if out is None:
+            out = torch.empty_like(strip)
+        _check_dev(strip, out)
+        _check(_lib.sat_compute_sharded_fused(strip.data_ptr(), out.data_ptr(), strip.shape[0],
+                                              self._h, _stream(stream)))
+        return out
+
+    def close(self):
+        if self._h:
+            _lib.sat_exchange_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def ipc_handle(t) -> bytes:
+    buf = ctypes.create_string_buffer(64)
+    _check(_lib.sat_ipc_get_handle(t.data_ptr(), buf))
+    return buf.raw
+
+
+def ipc_open(handle: bytes) -> int:
+    p = ctypes.c_void_p()
+    _check(_lib.sat_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)))
+    return int(p.value)
+
+
+def ipc_close(ptr: int) -> None:
+    _check(_lib.sat_ipc_close(ctypes.c_void_p(ptr)))
 
 
 def last_launch_count() -> int:

@@ -24,6 +24,7 @@
 #include "sat_band.cuh"
 #include "sat_paper.cuh"
 #include "sat_box.cuh"
+#include "sat_xchg.cuh"
 
 using namespace sat;
 
@@ -807,10 +808,147 @@ int exscan_core(const void* gathered, void* carry, int64_t nranks, int64_t cols,
 
 size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
+// ------------------------------------------------------------------ fused peer exchange
+struct PeerExchange {
+    int rank, nranks, dtype;
+    int64_t cols;
+    XchgParams x;             // epoch advanced per call
+    unsigned int* done;       // device block counter
+};
+
+template <typename T>
+int sharded_fused_t(const void* in, void* out, int64_t strip_rows, PeerExchange& ex, cudaStream_t st) {
+    int dev;
+    DevInfo di;
+    SAT_TRY(get_dev(dev, di));
+    Workspace* ws;
+    SAT_TRY(get_ws(dev, st, ws));
+    const int64_t cols = ex.cols;
+    ex.x.epoch += 1;
+    int launches = 0;
+    if (ex.rank < ex.nranks - 1) {
+        // 1. strip column totals; the epilogue pushes them into the higher
+        //    ranks' mailboxes and raises their flags
+        const int nc = int((cols + TW - 1) / TW);
+        long long splits = 0;
+        if (strip_rows > 0) {
+            splits = std::max<long long>(1, (4LL * di.sms + nc - 1) / nc);
+            splits = std::min<long long>(splits, (strip_rows + 63) / 64);
+            const int64_t seg = (strip_rows + splits - 1) / splits;
+            splits = (strip_rows + seg - 1) / seg;
+            SAT_TRY(ensure(ws->part, size_t(splits) * nc * TW * sizeof(T), false));
+            sat_colsum_partial_kernel<T><<<dim3(nc, unsigned(splits)), 256, 0, st>>>(
+                static_cast<const T*>(in), static_cast<T*>(ws->part.p), strip_rows, cols, seg);
+            CUDA_TRY(cudaGetLastError());
+            ++launches;
+        }
+        const unsigned blocks = unsigned(std::min<int64_t>((cols + 255) / 256, 4LL * di.sms));
+        sat_colsum_push_kernel<T><<<blocks, 256, 0, st>>>(static_cast<const T*>(ws->part.p), cols, int(splits),
+                                                          nc * TW, ex.x);
+        CUDA_TRY(cudaGetLastError());
+        ++launches;
+    }
+    const void* seed = nullptr;
+    if (ex.rank > 0) {
+        // 2. wait for ranks < p, exscan in rank order, SAT row above the strip
+        SAT_TRY(ensure(ws->seedrow, size_t(cols) * sizeof(T), false));
+        sat_seed_from_peers_kernel<T><<<1, 1024, 0, st>>>(static_cast<T*>(ws->seedrow.p), cols, ex.x);
+        CUDA_TRY(cudaGetLastError());
+        ++launches;
+        seed = ws->seedrow.p;
+    }
+    // 3. seeded local 1R1W
+    if (strip_rows > 0) {
+        SAT_TRY(compute_core(in, out, 1, strip_rows, cols, ex.dtype, SAT_1R1W, nullptr, seed,
+                             seed ? SEED_SATROW : SEED_NONE, st));
+        launches += t_launches;
+    }
+    t_launches = launches;
+    return SAT_OK;
+}
+
 }  // namespace
 
 // ====================================================================== C ABI
 extern "C" {
+
+size_t sat_exchange_mailbox_bytes(int64_t cols, int nranks, int dtype) {
+    if (cols <= 0 || nranks <= 0 || !dtype_ok(dtype)) return 0;
+    XchgLayout L{nranks, cols, esize(dtype)};
+    return L.bytes();
+}
+
+int sat_exchange_create(void** handle, int rank, int nranks, int64_t cols, int dtype, void* mailbox,
+                        void* const* peers) {
+    if (!handle) return fail(SAT_ERR_INVALID, "null handle");
+    *handle = nullptr;
+    if (!dtype_ok(dtype)) return fail(SAT_ERR_INVALID, "bad dtype");
+    if (nranks < 1 || nranks > 16 || rank < 0 || rank >= nranks)
+        return fail(SAT_ERR_INVALID, "nranks must be 1..16 and 0 <= rank < nranks");
+    if (cols <= 0 || !mailbox || !peers) return fail(SAT_ERR_INVALID, "bad cols / null pointer");
+    for (int q = 0; q < nranks; ++q)
+        if (!peers[q]) return fail(SAT_ERR_INVALID, "null peer mailbox");
+    if (reinterpret_cast<uintptr_t>(mailbox) & 255) return fail(SAT_ERR_INVALID, "mailbox must be 256-B aligned");
+    PeerExchange* ex = new PeerExchange();
+    ex->rank = rank; ex->nranks = nranks; ex->dtype = dtype; ex->cols = cols;
+    std::memset(&ex->x, 0, sizeof(ex->x));
+    ex->x.L = XchgLayout{nranks, cols, esize(dtype)};
+    ex->x.rank = rank;
+    ex->x.epoch = 0;
+    ex->x.mine = static_cast<uint8_t*>(mailbox);
+    for (int q = 0; q < nranks; ++q) ex->x.peers[q] = static_cast<uint8_t*>(peers[q]);
+    if (cudaMalloc(&ex->done, sizeof(unsigned int)) != cudaSuccess) {
+        cudaGetLastError();
+        delete ex;
+        return fail(SAT_ERR_NOMEM, "exchange counter");
+    }
+    ex->x.done = ex->done;
+    CUDA_TRY(cudaMemset(ex->done, 0, sizeof(unsigned int)));
+    CUDA_TRY(cudaMemset(mailbox, 0, ex->x.L.bytes()));
+    CUDA_TRY(cudaDeviceSynchronize());
+    *handle = ex;
+    return SAT_OK;
+}
+
+int sat_exchange_destroy(void* handle) {
+    PeerExchange* ex = static_cast<PeerExchange*>(handle);
+    if (!ex) return SAT_OK;
+    cudaFree(ex->done);
+    delete ex;
+    return SAT_OK;
+}
+
+int sat_compute_sharded_fused(const void* in_strip, void* out_strip, int64_t strip_rows, void* handle,
+                              void* stream) {
+    t_launches = 0;
+    PeerExchange* ex = static_cast<PeerExchange*>(handle);
+    if (!ex) return fail(SAT_ERR_INVALID, "null exchange");
+    SAT_TRY(validate(in_strip, out_strip, 1, strip_rows, ex->cols, ex->dtype));
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    return SAT_DISPATCH(ex->dtype, T, sharded_fused_t<T>(in_strip, out_strip, strip_rows, *ex, st));
+}
+
+int sat_ipc_get_handle(const void* dev_ptr, void* handle64) {
+    if (!dev_ptr || !handle64) return fail(SAT_ERR_INVALID, "null pointer");
+    cudaIpcMemHandle_t h;
+    CUDA_TRY(cudaIpcGetMemHandle(&h, const_cast<void*>(dev_ptr)));
+    std::memcpy(handle64, &h, sizeof(h));
+    return SAT_OK;
+}
+
+int sat_ipc_open(const void* handle64, void** dev_ptr) {
+    if (!handle64 || !dev_ptr) return fail(SAT_ERR_INVALID, "null pointer");
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle64, sizeof(h));
+    CUDA_TRY(cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+    return SAT_OK;
+}
+
+int sat_ipc_close(void* dev_ptr) {
+    if (!dev_ptr) return SAT_OK;
+    CUDA_TRY(cudaIpcCloseMemHandle(dev_ptr));
+    return SAT_OK;
+}
 
 void sat_options_init(sat_options* opt) {
     if (!opt) return;

@@ -77,3 +77,26 @@ def sharded_sat(strip: torch.Tensor, group=None, ops=None, out=None, timings=Non
                  extra_bytes_read=(rows * cols * eb if (P > 1 and rank < P - 1) else 0),
                  allgather_bytes=(P * cols * eb if P > 1 else 0))
     return out, stats
+
+
+def make_peer_exchange(cols: int, dtype, group=None, device=None, ipc=None, factory=None):
+    """Set up this rank's fused peer exchange.
+
+    Every rank allocates a zeroed mailbox on its GPU, publishes its CUDA IPC
+    handle with one ``all_gather_object`` (set-up only, not per call) and maps
+    the other ranks' mailboxes.  ``ipc`` = (get_handle, open) and ``factory``
+    (the PeerExchange constructor) are injectable so the set-up can be tested
+    on CPU with gloo.  Returns ``(exchange, peer_ptrs)``.
+    """
+    from . import PeerExchange, ipc_handle, ipc_open
+    get_handle, open_handle = ipc or (ipc_handle, ipc_open)
+    factory = factory or PeerExchange
+    rank = dist.get_rank(group)
+    P = dist.get_world_size(group)
+    nbytes = PeerExchange.mailbox_bytes(cols, P, dtype) if factory is PeerExchange else 4096
+    mailbox = torch.zeros(nbytes, dtype=torch.uint8, device=device)
+    handles = [None] * P
+    dist.all_gather_object(handles, get_handle(mailbox), group=group)
+    ptrs = [mailbox.data_ptr() if q == rank else open_handle(handles[q]) for q in range(P)]
+    ex = factory(rank, P, cols, dtype, mailbox, ptrs)
+    return ex, ptrs

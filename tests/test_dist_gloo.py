@@ -91,3 +91,51 @@ def test_partition_rows():
         assert all(b[i][1] == b[i + 1][0] for i in range(P - 1))
     r = [partition_rows(65536, 8, p, 1.5) for p in range(8)]
     assert r[-1][1] - r[-1][0] > r[0][1] - r[0][0]
+
+
+def _xchg_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_kasagini14_b200.dist import make_peer_exchange
+    opened = []
+
+    def get_handle(t):
+        return f"mailbox-of-{rank}".encode()
+
+    def open_handle(h):
+        opened.append(h)
+        return 1000 + int(h.decode().rsplit("-", 1)[1])      # fake peer address of that rank
+
+    made = {}
+
+    def factory(r, P, cols, dtype, mailbox, ptrs):
+        made.update(rank=r, P=P, cols=cols, nbytes=mailbox.numel(), ptrs=list(ptrs),
+                    own=mailbox.data_ptr())
+        return "exchange"
+    ex, ptrs = make_peer_exchange(777, torch.int32, ipc=(get_handle, open_handle), factory=factory)
+    q.put((rank, ex, made, opened))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_peer_exchange_setup_world3():
+    """Fused-exchange set-up: every rank maps every OTHER rank's
+    mailbox from its published handle, in rank order, and keeps its own."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    world = 3
+    procs = [ctx.Process(target=_xchg_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=60) for _ in range(world)], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, ex, made, opened in res:
+        assert ex == "exchange" and made["rank"] == rank and made["P"] == world and made["cols"] == 777
+        assert made["ptrs"][rank] == made["own"]
+        assert [made["ptrs"][qq] for qq in range(world) if qq != rank] == \
+            [1000 + qq for qq in range(world) if qq != rank]
+        assert sorted(opened) == sorted(f"mailbox-of-{qq}".encode() for qq in range(world) if qq != rank)

@@ -451,3 +451,40 @@ def test_4r4w_cfg2_and_4r1w_4096(libsat):
     a = gen(4096, 4096, "int32", seed=2)
     check(libsat.sat(dev(a), variant="4r1w"), oracle.sat(a), "int32")
     assert libsat.last_launch_count() == 4096 + 4096 - 1
+
+
+# ------------------------------------------------------------------ fused peer exchange
+@pytest.mark.parametrize("P", [2, 3, 8])
+@pytest.mark.parametrize("dtype", ["int32", "float32", "float64"])
+def test_fused_exchange_single_device(libsat, P, dtype):
+    """P virtual ranks on one GPU, each on its own stream with its own mailbox
+    (the peer pointers are plain device pointers instead of IPC mappings --
+    the kernels and the flag/acknowledge protocol are the same).  Several
+    consecutive calls reuse both mailbox parities without any barrier; every
+    call must equal the unsharded SAT (bit-exact for int32 / dyadic float64)."""
+    from paper_conf_icpp_kasagini14_b200.dist import partition_rows
+    tdt = {"int32": torch.int32, "float32": torch.float32, "float64": torch.float64}[dtype]
+    n, m = 1500, 1300
+    nb = libsat.PeerExchange.mailbox_bytes(m, P, tdt)
+    boxes = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(P)]
+    ptrs = [b.data_ptr() for b in boxes]
+    exs = [libsat.PeerExchange(p, P, m, tdt, boxes[p], ptrs) for p in range(P)]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    bounds = [partition_rows(n, P, p) for p in range(P)]
+    for it in range(5):
+        full = make_np(n, m, dtype, "u32" if dtype == "int32" else "unit", seed=it)
+        ref = oracle.sat(full)
+        strips = [dev(full[a:b]) for a, b in bounds]
+        outs = [torch.empty_like(s) for s in strips]
+        torch.cuda.synchronize()
+        for p in range(P):
+            with torch.cuda.stream(streams[p]):
+                exs[p].sat(strips[p], out=outs[p], stream=streams[p])
+        torch.cuda.synchronize()
+        got = np.concatenate([o.cpu().numpy() for o in outs])
+        if dtype == "float32":
+            check(got, ref, "float32")
+        else:
+            assert np.array_equal(got, ref), f"call {it}"
+    for e in exs:
+        e.close()
