@@ -227,6 +227,9 @@ constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
+// TH = 112: 14 compute warps, one CTA per SM; fills the SMs where TH = 128
+// leaves a partial wave (16384 rows: 147 bands on 148 SMs instead of 128)
+constexpr BandCfg kCfg112{8, 14, 3, 4, 1, 3, 1, 1};
 // float64 (8-byte elements: 1 KB chunk rows, two TMEM words per element)
 constexpr BandCfg kCfgD16{2, 8, 4, 4, 1, 3, 1, 2};   //  96 KB smem, 128 TMEM cols: 2 CTAs/SM
 constexpr BandCfg kCfgD32{4, 8, 4, 8, 1, 4, 1, 1};   // 192 KB smem, 512 TMEM cols
@@ -236,7 +239,7 @@ constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 3, 1, 1};   // 224 KB smem, 512 TMEM co
 // CTAs per SM of a configuration (for wave counts before launch)
 int ctas_per_sm(int dtype, int th, bool big) {
     if (dtype == SAT_FLOAT64) return th == 16 ? 2 : 1;
-    return (th == 128 || big) ? 1 : 2;
+    return (th == 128 || th == 112 || big) ? 1 : 2;
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
@@ -335,6 +338,14 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
             }
             return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1>(p, ti, to, di, st, grid);
         }
+        if (th == 128) {
+            if (const char* e = getenv("SAT_DEBUG_LBW")) {
+                const int lbw = atoi(e);
+                if (lbw == 8) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
+                if (lbw == 2) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (lbw == 42) return launch_band_t<T, 8, 16, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+            }
+        }
         if (p.cluster == 8 && th == 64)
             return launch_band_t<T, 8, 8, 3, 3, 1, 3, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
         if (p.cluster == 8 && th == 48)
@@ -345,9 +356,10 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
         case 48: return launch_band_t<T, SAT_CFG(kCfg48), MODE, TMA, kCfg48.MINB>(p, ti, to, di, st, grid);
         case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
+        case 112: return launch_band_t<T, SAT_CFG(kCfg112), MODE, TMA, kCfg112.MINB>(p, ti, to, di, st, grid);
         case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
     }
-    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64 or 128");
+    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64, 112 or 128");
     }
 }
 
@@ -475,6 +487,8 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         }
     }
     p.jitter = j.jitter;
+    p.pf = 0;
+    if (const char* e = getenv("SAT_PF")) p.pf = std::max(0, atoi(e));
     p.diag = g_diag_dev;
     if (const char* e = getenv("SAT_DEBUG_NOLB")) p.dbg = atoi(e);   // 1: no look-back, 2: publish only
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
@@ -684,8 +698,8 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     sat_options_init(&o);
     if (opt) o = *opt;
     if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 48 &&
-        o.tile_rows != 64 && o.tile_rows != 128)
-        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48, 64 or 128");
+        o.tile_rows != 64 && o.tile_rows != 112 && o.tile_rows != 128)
+        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48, 64, 112 or 128");
     if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     int dev;
@@ -1199,9 +1213,14 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
         CUDA_TRY(cudaStreamCreateWithFlags(&ws->cstream_in, cudaStreamNonBlocking));
         CUDA_TRY(cudaStreamCreateWithFlags(&ws->cstream_out, cudaStreamNonBlocking));
     }
-    const int nstrips = int(std::min<int64_t>(8, rows / 256));
+    // 32 strips: fill/drain of the copy pipeline is 1/32 of the transfer
+    // (32768^2 int32: 89.9 ms vs 95.3 ms with 8 strips; H2D+D2H concurrently
+    // take 87.8 ms, tools/pcie_probe.py)
+    int want = 32;
+    if (const char* e = getenv("SAT_HOST_STRIPS")) want = std::max(1, std::min(64, atoi(e)));
+    const int nstrips = int(std::min<int64_t>(want, rows / 256));
     const int64_t srows = (rows + nstrips - 1) / nstrips;
-    cudaEvent_t ev_start, ev_in[8], ev_done[8];
+    cudaEvent_t ev_start, ev_in[64], ev_done[64];
     CUDA_TRY(cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming));
     for (int k = 0; k < nstrips; ++k) {
         CUDA_TRY(cudaEventCreateWithFlags(&ev_in[k], cudaEventDisableTiming));

@@ -822,10 +822,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if constexpr (TMA) {
                 if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
+                    int kpf = S * SUB;                       // next chunk to prefetch into L2
                     for (int k0 = 0; k0 < nch; k0 += SUB) {
                         const uint32_t q = gq + uint32_t(k0 / SUB);
                         const int s = q % S;
                         const int nsub = nch - k0 < SUB ? nch - k0 : SUB;
+                        // L2 prefetch p.pf chunks ahead of the load (beyond the ring)
+                        for (; kpf < nch && kpf < k0 + p.pf; ++kpf)
+                            tma_prefetch_3d(&tm_in, (j0 + kpf) * TW, row0, img);
                         if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
                         if (traced)
                             p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();

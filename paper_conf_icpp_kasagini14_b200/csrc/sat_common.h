@@ -69,6 +69,7 @@ struct BandParams {
     int nseg;                  // 1 = whole bands
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
+    int pf;                    // L2 prefetch distance in chunks (TMA path; 0 = off)
 };
 
 }  // namespace sat

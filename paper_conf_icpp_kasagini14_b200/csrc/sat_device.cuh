@@ -153,6 +153,12 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* m, uin
            "r"(smem_u32(bar)), "l"(policy)
         : "memory");
 }
+// HBM -> L2 only (no shared memory, no barrier): raises the bytes in flight
+// per SM beyond the shared-memory ring
+__device__ __forceinline__ void tma_prefetch_3d(const CUtensorMap* m, int c0, int c1, int c2) {
+    asm volatile("cp.async.bulk.prefetch.tensor.3d.L2.global.tile [%0, {%1, %2, %3}];"
+                 :: "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(c2) : "memory");
+}
 __device__ __forceinline__ void tma_store_3d(const CUtensorMap* m, const void* src,
                                              int c0, int c1, int c2, uint64_t policy) {
     asm volatile(

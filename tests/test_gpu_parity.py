@@ -69,7 +69,7 @@ def test_shapes(libsat, variant, dtype, shape):
     check(libsat.sat(dev(a), variant=variant), ref, dtype)
 
 
-@pytest.mark.parametrize("tile_rows", [16, 32, 48, 64, 128])
+@pytest.mark.parametrize("tile_rows", [16, 32, 48, 64, 112, 128])
 @pytest.mark.parametrize("generic", [False, True])
 @pytest.mark.parametrize("variant", VARIANTS)
 def test_tile_configs(libsat, tile_rows, generic, variant):
@@ -134,7 +134,7 @@ def test_repeated_calls_fresh_tags(libsat):
 
 
 def test_lookback_jitter_stress(libsat):
-    for th in (16, 32, 48, 64, 128):
+    for th in (16, 32, 48, 64, 112, 128):
         a = gen(3000, 2500, "int32", seed=th)
         check(libsat.sat(dev(a), tile_rows=th, jitter=20000), oracle.sat(a), "int32")
         af = gen(3000, 2500, "float32", seed=th)
@@ -372,7 +372,7 @@ def test_big_ring_config(libsat, shape, monkeypatch):
 
 
 @pytest.mark.parametrize("nseg", [2, 3, 7])
-@pytest.mark.parametrize("tile_rows", [64, 128])
+@pytest.mark.parametrize("tile_rows", [64, 112, 128])
 def test_band_segments(libsat, nseg, tile_rows, monkeypatch):
     """Band segments: a ticket is (segment, band) and the
     row carry crosses segments through tagged words; every split is exact."""
