@@ -227,6 +227,8 @@ constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
+constexpr int kLbw128 = 2;   // look-back window (bands per round trip) at TH = 128:
+                             // 2 measured ~1 % faster than 4 at 16384^2/18432^2, 8 slower
 // TH = 112: 14 compute warps, one CTA per SM; fills the SMs where TH = 128
 // leaves a partial wave (16384 rows: 147 bands on 148 SMs instead of 128)
 constexpr BandCfg kCfg112{8, 14, 3, 4, 1, 3, 1, 1};
@@ -338,12 +340,11 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
             }
             return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1>(p, ti, to, di, st, grid);
         }
-        if (th == 128) {
+        if (th == 128) {   // A/B of the look-back window (8 and NS = 2 measured slower)
             if (const char* e = getenv("SAT_DEBUG_LBW")) {
                 const int lbw = atoi(e);
-                if (lbw == 8) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
-                if (lbw == 2) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (lbw == 42) return launch_band_t<T, 8, 16, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (lbw == 4) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 4>(p, ti, to, di, st, grid);
+                if (lbw == 1) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
             }
         }
         if (p.cluster == 8 && th == 64)
@@ -357,7 +358,11 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         case 48: return launch_band_t<T, SAT_CFG(kCfg48), MODE, TMA, kCfg48.MINB>(p, ti, to, di, st, grid);
         case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
         case 112: return launch_band_t<T, SAT_CFG(kCfg112), MODE, TMA, kCfg112.MINB>(p, ti, to, di, st, grid);
-        case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
+        case 128:
+            if constexpr (MODE == MODE_SAT)
+                return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, 1, kLbw128>(p, ti, to, di, st, grid);
+            else
+                return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
     }
     return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64, 112 or 128");
     }
