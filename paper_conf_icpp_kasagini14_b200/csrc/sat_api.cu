@@ -494,6 +494,7 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.jitter = j.jitter;
     p.pf = 0;
     if (const char* e = getenv("SAT_PF")) p.pf = std::max(0, atoi(e));
+    if (const char* e = getenv("SAT_UNIT_SYNC")) p.unit_sync = atoi(e) != 0;
     p.diag = g_diag_dev;
     if (const char* e = getenv("SAT_DEBUG_NOLB")) p.dbg = atoi(e);   // 1: no look-back, 2: publish only
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {

@@ -105,8 +105,9 @@ struct BandSmem {
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
     // clusters: incoming partial aggregate (chain) and cluster top row per carry slot
     static constexpr size_t cbuf = CL > 1 ? size_t(2) * XS * TW * sizeof(T) : 0;
-    static constexpr size_t nbars = 2 * S + 2 * XS + (CL > 1 ? 4 * XS : 0);
-    static constexpr size_t bars = nbars * sizeof(uint64_t) + 16;
+    // + unit queue (CL == 1): ufull[2], uempty[2]
+    static constexpr size_t nbars = 2 * S + 2 * XS + (CL > 1 ? 4 * XS : 4);
+    static constexpr size_t bars = nbars * sizeof(uint64_t) + 32;   // + s_unit[2], s_tmem
     static constexpr size_t total = tiles + xbuf + cbuf + bars;
 };
 
@@ -328,8 +329,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint64_t* aggfree = aggb + XS;
     uint64_t* ctopb = aggb + 2 * XS;
     uint64_t* ctopfree = aggb + 3 * XS;
+    // unit queue (CL == 1): the producer warp takes the
+    // next ticket as soon as it has issued the last load of the current unit
+    // and posts it in s_unit[u & 1] (ufull); the other warps read it and
+    // release the entry (uempty), so the next unit's loads overlap the
+    // current unit's last look-backs and stores
+    uint64_t* ufull = bars + 2 * S + 2 * XS;
+    uint64_t* uempty = ufull + 2;
     long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
-    uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 1);
+    uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 2);
     const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
 
     const int warp = threadIdx.x >> 5;
@@ -339,6 +347,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         for (int s = 0; s < S; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], W * 32);
+        }
+        if constexpr (CL == 1) {
+            for (int u = 0; u < 2; ++u) {
+                mbar_init(&ufull[u], 1);
+                mbar_init(&uempty[u], W + NCW);      // lane 0 of every non-producer warp
+            }
         }
         for (int x = 0; x < XS; ++x) {
             mbar_init(&colr[x], W * 32);
@@ -371,7 +385,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint32_t g = 0;                              // CTA-local chunk counter (carry / TMEM slots)
     uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
 
-    for (;;) {
+    for (uint32_t useq = 0;; ++useq) {
         if constexpr (CL > 1) {
             // one ticket per cluster: CL consecutive bands, rank r takes band CL*u + r
             if (crank == 0 && threadIdx.x == 0) {
@@ -379,12 +393,27 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 for (uint32_t r = 0; r < CL; ++r) st_cluster_u64(mapa(smem_u32(s_unit), r), u);
             }
             cluster_sync_all();
-        } else {
-            if (threadIdx.x == 0)
-                *s_unit = (long long)(atomicAdd(p.ticket, 1ull) - p.base);
-            __syncthreads();
         }
-        const long long unit = *s_unit;
+        long long unit;
+        if constexpr (CL > 1) {
+            unit = *s_unit;
+        } else {
+            const uint32_t qs = useq & 1u, qph = (useq >> 1) & 1u;
+            if (warp == PW) {
+                if (lane == 0) {
+                    if (useq >= 2) mbar_wait(&uempty[qs], qph ^ 1u);   // every warp read unit useq-2
+                    s_unit[qs] = (long long)(atomicAdd(p.ticket, 1ull) - p.base);
+                    mbar_arrive(&ufull[qs]);
+                }
+                __syncwarp();
+                mbar_wait(&ufull[qs], qph);
+            } else {
+                mbar_wait(&ufull[qs], qph);
+            }
+            unit = s_unit[qs];
+            __syncwarp();
+            if (warp != PW && lane == 0) mbar_arrive(&uempty[qs]);
+        }
         diag_mark(p.diag, uint32_t(unit), 0, 1);
         if (unit < 0) __trap();                       // ticket accounting out of sync: never silently
         if (p.diag != nullptr && threadIdx.x == 0) {
@@ -619,7 +648,12 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
                 const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
-                for (int k = grp; k < nch; k += G) {
+                // group grp owns the CTA-global chunks it = g + k with it = grp
+                // (mod G), across unit boundaries: consecutive chunks of a
+                // group are exactly G <= XS apart, so its parity waits on
+                // colr[] can never pass on a stale phase (with the unit queue
+                // the next unit starts before every group finished this one)
+                for (int k = int((uint32_t(grp) + uint32_t(G) - g % uint32_t(G)) % uint32_t(G)); k < nch; k += G) {
                     const uint32_t it = g + k;
                     const int J = j0 + k;
                     const int c0 = J * TW + cl;
@@ -845,7 +879,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
         if constexpr (CL > 1) cluster_sync_all();      // before rank 0 overwrites s_unit
-        else __syncthreads();
+        else if (p.unit_sync) __syncthreads();         // A/B: no overlap of consecutive units
     }
     diag_mark(p.diag, 0xFFFFFFFFu, 0, 6);
     if (HOLD) {

@@ -70,6 +70,7 @@ struct BandParams {
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
     int pf;                    // L2 prefetch distance in chunks (TMA path; 0 = off)
+    int unit_sync;             // A/B: 1 = the next unit starts only after every warp finished this one
 };
 
 }  // namespace sat

@@ -393,6 +393,33 @@ def test_band_segments(libsat, nseg, tile_rows, monkeypatch):
     check(libsat.sat(x, tile_rows=tile_rows, jitter=20000), ref, "int32")
 
 
+@pytest.mark.parametrize("nseg", [3, 4, 5])
+@pytest.mark.parametrize("tile_rows", [64, 112, 128])
+def test_unit_queue_many_units(libsat, nseg, tile_rows, monkeypatch):
+    """Many short units per CTA: the next unit's loads
+    start before the current unit's control groups are done, so a group's
+    chunks must stay G apart across unit boundaries.  Segments of a number of
+    chunks that is not a multiple of the control-group count (3 at TH 112/128)
+    failed before the assignment became CTA-global."""
+    monkeypatch.setenv("SAT_SEG", str(nseg))
+    a = gen(20000, 3000, "int32", seed=nseg + tile_rows)
+    ref = oracle.sat(a)
+    x = dev(a)
+    check(libsat.sat(x, tile_rows=tile_rows), ref, "int32")
+    check(libsat.sat(x, tile_rows=tile_rows, jitter=20000), ref, "int32")
+    af = gen(9000, 2500, "float32", seed=nseg)
+    check(libsat.sat(dev(af), tile_rows=tile_rows), oracle.sat(af), "float32")
+    # 65536 x 4096 all ones, in place (1 GiB): 2048 units of 8 chunks at nseg 4
+    if nseg == 4:
+        n, m = 65536, 4096
+        y = torch.ones(n, m, dtype=torch.int32, device="cuda")
+        libsat.sat(y, out=y, tile_rows=tile_rows)
+        jj = torch.arange(1, m + 1, device="cuda", dtype=torch.int64)
+        for r in (0, 127, 17664, 18944, 40000, n - 1):
+            assert torch.equal(y[r].to(torch.int64) % 2**32, ((r + 1) * jj) % 2**32), r
+        assert int(y[n - 1, m - 1]) == (n * m) % 2**32 - (2**32 if (n * m) % 2**32 >= 2**31 else 0)
+
+
 # ------------------------------------------------------------------ 4R4W / 4R1W (SURVEY 8(f3))
 PAPER_VARIANTS = ["4r4w", "4r1w"]
 
