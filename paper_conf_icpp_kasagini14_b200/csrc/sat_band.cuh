@@ -862,8 +862,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         const int s = q % S;
                         const int nsub = nch - k0 < SUB ? nch - k0 : SUB;
                         // L2 prefetch p.pf chunks ahead of the load (beyond the ring)
-                        for (; kpf < nch && kpf < k0 + p.pf; ++kpf)
-                            tma_prefetch_3d(&tm_in, (j0 + kpf) * TW, row0, img);
+                        if (p.pf > S * SUB)
+                            for (; kpf < nch && kpf < k0 + p.pf; ++kpf)
+                                tma_prefetch_3d(&tm_in, (j0 + kpf) * TW, row0, img);
                         if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
                         if (traced)
                             p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();

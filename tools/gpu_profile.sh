@@ -15,3 +15,11 @@ for cfg in ${EXTRA_CFGS:-cfg3b}; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:sat_band_kernel -s 2 -c 1 \
     -o gpurun_out/prof_$cfg python tools/prof_one.py $cfg 0 3 >> gpurun_out/ncu_full.log 2>&1
 done
+# export text pages on the box (the .ncu-rep files exceed gpurun's 64 MiB return limit)
+for r in gpurun_out/prof_*.ncu-rep; do
+  b=${r%.ncu-rep}
+  ncu -i $r --page raw --csv > ${b}_raw.csv 2>/dev/null
+  ncu -i $r --page details > ${b}_details.txt 2>/dev/null
+  ncu -i $r --page source --csv > ${b}_source.csv 2>/dev/null
+  rm -f $r
+done

@@ -1,6 +1,6 @@
 """Summarise ncu captures into profiles/ (run here, on the CPU box).
 
-python tools/ncu_summarize.py <rep.ncu-rep> <workload key> <alg_bytes_per_launch> [out_dir]
+python tools/ncu_summarize.py <rep.ncu-rep | raw.csv> <workload key> <alg_bytes_per_launch> [out_dir]
 
 Appends/updates profiles/ncu_summary.json[key] with the per-launch DRAM bytes,
 duration and throughput of the captured band-kernel launch(es), and writes a
@@ -25,8 +25,11 @@ UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
 def main():
     rep, key, alg = sys.argv[1], sys.argv[2], float(sys.argv[3])
     out_dir = sys.argv[4] if len(sys.argv) > 4 else "profiles"
-    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
-                         text=True, check=True).stdout
+    if rep.endswith(".csv"):          # `ncu -i X --page raw --csv` exported on the GPU box
+        raw = open(rep).read()
+    else:
+        raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
+                             text=True, check=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units = rows[0], rows[1]
     launches = []
