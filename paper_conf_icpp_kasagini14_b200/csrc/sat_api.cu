@@ -479,11 +479,14 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.segc = p.nc;
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && p.region == REG_ALL && !p.tile_units &&
         p.cluster == 1 && p.Lx == nullptr && p.Lb == nullptr) {
-        // >= 2 waves of bands: ~16 segments of >= 32 chunks (65536^2, TH 128:
-        // 5.97 ms with 16 segments vs 6.34 ms whole bands); one wave: whole
-        // bands (a segment would wait for the band's previous segment)
+        // more bands than resident CTAs: up to 16 segments of >= 16 chunks, so
+        // the partial last wave of whole bands becomes many short units
+        // (65536^2 TH 128: 5.97 ms with 16 segments vs 6.34 ms whole bands;
+        // 20480^2: 0.614 ms with 8-10 vs 0.887 ms; 12288^2 float64: 0.608 vs
+        // 0.785 ms); at most one wave: whole bands (a segment would wait for
+        // the band's previous segment)
         const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0);
-        int want = p.total_bands >= 2 * slots ? std::min(16, p.nc / 32) : 1;
+        int want = p.total_bands > slots ? std::min(16, p.nc / 16) : 1;
         if (const char* e = getenv("SAT_SEG")) want = std::max(1, atoi(e));
         if (want > 1 && p.nc > 1) {
             p.segc = (p.nc + want - 1) / want;
