@@ -236,7 +236,10 @@ constexpr BandCfg kCfg112{8, 14, 3, 4, 1, 3, 1, 1};
 constexpr BandCfg kCfgD16{2, 8, 4, 4, 1, 3, 1, 2};   //  96 KB smem, 128 TMEM cols: 2 CTAs/SM
 constexpr BandCfg kCfgD32{4, 8, 4, 8, 1, 4, 1, 1};   // 192 KB smem, 512 TMEM cols
 constexpr BandCfg kCfgD48{8, 6, 3, 4, 1, 4, 1, 1};   // 168 KB smem, 512 TMEM cols
-constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 3, 1, 1};   // 224 KB smem, 512 TMEM cols
+// TH 64: ONE control group of 2 warps that split the columns (NS = 2: 2
+// columns per lane, 4 descriptor words per band, look-back window 4):
+// 16384^2 0.917 vs 1.04 ms with 3 groups of 1 warp, 32768^2 3.49 vs 3.87
+constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM cols
 
 // CTAs per SM of a configuration (for wave counts before launch)
 int ctas_per_sm(int dtype, int th, bool big) {
@@ -322,6 +325,23 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
         }
     }
     if constexpr (sizeof(T) == 8) {
+        if constexpr (MODE == MODE_SAT && TMA) {
+            if (const char* e = getenv("SAT_DEBUG_F64")) {   // A/B of the float64 look-back
+                const int v = atoi(e);
+                if (th == 64 && v == 1) return launch_band_t<T, 8, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 2) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 3) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 1, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 5) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 6) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 7) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 8) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 9) return launch_band_t<T, 8, 8, 3, 4, 1, 1, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 10) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (th == 64 && v == 11) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
+                if (th == 32 && v == 6) return launch_band_t<T, 4, 8, 4, 8, 1, 2, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
+            }
+        }
         switch (th) {
             case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, to, di, st, grid);
             case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, to, di, st, grid);
@@ -345,6 +365,9 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
                 const int lbw = atoi(e);
                 if (lbw == 4) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 4>(p, ti, to, di, st, grid);
                 if (lbw == 1) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
+                if (lbw == 22) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (lbw == 12) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
+                if (lbw == 24) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 4>(p, ti, to, di, st, grid);
             }
         }
         if (p.cluster == 8 && th == 64)
