@@ -322,6 +322,11 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUt
             if (th == 64 && ns == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
             if (th == 32 && ns == 2) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
             if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            // one group of two column-splitting control warps (as float64 TH 64)
+            if (th == 16 && ns == 22) return launch_band_t<T, 4, 4, 3, 8, 4, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 32 && ns == 22) return launch_band_t<T, 8, 4, 3, 8, 2, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 64 && ns == 22) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
+            if (th == 48 && ns == 22) return launch_band_t<T, 8, 6, 2, 4, 2, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
         }
     }
     if constexpr (sizeof(T) == 8) {
@@ -432,19 +437,25 @@ int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtenso
 // raise parallelism, taller bands cut descriptor traffic).
 int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dtype) {
     if (dtype == SAT_FLOAT64) {
-        // one CTA per SM for TH 32/64 (1-KB rows): the tallest band with a wave
+        // one CTA per SM for TH 32/64 (1-KB rows): the tallest band with a
+        // wave; below that TH 32 from 1024 rows (a shorter look-back chain
+        // beats filling the SMs: 1024^2 0.031 vs 0.034 ms, 2048^2 0.054 vs 0.063)
         for (int th : {64, 32}) {
             const long long bands = batch * ((rows + th - 1) / th);
             if (bands * 5 >= 4LL * di.sms) return th;
         }
-        return 16;
+        return rows * batch >= 1024 ? 32 : 16;
     }
-    // 1R1W: TH = 128 (one CTA per SM) once its bands fill a wave (16K^2,
-    // 18432^2: measured 5.3-5.4 TB/s vs 5.0 for TH = 64; 65536^2 with band
-    // segments: 5.97 ms vs 6.27 ms for TH = 64).
+    // 1R1W: TH = 128 (one CTA per SM) once its bands fill half the SMs: in
+    // the one-wave regime the look-back chain (one hop per band) costs more
+    // than idle SMs (A/B sweep, int32: 10240^2 0.200 ms vs 0.224 for TH 32,
+    // 12288^2 0.254 vs 0.313, 14336^2 0.327 vs 0.417; 16K^2+: 5.3-5.4 TB/s vs
+    // 5.0 for TH 64); below that TH 32 from 1536 rows (2048^2-8192^2: 15-25 %
+    // faster than TH 16), else TH 16.
     if (variant == SAT_1R1W) {
         const long long b128 = batch * ((rows + 127) / 128);
-        if (b128 * 5 >= 4LL * di.sms) return 128;
+        if (b128 * 2 >= di.sms) return 128;
+        return rows * batch >= 1536 ? 32 : 16;
     }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
     for (int th : {64, 32}) {
