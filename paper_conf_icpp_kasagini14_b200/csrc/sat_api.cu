@@ -643,7 +643,8 @@ int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, cons
     // Step 3: re-read, add carries, tile SAT, write (tile tickets, external carries)
     BandParams p = base_params();
     p.top_src = TOP_EXTERNAL;
-    p.tile_units = 1;
+    p.tile_units = 0;
+    if (const char* e = getenv("SAT_TILE_UNITS")) p.tile_units = atoi(e) != 0;
     p.region = region;
     p.tA = tA;
     p.Lx = ws.lx.p;
