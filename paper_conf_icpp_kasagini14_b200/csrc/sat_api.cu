@@ -637,7 +637,7 @@ int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, cons
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     const int W = c.nc * TW;
-    sat_carry_top_kernel<T><<<dim3((W + 255) / 256, unsigned(j.batch)), 256, 0, j.st>>>(cp);
+    sat_carry_top_kernel<T><<<dim3((W + 31) / 32, unsigned(j.batch)), 256, 0, j.st>>>(cp);
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     // Step 3: re-read, add carries, tile SAT, write (tile tickets, external carries)

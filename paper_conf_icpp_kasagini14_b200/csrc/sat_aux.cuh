@@ -41,23 +41,36 @@ sat_reduce_kernel(const TileParams p)
     const bool vec = (p.cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(p.in) & 15) == 0);
     T cs[4] = {T(0), T(0), T(0), T(0)};
     T* rs = reinterpret_cast<T*>(p.RS) + int64_t(J) * p.total_bands * p.th + int64_t(gb) * p.th;
-    for (int r = warp; r < p.th; r += 8) {
-        const int64_t row = int64_t(band) * p.th + r;
-        T e[4] = {T(0), T(0), T(0), T(0)};
-        if (row < p.rows) {
-            if (vec && c + 3 < p.cols) {
-                ldg4<T>(gin + row * p.cols + c, e);
-            } else {
+    // rows warp, warp+8, ... in batches of 8: all loads of a batch are issued
+    // before the first shuffle reduction (memory-level parallelism)
+    constexpr int B = 8;
+    for (int r0 = warp; r0 < p.th; r0 += 8 * B) {
+        T e[B][4];
 #pragma unroll
-                for (int i = 0; i < 4; ++i) if (c + i < p.cols) e[i] = gin[row * p.cols + c + i];
+        for (int q = 0; q < B; ++q) {
+            const int r = r0 + 8 * q;
+            const int64_t row = int64_t(band) * p.th + r;
+#pragma unroll
+            for (int i = 0; i < 4; ++i) e[q][i] = T(0);
+            if (r < p.th && row < p.rows) {
+                if (vec && c + 3 < p.cols) {
+                    ldg4<T>(gin + row * p.cols + c, e[q]);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) if (c + i < p.cols) e[q][i] = gin[row * p.cols + c + i];
+                }
             }
         }
-        T sr = (e[0] + e[1]) + (e[2] + e[3]);
 #pragma unroll
-        for (int i = 0; i < 4; ++i) cs[i] += e[i];
+        for (int q = 0; q < B; ++q) {
+            const int r = r0 + 8 * q;
+            T sr = (e[q][0] + e[q][1]) + (e[q][2] + e[q][3]);
 #pragma unroll
-        for (int d = 16; d > 0; d >>= 1) sr += __shfl_xor_sync(0xffffffffu, sr, d);
-        if (lane == 0) rs[r] = sr;
+            for (int i = 0; i < 4; ++i) cs[i] += e[q][i];
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) sr += __shfl_xor_sync(0xffffffffu, sr, d);
+            if (lane == 0 && r < p.th) rs[r] = sr;
+        }
     }
 #pragma unroll
     for (int i = 0; i < 4; ++i) colp[warp][4 * lane + i] = cs[i];
@@ -94,7 +107,11 @@ struct CarryParams {
 };
 
 // Step 2a: row carries.  One CTA per band, one thread per row of the band.
-// Writes Lx for J in [j0, j1] (j1 inclusive: the carry into the next region).
+// Writes Lx for J in [j0, j1] (j1 inclusive: the carry into the next region);
+// the loads of RS are independent of the running sum, so batches of 8 are in
+// flight at once.  Lsum(J) = sum over the band's rows of Lx(J) = sum(Lb) +
+// the exclusive prefix over the region's chunks of the tile totals, and a tile
+// total is the last entry of its chunk-local column-sum prefix Bt (Step 1).
 template <typename T>
 __global__ void sat_carry_rows_kernel(const CarryParams p)
 {
@@ -106,39 +123,65 @@ __global__ void sat_carry_rows_kernel(const CarryParams p)
     const bool valid = r < p.th;
     const int64_t stride = int64_t(p.total_bands) * p.th;
     const int64_t idx = int64_t(gb) * p.th + r;
-    T L = (p.Lb && valid) ? reinterpret_cast<const T*>(p.Lb)[idx] : T(0);
+    const T* __restrict__ RS = reinterpret_cast<const T*>(p.RS);
+    T* __restrict__ Lx = reinterpret_cast<T*>(p.Lx);
+    const T L0 = (p.Lb && valid) ? reinterpret_cast<const T*>(p.Lb)[idx] : T(0);
+    const int jend = min(j1, p.nc);      // last Lx index written
+    if (valid) {
+        T L = L0;
+        constexpr int B = 8;
+        for (int J = j0; J <= jend; J += B) {
+            T v[B];
+#pragma unroll
+            for (int q = 0; q < B; ++q)
+                v[q] = (J + q < j1) ? RS[int64_t(J + q) * stride + idx] : T(0);
+#pragma unroll
+            for (int q = 0; q < B; ++q) {
+                if (J + q <= jend) Lx[int64_t(J + q) * stride + idx] = L;
+                L += v[q];
+            }
+        }
+    }
+    // sum over the band's rows of Lb
     __shared__ T red[32];
     const int warp = r >> 5, lane = r & 31, nw = (p.th + 31) / 32;
-    for (int J = j0; J <= j1 && J <= p.nc; ++J) {
-        if (valid) reinterpret_cast<T*>(p.Lx)[int64_t(J) * stride + idx] = L;
-        T s = L;
+    T s = valid ? L0 : T(0);
 #pragma unroll
-        for (int d = 16; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
-        if (lane == 0) red[warp] = s;
-        __syncthreads();
-        if (r == 0) {
-            T t = T(0);
-            for (int w = 0; w < nw; ++w) t += red[w];
-            reinterpret_cast<T*>(p.Lsum)[int64_t(gb) * (p.nc + 1) + J] = t;
+    for (int d = 16; d > 0; d >>= 1) s += __shfl_xor_sync(0xffffffffu, s, d);
+    if (lane == 0) red[warp] = s;
+    __syncthreads();
+    if (warp == 0) {
+        T base = T(0);
+        for (int w = 0; w < nw; ++w) base += red[w];
+        const int W = p.nc * TW;
+        const T* bt = reinterpret_cast<const T*>(p.Bt) + int64_t(gb) * W;
+        T* lsum = reinterpret_cast<T*>(p.Lsum) + int64_t(gb) * (p.nc + 1);
+        for (int J0 = j0; J0 <= jend; J0 += 32) {
+            const int J = J0 + lane;
+            const T tot = (J < j1) ? bt[int64_t(J) * TW + TW - 1] : T(0);
+            const T inc = warp_inclusive_scan(tot, lane);
+            if (J <= jend) lsum[J] = base + inc - tot;
+            base += __shfl_sync(0xffffffffu, inc, 31);
         }
-        __syncthreads();
-        if (J < j1 && valid) L += reinterpret_cast<const T*>(p.RS)[int64_t(J) * stride + idx];
     }
 }
 
-// Step 2b: SAT row above every region tile.  One thread per (image, column).
-// Walks down the region's tiles of the column's chunk:
+// Step 2b: SAT row above every region tile:
 //   Top(I+1) = Top(I) + Lsum(I, J) + Bt(I)[c]
 // starting from 0 at the matrix top, or -- for region B -- from the final SAT
-// row just above the region (already in `out`).
+// row just above the region (already in `out`).  Block = 32 columns x 8 band
+// groups: each thread sums its group's increments, an exclusive scan over the
+// 8 groups gives every group its starting Top, then each thread writes its
+// group's rows (loads independent of the running sum, 4 in flight).
 template <typename T>
-__global__ void sat_carry_top_kernel(const CarryParams p)
+__global__ void __launch_bounds__(256) sat_carry_top_kernel(const CarryParams p)
 {
-    const int64_t c = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    const int cx = threadIdx.x & 31, grp = threadIdx.x >> 5;
+    const int64_t c = int64_t(blockIdx.x) * 32 + cx;
     const int img = blockIdx.y;
     const int W = p.nc * TW;
-    if (c >= W) return;
-    const int J = int(c / TW);
+    const bool live = c < W;
+    const int J = live ? int(c / TW) : 0;
     // bands I of this image whose tile (I, J) is in the region: contiguous
     int i0 = -1, i1 = -1;
     for (int I = 0; I < p.nb; ++I) {
@@ -146,17 +189,48 @@ __global__ void sat_carry_top_kernel(const CarryParams p)
         region_range(p.region, p.tA, p.nb, p.nc, I, j0, j1);
         if (J >= j0 && J < j1) { if (i0 < 0) i0 = I; i1 = I + 1; }
     }
-    if (i0 < 0) return;
+    const bool any = live && i0 >= 0;
+    const int n = any ? i1 - i0 : 0;
+    const int per = (n + 7) / 8;
+    const int g0 = i0 + grp * per, g1 = min(i1, g0 + per);
+    const T* __restrict__ lsum = reinterpret_cast<const T*>(p.Lsum);
+    const T* __restrict__ bt = reinterpret_cast<const T*>(p.Bt);
+    T* __restrict__ topx = reinterpret_cast<T*>(p.TopX);
+    auto inc = [&](int I) {
+        const int gb = img * p.nb + I;
+        return lsum[int64_t(gb) * (p.nc + 1) + J] + bt[int64_t(gb) * W + c];
+    };
+    T part = T(0);
+    if (any) {
+        int I = g0;
+        for (; I + 4 <= g1; I += 4) {
+            const T a = inc(I), b = inc(I + 1), d = inc(I + 2), e = inc(I + 3);
+            part += (a + b) + (d + e);
+        }
+        for (; I < g1; ++I) part += inc(I);
+    }
+    __shared__ T sums[8][32];
+    sums[grp][cx] = part;
+    __syncthreads();
+    if (!any) return;
     T top = T(0);
     if (i0 > 0 && c < p.cols) {
         const T* o = reinterpret_cast<const T*>(p.out) + int64_t(img) * p.rows * p.cols;
         top = o[(int64_t(i0) * p.th - 1) * p.cols + c];
     }
-    for (int I = i0; I < i1; ++I) {
-        const int gb = img * p.nb + I;
-        reinterpret_cast<T*>(p.TopX)[int64_t(gb) * W + c] = top;
-        top += reinterpret_cast<const T*>(p.Lsum)[int64_t(gb) * (p.nc + 1) + J]
-             + reinterpret_cast<const T*>(p.Bt)[int64_t(gb) * W + c];
+    for (int g = 0; g < grp; ++g) top += sums[g][cx];
+    int I = g0;
+    for (; I + 4 <= g1; I += 4) {
+        const T a = inc(I), b = inc(I + 1), d = inc(I + 2), e = inc(I + 3);
+        const int64_t gb = int64_t(img) * p.nb + I;
+        topx[gb * W + c] = top; top += a;
+        topx[(gb + 1) * W + c] = top; top += b;
+        topx[(gb + 2) * W + c] = top; top += d;
+        topx[(gb + 3) * W + c] = top; top += e;
+    }
+    for (; I < g1; ++I) {
+        topx[(int64_t(img) * p.nb + I) * W + c] = top;
+        top += inc(I);
     }
 }
 
