@@ -97,7 +97,10 @@ typedef struct sat_options {
     double r;            /* SAT_1PLUSR_R1W: target fraction of tiles done by 2R1W
                             (0..1, default 0.25); the realised value is the tile
                             count ratio, see sat_last_r_effective() */
-    int tile_rows;       /* band height TH in {16, 32, 48, 64, 128}; 0 = automatic */
+    int tile_rows;       /* band height TH in {16, 32, 48, 64, 112, 128} (float64:
+                            16, 32, 48, 64); 0 = automatic (DESIGN.md Sec. 5:
+                            1R1W takes 128 once its bands fill half the SMs,
+                            else 32 from 1536 rows, else 16) */
     int force_generic;   /* 1 = use the non-TMA load/store path (tests) */
     int jitter;          /* debug: random delay (ns) before descriptor
                             publication, to stress the look-back; 0 = off */

@@ -682,6 +682,17 @@ int choose_tA(int nb, int nc, double r, double& r_eff) {
 // ------------------------------------------------------------------ 4R4W / 4R1W (Table II columns)
 template <typename T>
 int transpose_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols, cudaStream_t st) {
+    const uintptr_t al = 2 * sizeof(T) - 1;
+    if (rows % 2 == 0 && cols % 2 == 0 && !(reinterpret_cast<uintptr_t>(in) & al) &&
+        !(reinterpret_cast<uintptr_t>(out) & al) && !getenv("SAT_TRANSPOSE32")) {
+        const int64_t ntr = (rows + 63) / 64;
+        const dim3 grid(unsigned((cols + 63) / 64), unsigned(std::min<int64_t>(ntr, 65535)), unsigned(batch));
+        sat_transpose64_kernel<T><<<grid, 256, 0, st>>>(static_cast<const T*>(in), static_cast<T*>(out),
+                                                        rows, cols);
+        CUDA_TRY(cudaGetLastError());
+        ++t_launches;
+        return SAT_OK;
+    }
     const int64_t ntr = (rows + 31) / 32;
     const dim3 grid(unsigned((cols + 31) / 32), unsigned(std::min<int64_t>(ntr, 65535)), unsigned(batch));
     sat_transpose_kernel<T><<<grid, dim3(32, 8), 0, st>>>(static_cast<const T*>(in), static_cast<T*>(out),

@@ -48,6 +48,51 @@ __global__ void __launch_bounds__(256) sat_transpose_kernel(const T* __restrict_
     }
 }
 
+// Wide transpose: 64 x 64 tiles, two consecutive elements per lane on both
+// sides (8-B accesses for 4-byte types, 16-B for float64), so every warp reads
+// and writes 256-B (512-B) row segments; smem rows padded by one element (at
+// most a 2-way bank conflict on the transposed read).  Requires even rows and
+// cols and 2-element-aligned pointers (the host falls back to the 32 x 32
+// kernel otherwise).  Measured 16384^2 int32: see DESIGN.md Sec. 5.
+template <typename T>
+struct alignas(2 * sizeof(T)) Pair { T a, b; };
+
+template <typename T>
+__global__ void __launch_bounds__(256) sat_transpose64_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                              int64_t rows, int64_t cols) {
+    __shared__ T tile[64][65];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t img = blockIdx.z;
+    const T* src = in + img * rows * cols;
+    T* dst = out + img * rows * cols;
+    const int64_t ntr = (rows + 63) / 64;
+    const int64_t c0 = int64_t(blockIdx.x) * 64;
+    for (int64_t tr = blockIdx.y; tr < ntr; tr += gridDim.y) {
+        const int64_t r0 = tr * 64;
+        Pair<T> v[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const int64_t r = r0 + warp + 8 * k, c = c0 + 2 * lane;
+            v[k] = (r < rows && c < cols) ? *reinterpret_cast<const Pair<T>*>(src + r * cols + c)
+                                          : Pair<T>{T(0), T(0)};
+        }
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            tile[warp + 8 * k][2 * lane] = v[k].a;
+            tile[warp + 8 * k][2 * lane + 1] = v[k].b;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            const int cc = warp + 8 * k;                  // output row = input column c0 + cc
+            const int64_t c = c0 + cc, r = r0 + 2 * lane;
+            if (c < cols && r < rows)
+                *reinterpret_cast<Pair<T>*>(dst + c * rows + r) = Pair<T>{tile[2 * lane][cc], tile[2 * lane + 1][cc]};
+        }
+        __syncthreads();
+    }
+}
+
 // One stage of 4R1W: every element (i, t - i) of anti-diagonal t, i in
 // [i0, i0 + cnt).  Formula (1) evaluated left to right,
 // ((a + b_up) + b_left) - b_diag; uint32 wraps, floating point rounds per add.
