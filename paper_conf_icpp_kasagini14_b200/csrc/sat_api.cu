@@ -489,7 +489,8 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.nb = int((j.rows + j.th - 1) / j.th);
     p.nc = int((j.cols + TW - 1) / TW);
     p.total_bands = int(j.batch * p.nb);
-    p.total_units = p.tile_units ? (long long)p.total_bands * p.nc : p.total_bands;
+    p.total_units = p.tile_units ? (long long)p.total_bands * ((p.nc + p.tile_units - 1) / p.tile_units)
+                                 : p.total_bands;
     // Clusters of 8 bands that pass the vertical carry through DSMEM (DESIGN.md
     // Sec. 4.5) are correct but measured slower than the plain look-back, so
     // they are opt-in (SAT_CLUSTER=8) for plain 1R1W on the TMA path.
@@ -643,8 +644,12 @@ int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, cons
     // Step 3: re-read, add carries, tile SAT, write (tile tickets, external carries)
     BandParams p = base_params();
     p.top_src = TOP_EXTERNAL;
-    p.tile_units = 0;
-    if (const char* e = getenv("SAT_TILE_UNITS")) p.tile_units = atoi(e) != 0;
+    // units of K chunks of a band (external carries make every range
+    // independent): whole bands for the full matrix up to 64 chunks, 8-chunk
+    // ranges above (16384^2 2R1W 0.657 -> 0.625 ms); 16-chunk ranges for the
+    // (1+r)R1W triangles, whose top bands are long (16384^2 0.952 -> 0.705 ms)
+    p.tile_units = region == REG_ALL ? (c.nc >= 64 ? 8 : 0) : 16;
+    if (const char* e = getenv("SAT_TILE_UNITS")) p.tile_units = std::max(0, atoi(e));
     p.region = region;
     p.tA = tA;
     p.Lx = ws.lx.p;

@@ -435,11 +435,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             gb = im * p.nb + cb * CL + int(crank);      // may exceed the image: a virtual band
             j0 = 0; j1 = p.nc;
         } else if (p.tile_units) {
-            gb = int(unit / p.nc);
-            const int J = int(unit % p.nc);
+            // ranges of tile_units chunks of a band's region (external
+            // carries: the row carry at the range start comes from Lx)
+            const int per = (p.nc + p.tile_units - 1) / p.tile_units;
+            gb = int(unit / per);
+            const int sr = int(unit % per);
             int r0, r1;
             region_range(p.region, p.tA, p.nb, p.nc, gb % p.nb, r0, r1);
-            j0 = J; j1 = (J >= r0 && J < r1) ? J + 1 : J;
+            j0 = min(r1, r0 + sr * p.tile_units);
+            j1 = min(r1, j0 + p.tile_units);
         } else if (p.nseg > 1) {
             seg = int(unit / p.total_bands);
             gb = int(unit - (long long)seg * p.total_bands);

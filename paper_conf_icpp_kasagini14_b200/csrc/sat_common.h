@@ -44,7 +44,7 @@ struct BandParams {
     int nc;                    // chunks per band = ceil(cols / TW)
     int total_bands;           // batch * nb
     long long total_units;     // bands (band units) or bands*nc (tile units)
-    int tile_units;            // 1: one ticket = one tile (external carries)
+    int tile_units;            // K > 0: one ticket = K consecutive tiles of a band (external carries); 0 = whole bands
     int cluster;               // CTAs per cluster (1, or 8: one ticket = 8 bands)
     int big;                   // 1: one CTA per SM with a 2x ring of 1-KB row segments (TH 64)
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
