@@ -62,6 +62,8 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
+constexpr int kMaxDev = 64;
+
 struct DevInfo {
     int sms = 0;
     int smem_optin = 0;
@@ -244,7 +246,7 @@ constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM co
 // CTAs per SM of a configuration (for wave counts before launch)
 int ctas_per_sm(int dtype, int th, bool big) {
     if (dtype == SAT_FLOAT64) return th == 16 ? 2 : 1;
-    return (th == 128 || th == 112 || big) ? 1 : 2;
+    return (th >= 112 || big) ? 1 : 2;
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
@@ -255,18 +257,25 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
     auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB, LBW, TI>;
     const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL, TI>::total;
     const int threads = (W + NCW + 1) * 32;
-    static int configured = 0;   // per instantiation (per process; devices share the attribute)
-    if (!configured) {
+    // per instantiation and device: attributes set once, resources queried once
+    // (a per-call cudaFuncGetAttributes was a visible part of the ~15 us host
+    // cost of a small call)
+    static int configured[kMaxDev] = {};
+    static cudaFuncAttributes fa_dev[kMaxDev];
+    int dev = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    if (dev < 0 || dev >= kMaxDev) return fail(SAT_ERR_CUDA, "device ordinal out of range");
+    if (!configured[dev]) {
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
         CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
                                       int(cudaSharedmemCarveoutMaxShared)));
-        configured = 1;
+        CUDA_TRY(cudaFuncGetAttributes(&fa_dev[dev], kern));
+        configured[dev] = 1;
     }
     // Resident CTAs per SM, from the kernel's own resources.  (The runtime's
     // occupancy query reports 1 for kernels that allocate tensor memory; two
     // CTAs of ours fit: TC::alloc <= 256 columns of the SM's 512.)
-    cudaFuncAttributes fa;
-    CUDA_TRY(cudaFuncGetAttributes(&fa, kern));
+    const cudaFuncAttributes& fa = fa_dev[dev];
     const int warps = threads / 32;
     const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
     int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
