@@ -249,7 +249,20 @@ sat_colsum_partial_kernel(const T* __restrict__ in, T* __restrict__ part,
     if (r1 > rows) r1 = rows;
     const bool vec = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) && (c + 3 < cols);
     T cs[4] = {T(0), T(0), T(0), T(0)};
-    for (int64_t r = r0 + warp; r < r1; r += 8) {
+    int64_t r = r0 + warp;
+    if (vec) {
+        // 8 independent 16-B loads in flight per lane (the sums wait, the loads do not)
+        for (; r + 56 < r1; r += 64) {
+            T e[8][4];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) ldg4<T>(in + (r + 8 * q) * cols + c, e[q]);
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+#pragma unroll
+                for (int i = 0; i < 4; ++i) cs[i] += e[q][i];
+        }
+    }
+    for (; r < r1; r += 8) {
         if (vec) {
             T e[4];
             ldg4<T>(in + r * cols + c, e);
