@@ -461,7 +461,7 @@ int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dty
     // 12288^2 0.254 vs 0.313, 14336^2 0.327 vs 0.417; 16K^2+: 5.3-5.4 TB/s vs
     // 5.0 for TH 64); below that TH 32 from 1536 rows (2048^2-8192^2: 15-25 %
     // faster than TH 16), else TH 16.
-    if (variant == SAT_1R1W) {
+    if (variant == SAT_1R1W || variant == SAT_1PLUSR_R1W) {   // (1+r): its band C is 1R1W
         const long long b128 = batch * ((rows + 127) / 128);
         if (b128 * 2 >= di.sms) return 128;
         return rows * batch >= 1536 ? 32 : 16;
@@ -824,6 +824,12 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             double r_eff = 0;
             const int tA = choose_tA(c.nb, c.nc, o.r, r_eff);
             t_r = r_eff;
+            if (tA == 0) {
+                // r_eff = 0: both triangles are empty -- plain 1R1W (no empty
+                // Step 1/2 launches, band segments allowed)
+                BandParams p = base_params();
+                return run_band(j, MODE_SAT, in, out, p);
+            }
             // (A) 2R1W on the top-left triangle; its Step 2 also leaves the
             // row carry into (C) in Lx.
             SAT_TRY(run_2r1w_region(j, c, REG_A, tA, in, out, nullptr));
