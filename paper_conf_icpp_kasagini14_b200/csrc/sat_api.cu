@@ -1109,15 +1109,20 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     // 2. four SAT reads per output element
     const dim3 grid(unsigned((cols + 255) / 256), unsigned(std::min<int64_t>((rows + BOX_RB - 1) / BOX_RB, 65535)),
                     unsigned(batch));
-    if (sdt == SAT_INT32)
-        sat_box_kernel<uint32_t, int32_t><<<grid, 256, 0, st>>>(static_cast<const uint32_t*>(ws->box.p),
-                                                                static_cast<int32_t*>(out), rows, cols, rr, rc, 0);
-    else if (out_dtype == SAT_FLOAT32)
-        sat_box_kernel<double, float><<<grid, 256, 0, st>>>(static_cast<const double*>(ws->box.p),
-                                                           static_cast<float*>(out), rows, cols, rr, rc, normalize);
-    else
-        sat_box_kernel<double, double><<<grid, 256, 0, st>>>(static_cast<const double*>(ws->box.p),
-                                                            static_cast<double*>(out), rows, cols, rr, rc, normalize);
+    auto box = [&](auto idx) {
+        using I = decltype(idx);
+        if (sdt == SAT_INT32)
+            sat_box_kernel<uint32_t, int32_t, I><<<grid, 256, 0, st>>>(
+                static_cast<const uint32_t*>(ws->box.p), static_cast<int32_t*>(out), I(rows), I(cols), rr, rc, 0);
+        else if (out_dtype == SAT_FLOAT32)
+            sat_box_kernel<double, float, I><<<grid, 256, 0, st>>>(
+                static_cast<const double*>(ws->box.p), static_cast<float*>(out), I(rows), I(cols), rr, rc, normalize);
+        else
+            sat_box_kernel<double, double, I><<<grid, 256, 0, st>>>(
+                static_cast<const double*>(ws->box.p), static_cast<double*>(out), I(rows), I(cols), rr, rc, normalize);
+    };
+    if (rows * cols < (int64_t(1) << 31)) box(int32_t(0));
+    else box(int64_t(0));
     CUDA_TRY(cudaGetLastError());
     t_launches = launches + 1;
     return SAT_OK;

@@ -35,41 +35,49 @@ __device__ __forceinline__ TO box_out(T v) {
 // grid: (ceil(cols / 256), min(ceil(rows / BOX_RB), 65535), batch); block 256.
 // A thread owns one column and BOX_RB consecutive rows per iteration and
 // issues all 4*BOX_RB SAT loads before any arithmetic (memory-level
-// parallelism: one row per thread left the kernel latency-bound).
+// parallelism: one row per thread left the kernel latency-bound).  IDX is the
+// in-image index type: int32 when rows*cols < 2^31 (the kernel was
+// instruction-bound on 64-bit index arithmetic: ncu SM throughput 65 %, DRAM
+// 23 %); the image base is a 64-bit pointer either way.
 constexpr int BOX_RB = 8;
-template <typename T, typename TO>
+template <typename T, typename TO, typename IDX>
 __global__ void __launch_bounds__(256) sat_box_kernel(const T* __restrict__ S, TO* __restrict__ out,
-                                                      int64_t rows, int64_t cols, int rr, int rc,
+                                                      IDX rows, IDX cols, int rr, int rc,
                                                       int normalize) {
-    const int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    const IDX j = IDX(blockIdx.x) * IDX(blockDim.x) + IDX(threadIdx.x);
     if (j >= cols) return;
     const int64_t img = blockIdx.z;
-    const T* Si = S + img * rows * cols;
-    TO* Oi = out + img * rows * cols;
-    const int64_t j1 = j - rc > 0 ? j - rc : 0;
-    const int64_t j2 = j + rc < cols - 1 ? j + rc : cols - 1;
-    for (int64_t i0 = int64_t(blockIdx.y) * BOX_RB; i0 < rows; i0 += int64_t(gridDim.y) * BOX_RB) {
+    const T* Si = S + img * int64_t(rows) * int64_t(cols);
+    TO* Oi = out + img * int64_t(rows) * int64_t(cols);
+    const IDX j1 = j - rc > 0 ? j - rc : IDX(0);
+    const IDX j2 = j + rc < cols - 1 ? j + rc : cols - 1;
+    const bool left = j1 > 0;
+    const IDX jl = left ? j1 - 1 : IDX(0);
+    const IDX wc = j2 - j1 + 1;
+    for (IDX i0 = IDX(blockIdx.y) * BOX_RB; i0 < rows; i0 += IDX(gridDim.y) * BOX_RB) {
         T a[BOX_RB], b[BOX_RB], c[BOX_RB], d[BOX_RB];
 #pragma unroll
         for (int k = 0; k < BOX_RB; ++k) {
-            const int64_t i = i0 + k < rows ? i0 + k : rows - 1;
-            const int64_t i1 = i - rr > 0 ? i - rr : 0;
-            const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
-            a[k] = Si[i2 * cols + j2];
-            b[k] = i1 > 0 ? Si[(i1 - 1) * cols + j2] : T(0);
-            c[k] = j1 > 0 ? Si[i2 * cols + j1 - 1] : T(0);
-            d[k] = (i1 > 0 && j1 > 0) ? Si[(i1 - 1) * cols + j1 - 1] : T(0);
+            const IDX i = i0 + k < rows ? i0 + k : rows - 1;
+            const IDX i1 = i - rr > 0 ? i - rr : IDX(0);
+            const IDX i2 = i + rr < rows - 1 ? i + rr : rows - 1;
+            const T* s2 = Si + i2 * cols;
+            const T* s1 = Si + (i1 > 0 ? i1 - 1 : IDX(0)) * cols;
+            a[k] = s2[j2];
+            b[k] = i1 > 0 ? s1[j2] : T(0);
+            c[k] = left ? s2[jl] : T(0);
+            d[k] = (i1 > 0 && left) ? s1[jl] : T(0);
         }
 #pragma unroll
         for (int k = 0; k < BOX_RB; ++k) {
-            const int64_t i = i0 + k;
+            const IDX i = i0 + k;
             if (i >= rows) break;
             T v = ((a[k] - b[k]) - c[k]) + d[k];
             if constexpr (!std::is_same<T, uint32_t>::value) {
                 if (normalize) {
-                    const int64_t i1 = i - rr > 0 ? i - rr : 0;
-                    const int64_t i2 = i + rr < rows - 1 ? i + rr : rows - 1;
-                    v = v / T((i2 - i1 + 1) * (j2 - j1 + 1));
+                    const IDX i1 = i - rr > 0 ? i - rr : IDX(0);
+                    const IDX i2 = i + rr < rows - 1 ? i + rr : rows - 1;
+                    v = v / T(int64_t(i2 - i1 + 1) * int64_t(wc));
                 }
             }
             Oi[i * cols + j] = box_out<TO>(v);
