@@ -410,7 +410,11 @@ template <typename T, typename TI, bool TMA>
 int launch_band_widen(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
                       const DevInfo& di, cudaStream_t st, int& grid) {
     if constexpr (sizeof(TI) == 1) {
-        if (th == 128) return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, 0, TI>(p, ti, to, di, st, grid);
+        if (th == 128) {
+            if (getenv("SAT_DEBUG_U8LBW4"))
+                return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, 0, TI>(p, ti, to, di, st, grid);
+            return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, kLbw128, TI>(p, ti, to, di, st, grid);
+        }
         if (th == 64) return launch_band_t<T, 8, 8, 6, 4, 1, 4, 1, MODE_SAT, TMA, 2, 1, 0, TI>(p, ti, to, di, st, grid);
         return fail(SAT_ERR_INVALID, "uint8 input: tile_rows must be 64 or 128");
     } else {
