@@ -110,6 +110,11 @@ typedef struct sat_options {
 /* Fill *opt with defaults (r = 0.25, automatic tile, TMA when eligible). */
 void sat_options_init(sat_options *opt);
 
+/* Stream capture (CUDA graphs) is refused with SAT_ERR_UNSUPPORTED by every
+ * entry point that launches the band kernel: its look-back tags and ticket
+ * base are assigned per launch on the host, so a replayed graph would reuse
+ * them. */
+
 /* out = SAT(in) for one rows x cols matrix.  variant: sat_variant. */
 int sat_compute(const void *in, void *out, int64_t rows, int64_t cols,
                 int dtype, int variant, void *stream);

@@ -494,6 +494,15 @@ struct Job {
 
 // One band-kernel launch with ticket/tag bookkeeping.
 int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
+    // The ticket base and the descriptor tags come from a host-side counter
+    // advanced per launch; a captured launch replayed from a CUDA graph would
+    // reuse them and could accept its previous replay's descriptors.  Refuse
+    // capture instead of risking a silently wrong SAT.
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    CUDA_TRY(cudaStreamIsCapturing(j.st, &cap));
+    if (cap != cudaStreamCaptureStatusNone)
+        return fail(SAT_ERR_UNSUPPORTED, "stream capture is not supported: the look-back tags are "
+                                         "assigned per launch on the host (a graph replay would reuse them)");
     p.in = in;
     p.out = out;
     p.rows = j.rows;

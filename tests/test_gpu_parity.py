@@ -515,3 +515,18 @@ def test_fused_exchange_single_device(libsat, P, dtype):
             assert np.array_equal(got, ref), f"call {it}"
     for e in exs:
         e.close()
+
+
+def test_stream_capture_refused(libsat):
+    """A captured launch would replay with the same look-back tags (host-side
+    ticket base), so capture is refused loudly rather than producing a graph
+    that can return a wrong SAT on replay."""
+    x = dev(gen(512, 1024, "int32", seed=1))
+    y = libsat.sat(x)                      # warm: workspace exists
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with pytest.raises(Exception, match="capture"):
+        with torch.cuda.graph(g, stream=s):
+            libsat.sat(x, out=y)
+    torch.cuda.synchronize()
+    check(libsat.sat(x), oracle.sat(x.cpu().numpy()), "int32")
