@@ -36,6 +36,7 @@ thread_local int t_th = 0;
 thread_local int t_grid = 0;
 thread_local double t_r = 0.0;
 thread_local unsigned long long* t_trace = nullptr;
+thread_local bool t_capture = false;   // the current call's stream is being captured
 static unsigned int* g_diag_dev = nullptr;   // sat_debug_diag_enable (device view)
 
 int fail(int code, const std::string& msg) {
@@ -105,6 +106,11 @@ struct Buf {
 
 int ensure(Buf& b, size_t bytes, bool zero) {
     if (b.bytes >= bytes && b.p) return SAT_OK;
+    // a captured call cannot allocate (cudaMalloc / cudaMemset would break
+    // the capture): the workspace must have been sized by an eager call
+    if (t_capture)
+        return fail(SAT_ERR_UNSUPPORTED, "stream capture needs a warm workspace: run the same call once "
+                                         "on this stream before capturing it");
     if (b.p) { cudaFree(b.p); b.p = nullptr; b.bytes = 0; }
     size_t want = std::max<size_t>(bytes, 256);
     if (cudaMalloc(&b.p, want) != cudaSuccess) {
@@ -116,13 +122,20 @@ int ensure(Buf& b, size_t bytes, bool zero) {
     return SAT_OK;
 }
 
-constexpr unsigned long long kTagSpace = 1ull << 30;
+// look-back tags are 30 bits (band_tag); SAT_TAG_SPACE (tests only) shrinks
+// the space so the reset paths run
+unsigned long long tag_space() {
+    const char* e = getenv("SAT_TAG_SPACE");
+    const unsigned long long v = e ? strtoull(e, nullptr, 10) : 0ull;
+    return v > 0 && v < (1ull << 30) ? v : (1ull << 30);
+}
 
 struct Workspace {
     Buf desc;                 // look-back descriptors (zeroed when (re)allocated)
     Buf lseg;                 // band-segment row carries (zeroed when (re)allocated)
-    Buf ticket;               // unsigned long long counter
+    Buf ticket;               // [0] ticket counter, [1] device base, [2] reset flag (unsigned long long)
     unsigned long long next_base = 0;
+    bool dev_epoch = false;   // once captured: every launch takes its base from the device (Sec. 4)
     Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
     Buf tr;                   // 4R4W transposed copy
     Buf box;                  // box filter: the SAT it reads
@@ -137,6 +150,9 @@ std::map<std::pair<int, void*>, Workspace*> g_ws;
 
 int get_ws(int dev, cudaStream_t st, Workspace*& ws) {
     std::lock_guard<std::mutex> lk(g_mu);
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    CUDA_TRY(cudaStreamIsCapturing(st, &cap));
+    t_capture = (cap != cudaStreamCaptureStatusNone);
     Workspace*& w = g_ws[{dev, reinterpret_cast<void*>(st)}];
     if (!w) w = new Workspace();
     ws = w;
@@ -492,17 +508,38 @@ struct Job {
     cudaStream_t st;
 };
 
+// Device-side ticket base (graph capture): the ticket counter ends every band
+// launch at base + units + takers, the next launch's base; reset it (and
+// request a descriptor clear) when the tag space would run out.
+__global__ void sat_epoch_kernel(unsigned long long* tk, unsigned long long worst, unsigned long long space) {
+    if (threadIdx.x != 0) return;
+    const unsigned long long t = tk[0];
+    const bool reset = t + worst >= space;
+    if (reset) tk[0] = 0;
+    tk[1] = reset ? 0 : t;
+    tk[2] = reset ? 1 : 0;
+}
+
+__global__ void sat_epoch_clear_kernel(const unsigned long long* flag, uint4* a, size_t na, uint4* b, size_t nb) {
+    if (!*flag) return;
+    const uint4 z = make_uint4(0, 0, 0, 0);
+    for (size_t i = size_t(blockIdx.x) * blockDim.x + threadIdx.x; i < na + nb; i += size_t(gridDim.x) * blockDim.x) {
+        if (i < na) a[i] = z; else b[i - na] = z;
+    }
+}
+
 // One band-kernel launch with ticket/tag bookkeeping.
 int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     // The ticket base and the descriptor tags come from a host-side counter
-    // advanced per launch; a captured launch replayed from a CUDA graph would
-    // reuse them and could accept its previous replay's descriptors.  Refuse
-    // capture instead of risking a silently wrong SAT.
+    // advanced per launch.  A captured launch replayed from a CUDA graph would
+    // reuse a host value, so under capture (and on this workspace from then
+    // on, since replays advance the device ticket behind the host's back) the
+    // base is taken on the device: sat_epoch_kernel reads the ticket counter
+    // (it ends every launch at the next launch's base) right before the band
+    // kernel, on the same stream.
     cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
     CUDA_TRY(cudaStreamIsCapturing(j.st, &cap));
-    if (cap != cudaStreamCaptureStatusNone)
-        return fail(SAT_ERR_UNSUPPORTED, "stream capture is not supported: the look-back tags are "
-                                         "assigned per launch on the host (a graph replay would reuse them)");
+    if (cap != cudaStreamCaptureStatusNone) j.ws->dev_epoch = true;
     p.in = in;
     p.out = out;
     p.rows = j.rows;
@@ -566,12 +603,25 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t) * (esize(j.dtype) / 4);
         SAT_TRY(ensure(ws.desc, need, true));
     }
-    SAT_TRY(ensure(ws.ticket, sizeof(unsigned long long), true));
+    SAT_TRY(ensure(ws.ticket, 4 * sizeof(unsigned long long), true));
     if (p.nseg > 1)
         SAT_TRY(ensure(ws.lseg, size_t(p.total_bands) * j.th * sizeof(uint64_t) * (esize(j.dtype) / 4), true));
     const unsigned long long units = (unsigned long long)p.total_units;
     const unsigned long long worst = units + 4096ull * 64ull;   // units + max grid
-    if (ws.next_base + worst >= kTagSpace) {
+    p.base_dev = nullptr;
+    if (ws.dev_epoch) {
+        unsigned long long* tk = static_cast<unsigned long long*>(ws.ticket.p);
+        sat_epoch_kernel<<<1, 32, 0, j.st>>>(tk, worst, tag_space());
+        CUDA_TRY(cudaGetLastError());
+        const size_t dw = ws.desc.p ? ws.desc.bytes / 16 : 0, lw = ws.lseg.p ? ws.lseg.bytes / 16 : 0;
+        if (dw + lw) {
+            sat_epoch_clear_kernel<<<2 * j.di->sms, 256, 0, j.st>>>(tk + 2, static_cast<uint4*>(ws.desc.p), dw,
+                                                                    static_cast<uint4*>(ws.lseg.p), lw);
+            CUDA_TRY(cudaGetLastError());
+        }
+        p.base_dev = tk + 1;
+        t_launches += dw + lw ? 2 : 1;
+    } else if (ws.next_base + worst >= tag_space()) {
         // tag space exhausted: clear descriptors and the counter (rare)
         if (ws.desc.p) CUDA_TRY(cudaMemsetAsync(ws.desc.p, 0, ws.desc.bytes, j.st));
         if (ws.lseg.p) CUDA_TRY(cudaMemsetAsync(ws.lseg.p, 0, ws.lseg.bytes, j.st));

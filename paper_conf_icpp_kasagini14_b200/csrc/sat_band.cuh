@@ -339,6 +339,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
     uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 2);
     const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
+    // ticket/tag base: the host's counter, or (CUDA-graph capture, DESIGN.md
+    // Sec. 4) the value sat_epoch_kernel wrote just before this launch
+    const unsigned long long kbase = p.base_dev ? __ldcg(p.base_dev) : p.base;
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -389,7 +392,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         if constexpr (CL > 1) {
             // one ticket per cluster: CL consecutive bands, rank r takes band CL*u + r
             if (crank == 0 && threadIdx.x == 0) {
-                const unsigned long long u = atomicAdd(p.ticket, 1ull) - p.base;
+                const unsigned long long u = atomicAdd(p.ticket, 1ull) - kbase;
                 for (uint32_t r = 0; r < CL; ++r) st_cluster_u64(mapa(smem_u32(s_unit), r), u);
             }
             cluster_sync_all();
@@ -402,7 +405,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if (warp == PW) {
                 if (lane == 0) {
                     if (useq >= 2) mbar_wait(&uempty[qs], qph ^ 1u);   // every warp read unit useq-2
-                    s_unit[qs] = (long long)(atomicAdd(p.ticket, 1ull) - p.base);
+                    s_unit[qs] = (long long)(atomicAdd(p.ticket, 1ull) - kbase);
                     mbar_arrive(&ufull[qs]);
                 }
                 __syncwarp();
@@ -474,7 +477,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if (seg > 0) {
                 // row carry from segment seg-1 of this band (an earlier ticket,
                 // normally long finished): lane r < R polls row rbase + r
-                const uint32_t want = band_tag(p.base, (seg - 1) * p.total_bands + gb) | 3u;
+                const uint32_t want = band_tag(kbase, (seg - 1) * p.total_bands + gb) | 3u;
                 const bool mine = lane < R * NWE;        // word `lane` of this warp's rows
                 const uint64_t* q = p.Lseg + (int64_t(gb) * TH + rbase) * NWE + (mine ? lane : 0);
                 uint64_t wv;
@@ -625,7 +628,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 uint32_t mine = wl[0];
 #pragma unroll
                 for (int k = 1; k < R * NWE; ++k) if (lane == k) mine = wl[k];
-                const uint64_t w = (uint64_t(band_tag(p.base, seg * p.total_bands + gb) | 3u) << 32) | mine;
+                const uint64_t w = (uint64_t(band_tag(kbase, seg * p.total_bands + gb) | 3u) << 32) | mine;
                 asm volatile("st.relaxed.gpu.global.b64 [%0], %1;"
                              :: "l"(p.Lseg + (int64_t(gb) * TH + rbase) * NWE + lane), "l"(w) : "memory");
             }
@@ -648,7 +651,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const int cw = warp - CW;
                 const int grp = cw / NS;
                 const int cl = (cw % NS) * (TW / NS) + lane * CPL;   // column within the chunk
-                const uint32_t tagbase = band_tag(p.base, gb);
+                const uint32_t tagbase = band_tag(kbase, gb);
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
                 const T* gout = reinterpret_cast<const T*>(p.out) + int64_t(img) * img_elems;
@@ -721,7 +724,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                                 pend = 0;
                                 break;
                             }
-                            const uint32_t tk = band_tag(p.base, gidx - (idx - b2));
+                            const uint32_t tk = band_tag(kbase, gidx - (idx - b2));
                             bool ready = true;
 #pragma unroll
                             for (int i = 0; i < NW; ++i) {
@@ -774,7 +777,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         const int upi = (p.nb + CL - 1) / CL;
                         const bool pubc = cb + 1 < upi;
                         uint64_t* myc = p.desc + int64_t(gcb) * desc_w + c0;
-                        const uint32_t ctag = band_tag(p.base, gcb);
+                        const uint32_t ctag = band_tag(kbase, gcb);
                         T Sp[CPL] = {};
                         if (crank + 1 < CL) {
                             if (it >= uint32_t(XS)) mbar_wait_cluster(&aggfree[x], ph ^ 1u);

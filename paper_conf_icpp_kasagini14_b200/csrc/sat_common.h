@@ -50,6 +50,7 @@ struct BandParams {
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)
+    const unsigned long long* base_dev;   // nullable: read the base from device memory (graph capture)
     const void* seed;          // [cols] SAT row above band 0 of image 0, nullable
     int seed_kind;             // SEED_NONE or SEED_SATROW
     int top_src;               // TopSrc

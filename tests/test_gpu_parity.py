@@ -517,17 +517,69 @@ def test_fused_exchange_single_device(libsat, P, dtype):
         e.close()
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("shape,dtype", [((512, 1024), "int32"), ((1000, 3000), "float32"),
+                                         ((4096, 4096), "int32")])
+def test_cuda_graph_replay(libsat, variant, shape, dtype):
+    """Captured SAT calls replay correctly: the look-back ticket base comes
+    from the device, so every replay, and every eager call
+    on the same stream after it, sees fresh tags.  New input contents are
+    copied into the captured buffer between replays."""
+    n, m = shape
+    x = dev(gen(n, m, dtype, seed=1))
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        y = libsat.sat(x, variant=variant)          # warm: sizes the workspace of stream s
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.sat(x, variant=variant, out=y)
+    for it in range(4):
+        host = gen(n, m, dtype, seed=10 + it)
+        x.copy_(dev(host))
+        g.replay()
+        torch.cuda.synchronize()
+        check(y.cpu().numpy(), oracle.sat(host), dtype)
+        with torch.cuda.stream(s):                  # eager call between replays
+            z = libsat.sat(x, variant=variant)
+        s.synchronize()
+        check(z.cpu().numpy(), oracle.sat(host), dtype)
+
+
+def test_cuda_graph_tag_reset(libsat, monkeypatch):
+    """A tiny tag space (SAT_TAG_SPACE) forces the device-side reset in
+    sat_epoch_kernel (ticket to 0, descriptors cleared) during replays, and
+    the host-side reset on eager calls."""
+    monkeypatch.setenv("SAT_TAG_SPACE", "300000")
+    x = dev(gen(2048, 2048, "int32", seed=3))
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        y = libsat.sat(x)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.sat(x, out=y)
+    for it in range(6):
+        host = gen(2048, 2048, "int32", seed=20 + it)
+        x.copy_(dev(host))
+        g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(y.cpu().numpy(), oracle.sat(host)), f"replay {it}"
+    host = gen(2048, 2048, "int32", seed=40)
+    x2 = dev(host)
+    for it in range(3):
+        assert np.array_equal(libsat.sat(x2).cpu().numpy(), oracle.sat(host)), f"eager {it}"
+
+
 @pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")
-def test_stream_capture_refused(libsat):
-    """A captured launch would replay with the same look-back tags (host-side
-    ticket base), so capture is refused loudly rather than producing a graph
-    that can return a wrong SAT on replay."""
-    x = dev(gen(512, 1024, "int32", seed=1))
-    y = libsat.sat(x)                      # warm: workspace exists
+def test_capture_cold_workspace_refused(libsat):
+    """Capturing on a stream whose workspace was never sized fails loudly
+    (a captured call cannot allocate)."""
+    x = dev(gen(640, 1280, "int32", seed=5))
     s = torch.cuda.Stream()
     g = torch.cuda.CUDAGraph()
-    with pytest.raises(Exception, match="capture"):
+    with pytest.raises(Exception, match="warm workspace"):
         with torch.cuda.graph(g, stream=s):
-            libsat.sat(x, out=y)
+            libsat.sat(x)
     torch.cuda.synchronize()
     check(libsat.sat(x), oracle.sat(x.cpu().numpy()), "int32")
