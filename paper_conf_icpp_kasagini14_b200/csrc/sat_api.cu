@@ -508,20 +508,21 @@ struct Job {
     cudaStream_t st;
 };
 
-// Device-side ticket base (graph capture): the ticket counter ends every band
-// launch at base + units + takers, the next launch's base; reset it (and
-// request a descriptor clear) when the tag space would run out.
-__global__ void sat_epoch_kernel(unsigned long long* tk, unsigned long long worst, unsigned long long space) {
-    if (threadIdx.x != 0) return;
-    const unsigned long long t = tk[0];
-    const bool reset = t + worst >= space;
-    if (reset) tk[0] = 0;
-    tk[1] = reset ? 0 : t;
-    tk[2] = reset ? 1 : 0;
-}
-
-__global__ void sat_epoch_clear_kernel(const unsigned long long* flag, uint4* a, size_t na, uint4* b, size_t nb) {
-    if (!*flag) return;
+// Device-side ticket base (graph capture).  The ticket counter (64-bit, never
+// reset on this path) ends every band launch at base + units + takers, the
+// next launch's base; block 0 copies it to tk[1] for the band kernel (whose
+// CTAs advance tk[0] while they start).  Tags are 30 bits of base + unit, so a
+// stale descriptor could match again one tag space later: every block clears
+// the descriptors whenever this launch's value range [t, t + worst) crosses a
+// multiple of half the tag space.  Between clears every live descriptor was
+// written less than half a space + one launch earlier, so none can alias.
+// One launch, decided on the device from t alone (no state, no inter-block
+// race: nothing in this kernel writes tk[0]).
+__global__ void sat_epoch_kernel(unsigned long long* tk, unsigned long long worst, unsigned long long half,
+                                 uint4* a, size_t na, uint4* b, size_t nb) {
+    const unsigned long long t = __ldcg(tk);
+    if (blockIdx.x == 0 && threadIdx.x == 0) tk[1] = t;
+    if (t / half == (t + worst) / half) return;
     const uint4 z = make_uint4(0, 0, 0, 0);
     for (size_t i = size_t(blockIdx.x) * blockDim.x + threadIdx.x; i < na + nb; i += size_t(gridDim.x) * blockDim.x) {
         if (i < na) a[i] = z; else b[i - na] = z;
@@ -611,16 +612,12 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.base_dev = nullptr;
     if (ws.dev_epoch) {
         unsigned long long* tk = static_cast<unsigned long long*>(ws.ticket.p);
-        sat_epoch_kernel<<<1, 32, 0, j.st>>>(tk, worst, tag_space());
-        CUDA_TRY(cudaGetLastError());
         const size_t dw = ws.desc.p ? ws.desc.bytes / 16 : 0, lw = ws.lseg.p ? ws.lseg.bytes / 16 : 0;
-        if (dw + lw) {
-            sat_epoch_clear_kernel<<<2 * j.di->sms, 256, 0, j.st>>>(tk + 2, static_cast<uint4*>(ws.desc.p), dw,
-                                                                    static_cast<uint4*>(ws.lseg.p), lw);
-            CUDA_TRY(cudaGetLastError());
-        }
+        sat_epoch_kernel<<<2 * j.di->sms, 256, 0, j.st>>>(tk, worst, tag_space() / 2, static_cast<uint4*>(ws.desc.p),
+                                                          dw, static_cast<uint4*>(ws.lseg.p), lw);
+        CUDA_TRY(cudaGetLastError());
         p.base_dev = tk + 1;
-        t_launches += dw + lw ? 2 : 1;
+        ++t_launches;
     } else if (ws.next_base + worst >= tag_space()) {
         // tag space exhausted: clear descriptors and the counter (rare)
         if (ws.desc.p) CUDA_TRY(cudaMemsetAsync(ws.desc.p, 0, ws.desc.bytes, j.st));

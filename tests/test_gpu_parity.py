@@ -546,11 +546,14 @@ def test_cuda_graph_replay(libsat, variant, shape, dtype):
         check(z.cpu().numpy(), oracle.sat(host), dtype)
 
 
-def test_cuda_graph_tag_reset(libsat, monkeypatch):
-    """A tiny tag space (SAT_TAG_SPACE) forces the device-side reset in
-    sat_epoch_kernel (ticket to 0, descriptors cleared) during replays, and
-    the host-side reset on eager calls."""
-    monkeypatch.setenv("SAT_TAG_SPACE", "300000")
+@pytest.mark.parametrize("space,replays", [("300000", 6), ("540000", 60)])
+def test_cuda_graph_tag_reset(libsat, monkeypatch, space, replays):
+    """A tiny tag space (SAT_TAG_SPACE) makes sat_epoch_kernel clear the
+    descriptors on every replay (each launch's value range crosses a multiple
+    of half the space), and forces the host-side reset on eager calls of a
+    never-captured stream.  At 540000 (half the space just above the
+    per-launch bound) only some replays clear: the mixed regime."""
+    monkeypatch.setenv("SAT_TAG_SPACE", space)
     x = dev(gen(2048, 2048, "int32", seed=3))
     s = torch.cuda.Stream()
     with torch.cuda.stream(s):
@@ -559,7 +562,7 @@ def test_cuda_graph_tag_reset(libsat, monkeypatch):
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g, stream=s):
         libsat.sat(x, out=y)
-    for it in range(6):
+    for it in range(replays):
         host = gen(2048, 2048, "int32", seed=20 + it)
         x.copy_(dev(host))
         g.replay()
@@ -569,6 +572,10 @@ def test_cuda_graph_tag_reset(libsat, monkeypatch):
     x2 = dev(host)
     for it in range(3):
         assert np.array_equal(libsat.sat(x2).cpu().numpy(), oracle.sat(host)), f"eager {it}"
+        with torch.cuda.stream(s):
+            z = libsat.sat(x2)
+        s.synchronize()
+        assert np.array_equal(z.cpu().numpy(), oracle.sat(host)), f"eager after capture {it}"
 
 
 @pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")
