@@ -110,10 +110,13 @@ typedef struct sat_options {
 /* Fill *opt with defaults (r = 0.25, automatic tile, TMA when eligible). */
 void sat_options_init(sat_options *opt);
 
-/* Stream capture (CUDA graphs) is refused with SAT_ERR_UNSUPPORTED by every
- * entry point that launches the band kernel: its look-back tags and ticket
- * base are assigned per launch on the host, so a replayed graph would reuse
- * them. */
+/* Stream capture (CUDA graphs) is supported by every entry point that
+ * launches the band kernel on a device stream.  Requirement: one eager call of
+ * the same shape/variant on the same stream first (a captured call cannot
+ * allocate its workspace; otherwise SAT_ERR_UNSUPPORTED, "warm workspace").
+ * From the first capture on, that stream's launches take their look-back
+ * ticket base from the device (one extra small kernel per band launch,
+ * DESIGN.md Sec. 4), so replays and later eager calls stay correct. */
 
 /* out = SAT(in) for one rows x cols matrix.  variant: sat_variant. */
 int sat_compute(const void *in, void *out, int64_t rows, int64_t cols,
