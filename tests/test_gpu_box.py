@@ -158,3 +158,26 @@ def test_rect_sums(libsat):
     gf = libsat.rect_sums(sf, dev(rq)).cpu().numpy()
     for q, (_, r0, c0, r1, c1) in enumerate(rq.tolist()):
         assert gf[q] == f[r0:r1 + 1, c0:c1 + 1].sum()
+
+
+def test_box_filter_cuda_graph(libsat):
+    """The box filter (widening 1R1W SAT + box pass) captured in a CUDA graph
+    and replayed on fresh uint8 frames (the device-side ticket base,
+    DESIGN.md Sec. 4); the workspace is sized by one eager call first."""
+    B, n, m, rr, rc = 3, 540, 960, 4, 4
+    x = dev(u8img(n, m, seed=1, batch=B))
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        y = libsat.box_filter(x, rr, rc)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.box_filter(x, rr, rc, out=y)
+    for it in range(3):
+        a = u8img(n, m, seed=50 + it, batch=B)
+        x.copy_(dev(a))
+        g.replay()
+        torch.cuda.synchronize()
+        got = y.cpu().numpy()
+        for b in range(B):
+            assert np.array_equal(got[b], oracle.box_filter(a[b].astype(np.int32), rr, rc)), (it, b)

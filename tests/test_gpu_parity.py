@@ -546,6 +546,34 @@ def test_cuda_graph_replay(libsat, variant, shape, dtype):
         check(z.cpu().numpy(), oracle.sat(host), dtype)
 
 
+def test_cuda_graph_batched_two_shapes(libsat):
+    """Two captured calls of different shapes on one stream (batched and 2-D),
+    one graph, the workspace sized by eager calls of both."""
+    a = gen(700, 1500, "int32", seed=7)
+    xb = dev(make_np(300, 800, "int32", "u32", seed=8, batch=5))
+    x = dev(a)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        y = libsat.sat(x)
+        yb = libsat.sat_batched(xb)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.sat(x, out=y)
+        libsat.sat_batched(xb, out=yb)
+    for it in range(3):
+        a = gen(700, 1500, "int32", seed=60 + it)
+        ab = make_np(300, 800, "int32", "u32", seed=70 + it, batch=5)
+        x.copy_(dev(a))
+        xb.copy_(dev(ab))
+        g.replay()
+        torch.cuda.synchronize()
+        check(y, oracle.sat(a), "int32")
+        got = yb.cpu().numpy()
+        for b in range(5):
+            check(got[b], oracle.sat(ab[b]), "int32")
+
+
 @pytest.mark.parametrize("space,replays", [("300000", 6), ("540000", 60)])
 def test_cuda_graph_tag_reset(libsat, monkeypatch, space, replays):
     """A tiny tag space (SAT_TAG_SPACE) makes sat_epoch_kernel clear the
