@@ -116,7 +116,11 @@ void sat_options_init(sat_options *opt);
  * allocate its workspace; otherwise SAT_ERR_UNSUPPORTED, "warm workspace").
  * From the first capture on, that stream's launches take their look-back
  * ticket base from the device (one extra small kernel per band launch,
- * DESIGN.md Sec. 4), so replays and later eager calls stay correct. */
+ * DESIGN.md Sec. 4), so replays and later eager calls stay correct.
+ * The captured launches keep using the capture stream's workspace
+ * (descriptors, ticket): replays of graphs captured on one stream, and eager
+ * calls on that stream, must not run concurrently with each other (replay
+ * them in stream order, as with any graph that owns scratch memory). */
 
 /* out = SAT(in) for one rows x cols matrix.  variant: sat_variant. */
 int sat_compute(const void *in, void *out, int64_t rows, int64_t cols,
