@@ -111,7 +111,10 @@ typedef struct sat_options {
 void sat_options_init(sat_options *opt);
 
 /* Stream capture (CUDA graphs) is supported by every entry point that
- * launches the band kernel on a device stream.  Requirement: one eager call of
+ * launches the band kernel on a device stream, except
+ * sat_compute_sharded_fused (its exchange epoch is host-assigned) and
+ * sat_compute_host (it synchronizes), which return SAT_ERR_UNSUPPORTED under
+ * capture.  Requirement: one eager call of
  * the same shape/variant on the same stream first (a captured call cannot
  * allocate its workspace; otherwise SAT_ERR_UNSUPPORTED, "warm workspace").
  * From the first capture on, that stream's launches take their look-back

@@ -972,6 +972,9 @@ int sharded_fused_t(const void* in, void* out, int64_t strip_rows, PeerExchange&
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
+    if (t_capture)
+        return fail(SAT_ERR_UNSUPPORTED, "sat_compute_sharded_fused cannot be captured: the exchange epoch "
+                                         "is assigned per call on the host (a replay would reuse it)");
     const int64_t cols = ex.cols;
     ex.x.epoch += 1;
     int launches = 0;
@@ -1327,6 +1330,8 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
+    if (t_capture)
+        return fail(SAT_ERR_UNSUPPORTED, "sat_compute_host cannot be captured: it synchronizes the stream");
     const size_t bytes = size_t(rows) * size_t(cols) * esize(dtype);
     SAT_TRY(ensure(ws->din, bytes, false));
     SAT_TRY(ensure(ws->dout, bytes, false));

@@ -618,3 +618,18 @@ def test_capture_cold_workspace_refused(libsat):
             libsat.sat(x)
     torch.cuda.synchronize()
     check(libsat.sat(x), oracle.sat(x.cpu().numpy()), "int32")
+
+
+@pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")
+def test_capture_host_call_refused(libsat):
+    """sat_host synchronizes its stream, so it refuses capture loudly."""
+    a = torch.from_numpy(gen(256, 512, "int32", seed=9)).pin_memory()
+    o = torch.empty_like(a).pin_memory()
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with pytest.raises(Exception, match="cannot be captured"):
+        with torch.cuda.graph(g, stream=s):
+            libsat.sat_host(a, o)
+    torch.cuda.synchronize()
+    libsat.sat_host(a, o)
+    assert np.array_equal(o.numpy(), oracle.sat(a.numpy()))
