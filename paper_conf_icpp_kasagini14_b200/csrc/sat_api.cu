@@ -328,7 +328,28 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap&
         if (grid < 1) grid = 1;
         grid_out = int(grid);
         t_grid = int(grid);
-        kern<<<int(grid), threads, smem, st>>>(ti, p);
+        // programmatic dependent launch: the CTA prologue (barriers, TMEM
+        // alloc) overlaps the previous kernel's tail; the kernel waits
+        // (griddepcontrol.wait) before its first global access.  Back-to-back
+        // calls: 1024^2 16.7 -> 14.4 us, 4096^2 f32 47.9 -> 45.5 us
+        // (profiles/r01_pdl_ab.txt).  SAT_PDL=0 turns it off.
+        static const bool pdl = [] { const char* e = getenv("SAT_PDL"); return !e || atoi(e) != 0; }();
+        if (pdl) {
+            cudaLaunchConfig_t cfg;
+            std::memset(&cfg, 0, sizeof(cfg));
+            cfg.gridDim = dim3(unsigned(grid));
+            cfg.blockDim = dim3(unsigned(threads));
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = st;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            attr[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ti, p));
+        } else {
+            kern<<<int(grid), threads, smem, st>>>(ti, p);
+        }
     }
     CUDA_TRY(cudaGetLastError());
     ++t_launches;

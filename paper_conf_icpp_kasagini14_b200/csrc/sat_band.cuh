@@ -341,7 +341,6 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
     // ticket/tag base: the host's counter, or (CUDA-graph capture, DESIGN.md
     // Sec. 4) the value sat_epoch_kernel wrote just before this launch
-    const unsigned long long kbase = p.base_dev ? __ldcg(p.base_dev) : p.base;
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -381,6 +380,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     if constexpr (CL > 1) cluster_sync_all();    // peers' barriers initialised before any remote arrive
     tmem_fence_after();
     const uint32_t tmem_base = HOLD ? *s_tmem : 0u;
+    // Programmatic dependent launch (SAT_PDL): everything above is CTA-local
+    // and may overlap the previous kernel's tail; global memory from here on
+    // (a no-op when launched without the attribute)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    const unsigned long long kbase = p.base_dev ? __ldcg(p.base_dev) : p.base;
 
     const int64_t img_elems = p.rows * p.cols;
     const int desc_w = p.nc * TW;
