@@ -5,12 +5,16 @@ Default workload (BASELINE.json config 4, the one the metric "... at
 1/2/4/8 B200" is quoted on; it fits one GPU): the SAT of one 65536 x 65536
 int32 matrix (uint32 wrapping arithmetic), 1R1W.  At N=1 one GPU computes it
 with one kernel launch per step; at N>1 the matrix is split into N row strips
-(one per rank) and each step is: column totals -> NCCL all-gather -> rank
-exclusive scan -> seeded 1R1W (strong scaling: total work fixed).
+(one per rank, the last one 1.5x as tall: it skips the totals pass) and each
+step is: column totals (one launch) -> NCCL all-gather -> seeded 1R1W whose
+band 0 does the rank exclusive scan (one launch); rank 0's SAT does not wait
+for the gather (strong scaling: total work fixed).
 
 Timing: W untimed warm-up steps, then exactly K steps bracketed by barrier +
 cuda synchronize, CUDA events on the launching stream, max over ranks.  Inputs
-(16 GiB) are far larger than L2 (126 MB), so no flush is needed.
+(16 GiB) are far larger than L2 (126 MB), so no flush is needed; configs whose
+working set is < 4 x L2 (cfg1, cfg2, cfg5) write a 2 x L2 buffer between steps
+(the hot, un-flushed number is reported beside it).
 `--impl reference` times the CPU oracle (the reference arm of this tier).
 Other BASELINE configs: `--config cfg1|cfg2|cfg3|cfg3b|cfg4|cfg5`.
 """
@@ -217,6 +221,33 @@ def run_reference(args, cfg_key):
 
 
 # ------------------------------------------------------------------ our arm
+def strip_parity(x, y, dtype, r0, rows_above_gen, check_rows=256):
+    """Parity of this rank's strip (first ``check_rows`` rows) against the CPU
+    oracle streamed from the column sums of every row above the strip.  Those
+    sums are computed with torch (int64 / float64 accumulation of the seeded
+    generator's rows, independent of libsat), the strip rows by the oracle."""
+    import numpy as np
+    import torch
+    import oracle
+    cols = x.shape[1]
+    acc = torch.zeros(cols, dtype=torch.int64 if dtype == "int32" else torch.float64, device=x.device)
+    step = max(1, (1 << 27) // cols)
+    for a in range(0, r0, step):
+        blk = rows_above_gen(a, min(r0, a + step))
+        acc += blk.to(acc.dtype).sum(dim=0)
+    st = oracle.Stream(cols, dtype == "int32")
+    if dtype == "int32":
+        st.colsum[:] = (acc % (1 << 32)).cpu().numpy().astype(np.uint32)
+    else:
+        st.colsum[:] = acc.cpu().numpy()
+    n = min(check_rows, x.shape[0])
+    ref = st.feed(x[:n].cpu().numpy())
+    got = y[:n].cpu().numpy()
+    if dtype == "int32":
+        return bool(np.array_equal(got, ref))
+    return bool(oracle.max_rel_err(got, ref) <= 1e-5)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -229,7 +260,10 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--cpu-sample-rows", type=int, default=None)
+    ap.add_argument("--flush-l2", default="auto", choices=["auto", "on", "off"],
+                    help="write a 2 x L2 buffer between timed steps (auto: when the working set < 4 x L2)")
+    ap.add_argument("--last-weight", type=float, default=1.5,
+                    help="N>1 row strips: the last rank's share (it skips the totals pass)")
     ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
                     help="N>1 row strips: NCCL all-gather, or the fused peer exchange (IPC mailboxes)")
     args = ap.parse_args()
@@ -264,13 +298,13 @@ def main():
     tdt = torch.int32 if dtype == "int32" else torch.float32
     dist_name = "u32" if dtype == "int32" else "unit"
     eb = 4
+    l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
 
     # ---------------- per-rank work unit
+    r0, r1 = 0, rows
     if batch is None:
         if world > 1:
-            r0, r1 = partition_rows(rows, world, rank)
-        else:
-            r0, r1 = 0, rows
+            r0, r1 = partition_rows(rows, world, rank, args.last_weight)
         x = make_torch(r1 - r0, cols, dtype, dist_name, seed=4001, row0=r0, device=dev)
         y = torch.empty_like(x)
         my_elems = (r1 - r0) * cols
@@ -285,9 +319,12 @@ def main():
         scaling = "weak"
     sharded = world > 1 and batch is None
     opts = dict(tile_rows=args.tile_rows) if args.tile_rows else {}
+    flush = args.flush_l2 == "on" or (args.flush_l2 == "auto" and 2 * my_elems * eb < 4 * l2_bytes)
+    flushbuf = torch.empty(2 * l2_bytes, dtype=torch.uint8, device=dev) if flush else None
 
     launches = [0]
-
+    breakdown = None
+    # kernel events: (start, end) around the band kernel of each step
     if sharded and args.exchange == "fused":
         from paper_conf_icpp_kasagini14_b200.dist import make_peer_exchange
         xchg, _ = make_peer_exchange(cols, tdt, device=dev)
@@ -300,29 +337,25 @@ def main():
                 ev[1].record(stream)
             launches[0] += libsat.last_launch_count()
     elif sharded:
-        P = world
-        gathered = torch.empty(P * cols, dtype=tdt, device=dev)
-        send = torch.empty(cols, dtype=tdt, device=dev)
+        from paper_conf_icpp_kasagini14_b200.dist import RowStripSAT
+        op = RowStripSAT(cols, tdt, device=dev)
+        breakdown = {"totals_ms": [], "gather_ms": [], "sat_ms": []}
+        step_events = []
 
         def step(ev=None):
-            n = 0
-            if rank < P - 1:
-                libsat.column_totals(x, out=send)
-                n += libsat.last_launch_count()
-            else:
-                send.zero_()
-            dist.all_gather_into_tensor(gathered, send)
-            carry = None
-            if rank > 0:
-                carry = libsat.rank_exscan(gathered.view(P, cols), rank)
-                n += libsat.last_launch_count()
+            e = None
             if ev:
-                ev[0].record(stream)
-            libsat.sat_seeded(x, carry_row=carry, out=y)
-            if ev:
-                ev[1].record(stream)
-            n += libsat.last_launch_count()
+                e = {k: torch.cuda.Event(enable_timing=True) for k in ("t0", "totals", "gather", "sat")}
+                if rank == 0:
+                    e.pop("gather")
+                step_events.append(e)
+            op(x, out=y, events=e)
+            n = 1 + (1 if rank < world - 1 else 0)
             launches[0] += n
+            if ev:
+                # the band kernel: after the gather (ranks > 0), right after the totals (rank 0)
+                ev[0] = e["gather"] if "gather" in e else e["totals"]
+                ev[1] = e["sat"]
     else:
         def step(ev=None):
             if ev:
@@ -345,7 +378,7 @@ def main():
         step()
     barrier()
     parity = None
-    if rank == 0 and not sharded:
+    if not sharded and rank == 0:
         import numpy as np
         import oracle
 
@@ -359,32 +392,66 @@ def main():
             # first and last image of the batch, whole
             parity = all(same(y[i].cpu().numpy(), oracle.sat(x[i].cpu().numpy()))
                          for i in (0, batch - 1))
+    elif sharded:
+        # every rank: the first 256 rows of its strip against the oracle
+        # seeded with the column sums of all rows above it
+        ok = strip_parity(x, y, dtype, r0,
+                          lambda a, b: make_torch(b - a, cols, dtype, dist_name, seed=4001, row0=a,
+                                                  device=dev))
+        t = torch.tensor([0 if ok else 1], device=dev)
+        dist.all_reduce(t)
+        parity = {"ranks_checked": world, "rows_per_rank": 256, "ok": int(t.item()) == 0}
 
     # ---------------- timed region
-    launches[0] = 0
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
-    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(args.steps)]
-    barrier()
-    with ClockSampler(local) as clk:
-        time.sleep(0.3)                     # let the sampler start
+    def timed(flush_between):
+        launches[0] = 0
+        if breakdown is not None:
+            step_events.clear()
+        ev0 = torch.cuda.Event(enable_timing=True)
+        ev1 = torch.cuda.Event(enable_timing=True)
+        kev = [[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)]
+               for _ in range(args.steps)]
         barrier()
         ev0.record(stream)
         for i in range(args.steps):
+            if flush_between:
+                flushbuf.zero_()
             step(kev[i])
         ev1.record(stream)
         barrier()
+        kern_ms = [a.elapsed_time(b) for a, b in kev]
+        return ev0.elapsed_time(ev1), kern_ms
+
+    with ClockSampler(local) as clk:
+        time.sleep(0.3)                     # let the sampler start
+        ms_local, kern_ms = timed(flush)
+    clocks = clk.summary()
     tile_rows = libsat.last_tile_rows()
-    kern_ms = [a.elapsed_time(b) for a, b in kev]
-    ms_local = ev0.elapsed_time(ev1)
+    step_launches = launches[0]
+    if flush:
+        # the flush writes sit between steps: the step time is the band
+        # kernel's event time (one launch per step at N = 1)
+        ms_local = sum(kern_ms)
+    if breakdown is not None:
+        for e in step_events:
+            breakdown["totals_ms"].append(e["t0"].elapsed_time(e["totals"]))
+            if "gather" in e:
+                breakdown["gather_ms"].append(e["totals"].elapsed_time(e["gather"]))
+                breakdown["sat_ms"].append(e["gather"].elapsed_time(e["sat"]))
+            else:
+                breakdown["sat_ms"].append(e["totals"].elapsed_time(e["sat"]))
     t = torch.tensor([ms_local, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_total, kern_avg_ms = float(t[0]), float(t[1])
     ms_per_step = ms_total / args.steps
     value = total_elems * args.steps / (ms_total / 1e3)
-    clocks = clk.summary()
+    hot = None
+    if flush and not sharded:
+        hot_ms, hot_k = timed(False)
+        hot = {"value": total_elems * args.steps / (hot_ms / 1e3), "unit": "elem/s",
+               "ms_per_step": hot_ms / args.steps, "kernel_ms": statistics.mean(hot_k),
+               "l2": "no flush between steps (inputs may be L2-resident)"}
 
     # ---------------- roofline of the dominant kernel (the band kernel)
     peak, peak_kind = measured_peaks()
@@ -399,13 +466,18 @@ def main():
         alg_bytes = 8 * eb * my_elems
     elif variant == "4r1w":                            # Formula (1): 4 reads + 1 write, Lemma 5
         alg_bytes = 5 * eb * my_elems
-    achieved = alg_bytes / (kern_avg_ms / 1e3) / 1e9
+    mine = torch.tensor([alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(mine, op=dist.ReduceOp.MIN)    # the slowest rank's band kernel
+    achieved = float(mine[0])
     traffic = ncu_traffic(f"{cfg_key}:{variant}:n{world}")
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "peak_kind": peak_kind, "kernel": "sat_band_kernel",
                 "alg_bytes_per_launch": alg_bytes, "kernel_ms": round(kern_avg_ms, 4),
                 "frac_of_8TBs": round(achieved / 8000.0, 4)}
+    if world > 1:
+        roofline["note"] = "min over ranks of the band kernel's 1R1W byte rate on its own strip"
 
     # ---------------- end to end through the public API from pinned host memory
     e2e = None
@@ -429,6 +501,17 @@ def main():
                        "rule": "bit-exact" if dtype == "int32" else "max rel err <= 1e-5",
                        "max_rel_err": err if dtype != "int32" else None}
 
+    bd = None
+    if breakdown is not None:
+        vals = torch.tensor([statistics.mean(breakdown["totals_ms"]),
+                             statistics.mean(breakdown["gather_ms"]) if breakdown["gather_ms"] else 0.0,
+                             statistics.mean(breakdown["sat_ms"])], dtype=torch.float64, device=dev)
+        allv = [torch.zeros_like(vals) for _ in range(world)]
+        dist.all_gather(allv, vals)
+        bd = {"per_rank_ms": [[round(float(v), 4) for v in a.tolist()] for a in allv],
+              "columns": ["totals (extra read)", "all-gather wait", "seeded SAT (band kernel)"],
+              "rows": [list(partition_rows(rows, world, p, args.last_weight)) for p in range(world)]}
+
     if rank == 0:
         line = {
             "metric": BASELINE_METRIC, "value": value, "unit": "elem/s", "n_gpus": world,
@@ -438,19 +521,24 @@ def main():
             "data": "synthetic (splitmix64 counter hash: uniform 32-bit int / dyadic [0,1) float)",
             "config": {"workload": desc + (f" [{variant}]" if variant != "1r1w" else ""),
                        "rows": rows, "cols": cols, "batch": batch,
-                       "parallelism": (f"row-strips x{world} ({args.exchange} exchange)" if sharded else
+                       "parallelism": (f"row-strips x{world} ({args.exchange} exchange, last weight "
+                                       f"{args.last_weight})" if sharded else
                                        (f"dp{world}" if world > 1 else "1 GPU")),
-                       "l2": "inputs > L2, no flush" if my_elems * eb > 4 * 126e6 else
-                             "inputs near L2 size: hot-L2 number",
+                       "l2": ("flushed: a 2 x L2 buffer written between steps; the step time is the "
+                              "band kernel's event time" if flush else "inputs > 4 x L2, no flush"),
                        "tile_rows": tile_rows},
             "roofline": roofline,
             "cpu_baseline": cpu,
             "e2e": e2e,
-            "gpu_launches": launches[0],
+            "gpu_launches": step_launches,
             "clocks": clocks,
             "parity_recheck": parity,
             "parity_full": full_parity,
         }
+        if hot:
+            line["hot"] = hot
+        if bd:
+            line["breakdown"] = bd
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()

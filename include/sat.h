@@ -27,7 +27,7 @@
  *     paper's "double (64-bit)" precision) uses IEEE fp64 adds with
  *     the same ordering caveats; for inputs k*2^-24 every partial sum below
  *     2^29 is exact, so those results are unique.  Float64 takes tile_rows
- *     16, 32, 48 or 64 and needs 8-byte aligned pointers; the TMA path needs
+ *     16, 32 or 64 and needs 8-byte aligned pointers; the TMA path needs
  *     16-byte aligned pointers and cols % 4 == 0 (as for 4-byte types).
  *   - in == out (exact aliasing) is allowed for every entry point that takes
  *     both; a partial overlap returns SAT_ERR_INVALID.
@@ -52,7 +52,7 @@
 extern "C" {
 #endif
 
-#define SAT_ABI_VERSION 1
+#define SAT_ABI_VERSION 2
 
 typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1, SAT_FLOAT64 = 2,
                SAT_UINT8 = 3 /* input only: sat_compute_widening, sat_box_filter */ } sat_dtype;
@@ -97,14 +97,20 @@ typedef struct sat_options {
     double r;            /* SAT_1PLUSR_R1W: target fraction of tiles done by 2R1W
                             (0..1, default 0.25); the realised value is the tile
                             count ratio, see sat_last_r_effective() */
-    int tile_rows;       /* band height TH in {16, 32, 48, 64, 112, 128} (float64:
-                            16, 32, 48, 64); 0 = automatic (DESIGN.md Sec. 5:
-                            1R1W takes 128 once its bands fill half the SMs,
-                            else 32 from 1536 rows, else 16) */
+    int tile_rows;       /* 1R1W-family band height TH in {16, 32, 64, 128}
+                            (float64: 16, 32, 64; uint8 input: 64, 128); 0 =
+                            automatic (1R1W takes 128 once its
+                            bands fill half the SMs, else 32 from 1536 rows,
+                            else 16).  A height without an instantiated
+                            configuration is rounded down to one that has it
+                            (sat_last_tile_rows() reports the height used). */
     int force_generic;   /* 1 = use the non-TMA load/store path (tests) */
-    int jitter;          /* debug: random delay (ns) before descriptor
-                            publication, to stress the look-back; 0 = off */
-    int reserved[4];     /* must be 0 */
+    int jitter;          /* stress tests: random delay (ns) before descriptor
+                            publication, to shuffle the look-back; 0 = off */
+    int segments;        /* 1R1W band segments: 0 =
+                            automatic, n >= 1 = cut every band into n column
+                            segments (tests) */
+    int reserved[3];     /* must be 0 */
 } sat_options;
 
 /* Fill *opt with defaults (r = 0.25, automatic tile, TMA when eligible). */
@@ -180,9 +186,19 @@ int sat_rect_sums(const void *sat, int dtype, int64_t batch, int64_t rows, int64
 /* Seeded 1R1W: the rows x cols matrix is a strip of a taller matrix and
  * carry_row[j] (device, cols entries, same dtype) is the column sum of
  * everything above the strip in column j.  Result: the strip's rows of the
- * full matrix's SAT.  carry_row == NULL is the unseeded case. */
+ * full matrix's SAT.  carry_row == NULL is the unseeded case.  One launch:
+ * band 0 adds the carry to the strip's first input row before its row scan
+ * (SAT([c; a]) restricted to a's rows), so no carry-prefix pass runs. */
 int sat_compute_seeded(const void *in, void *out, int64_t rows, int64_t cols,
                        int dtype, const void *carry_row, void *stream);
+
+/* As sat_compute_seeded with carry_row[j] = sum_{q < nvec} vectors[q*stride + j]
+ * (q ascending; stride in elements, >= cols when nvec > 1): the row-strip
+ * sharded mode passes the all-gathered column totals of all ranks and its rank
+ * as nvec, so the exclusive scan over ranks happens inside the SAT kernel. */
+int sat_compute_seeded_sum(const void *in, void *out, int64_t rows, int64_t cols,
+                           int dtype, const void *vectors, int64_t nvec, int64_t stride,
+                           void *stream);
 
 /* As sat_compute_seeded, but sat_row[j] is the SAT row just above the strip
  * (the last SAT row of the strip above), not the column sums. */
@@ -190,11 +206,13 @@ int sat_compute_seeded_satrow(const void *in, void *out, int64_t rows, int64_t c
                               int dtype, const void *sat_row, void *stream);
 
 /* ---- Fused peer exchange ----
- * The sharded mode without a collective call: rank p's column-totals kernel
- * stores its totals straight into slot p of every higher rank's "mailbox"
- * (peer memory over NVLink, e.g. IPC-mapped) and raises a flag there; rank
- * p's SAT prologue waits for the flags of ranks < p, sums their slots in rank
- * order (the exclusive scan) and acknowledges; then the seeded 1R1W runs.
+ * The sharded mode without a collective call and with two launches per rank:
+ * rank p's column-totals kernel (one launch) ends by storing its totals
+ * straight into slot p of every higher rank's "mailbox" (peer memory over
+ * NVLink, e.g. IPC-mapped) and raising a flag there (st.release.sys); rank
+ * p's SAT kernel (one launch) waits in band 0 for the flags of ranks < p
+ * (ld.acquire.sys), adds the sum of their slots in rank order (the exclusive
+ * scan) to its first input row, and acknowledges once band 0 has read them.
  * Mailboxes are double-buffered by call parity with acknowledgements, so
  * consecutive calls need no barrier.  All ranks must make the same sequence of
  * calls.  Results are bit-identical to sat_compute_sharded (int32).
@@ -245,8 +263,9 @@ typedef struct sat_shard_stats {
  * `nranks` consecutive row strips of one matrix (strips may have different
  * heights; every rank passes the same cols).  Steps: column totals of the
  * strip (skipped on the last rank, whose totals nobody needs -- it sends
- * zeros), all-gather through `allgather`, exclusive scan over ranks, seeded
- * 1R1W.  `workspace` is a caller-owned device buffer of at least
+ * zeros), all-gather through `allgather`, seeded 1R1W whose band 0 sums the
+ * gathered totals of ranks < rank (the exclusive scan, in the SAT kernel).
+ * Two launches per rank + the callback.  `workspace` is a caller-owned device buffer of at least
  * sat_sharded_workspace_bytes(cols, nranks, dtype) bytes (NULL = library
  * allocated).  stats may be NULL. */
 int sat_compute_sharded(const void *in_strip, void *out_strip, int64_t strip_rows,
@@ -263,7 +282,8 @@ size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype);
 int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t cols,
                      int dtype, int variant, void *stream);
 
-/* Debug/profiling: the next 1R1W-family band launch on this thread records,
+/* Debug/profiling (builds with SAT_DEBUG=1 only; SAT_ERR_UNSUPPORTED
+ * otherwise): the next 1R1W-family band launch on this thread records,
  * per (band, chunk) of TH x 128 elements, eight 64-bit globaltimer stamps
  * (ns) into dev_buf[(band*nchunks + chunk)*8 + e]: e=0 tile data arrived,
  * e=1 band-local reductions done, e=2 look-back done (bits 48..55 = look-
@@ -273,12 +293,23 @@ int sat_compute_host(const void *in_host, void *out_host, int64_t rows, int64_t 
  * ceil(rows/TH)*batch*ceil(cols/128)*64 bytes; NULL disarms. */
 int sat_debug_trace(void *dev_buf);
 
-/* Debug: record, in host-mapped memory, what every spinning warp waits on
+/* Watchdog diagnostics: record, in host-mapped memory, what every spinning warp waits on
  * once a wait exceeds half the 4-s watchdog (before the kernel traps);
  * sat_debug_diag_dump prints the records to stderr (also after a failed
  * launch) and returns their number. */
 int sat_debug_diag_enable(void);
 int sat_debug_diag_dump(void);
+
+/* Free the library workspace of `stream` on the current device (look-back
+ * descriptors, ticket, carry buffers, and buffers retired after a graph
+ * capture).  Synchronizes the stream first.  CUDA graphs captured on that
+ * stream must not be replayed afterwards.  The next call on the stream
+ * allocates a fresh workspace. */
+int sat_release_workspace(void *stream);
+
+/* Tests only: shrink the look-back tag space (default and maximum 2^30;
+ * 0 restores the default) so the tag-exhaustion paths run. */
+int sat_debug_set_tag_space(uint64_t space);
 
 /* Number of kernels launched by the last successful call on this thread. */
 int sat_last_launch_count(void);

@@ -29,7 +29,7 @@ SAT_OK = 0
 class SatOptions(ctypes.Structure):
     _fields_ = [("r", ctypes.c_double), ("tile_rows", ctypes.c_int),
                 ("force_generic", ctypes.c_int), ("jitter", ctypes.c_int),
-                ("reserved", ctypes.c_int * 4)]
+                ("segments", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
 
 
 class SatShardStats(ctypes.Structure):
@@ -58,6 +58,7 @@ _SIGS = {
     "sat_ipc_open": ([_P, ctypes.POINTER(ctypes.c_void_p)], _I),
     "sat_ipc_close": ([_P], _I),
     "sat_compute_seeded": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
+    "sat_compute_seeded_sum": ([_P, _P, _I64, _I64, _I, _P, _I64, _I64, _P], _I),
     "sat_compute_seeded_satrow": ([_P, _P, _I64, _I64, _I, _P, _P], _I),
     "sat_column_totals": ([_P, _P, _I64, _I64, _I, _P], _I),
     "sat_rank_exscan": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
@@ -65,6 +66,8 @@ _SIGS = {
                              ctypes.POINTER(SatShardStats)], _I),
     "sat_sharded_workspace_bytes": ([_I64, _I, _I], ctypes.c_size_t),
     "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
+    "sat_release_workspace": ([_P], _I),
+    "sat_debug_set_tag_space": ([ctypes.c_uint64], _I),
     "sat_debug_trace": ([_P], _I),
     "sat_debug_diag_enable": ([], _I),
     "sat_debug_diag_dump": ([], _I),
@@ -128,18 +131,19 @@ def _check_dev(*ts):
 
 
 def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
-            jitter: int = 0) -> SatOptions:
+            jitter: int = 0, segments: int = 0) -> SatOptions:
     o = SatOptions()
     _lib.sat_options_init(ctypes.byref(o))
     o.r = float(r)
     o.tile_rows = int(tile_rows)
     o.force_generic = int(bool(force_generic))
     o.jitter = int(jitter)
+    o.segments = int(segments)
     return o
 
 
 def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
-        force_generic: bool = False, jitter: int = 0, stream=None):
+        force_generic: bool = False, jitter: int = 0, segments: int = 0, stream=None):
     """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32/float64 IEEE).
 
     ``out`` may be ``x`` itself (in place).  ``variant`` in
@@ -153,14 +157,14 @@ def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
     _check_dev(x, out)
     if out.shape != x.shape or out.dtype != x.dtype:
         raise ValueError("out must match x in shape and dtype")
-    o = options(r, tile_rows, force_generic, jitter)
+    o = options(r, tile_rows, force_generic, jitter, segments)
     _check(_lib.sat_compute_ex(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                _dtype_code(x), VARIANTS[variant], ctypes.byref(o), _stream(stream)))
     return out
 
 
 def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
-                force_generic: bool = False, stream=None):
+                force_generic: bool = False, segments: int = 0, stream=None):
     """SATs of a (batch, rows, cols) CUDA tensor, one launch for the batch."""
     import torch
     if x.dim() != 3:
@@ -168,7 +172,7 @@ def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: 
     if out is None:
         out = torch.empty_like(x)
     _check_dev(x, out)
-    o = options(r, tile_rows, force_generic)
+    o = options(r, tile_rows, force_generic, 0, segments)
     _check(_lib.sat_compute_batched(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                     x.shape[2], _dtype_code(x), VARIANTS[variant],
                                     ctypes.byref(o), _stream(stream)))
@@ -179,7 +183,8 @@ def _as3(x):
     return x if x.dim() == 3 else x.unsqueeze(0)
 
 
-def sat_widening(x, dtype, out=None, tile_rows: int = 0, force_generic: bool = False, stream=None):
+def sat_widening(x, dtype, out=None, tile_rows: int = 0, force_generic: bool = False, segments: int = 0,
+                 stream=None):
     """1R1W SAT of a uint8 (-> int32 sums) or float32 (-> float64 sums) CUDA
     tensor, 2-D or (batch, rows, cols), widened on load (no extra pass)."""
     import torch
@@ -187,7 +192,7 @@ def sat_widening(x, dtype, out=None, tile_rows: int = 0, force_generic: bool = F
     if out is None:
         out = torch.empty(x.shape, dtype=dtype, device=x.device)
     _check_dev(x, out)
-    o = options(0.25, tile_rows, force_generic)
+    o = options(0.25, tile_rows, force_generic, 0, segments)
     _check(_lib.sat_compute_widening(x.data_ptr(), _dtype_code(x), out.data_ptr(), _dtype_code(out),
                                      x3.shape[0], x3.shape[1], x3.shape[2], ctypes.byref(o),
                                      _stream(stream)))
@@ -226,16 +231,26 @@ def rect_sums(sat_t, rects, out=None, stream=None):
     return out
 
 
-def sat_seeded(x, carry_row=None, out=None, sat_row=None, stream=None):
+def sat_seeded(x, carry_row=None, out=None, sat_row=None, gathered=None, rank: int = 0, stream=None):
     """Rows of the SAT of a taller matrix: ``carry_row`` = column sums of
-    everything above ``x`` (or ``sat_row`` = the SAT row just above)."""
+    everything above ``x``; or ``gathered`` (nranks, cols) all-gathered column
+    totals of the strips of every rank, of which ranks < ``rank`` lie above
+    ``x`` (the sharded mode: the exclusive scan runs inside the SAT kernel);
+    or ``sat_row`` = the SAT row just above."""
     import torch
     if out is None:
         out = torch.empty_like(x)
-    _check_dev(x, out, carry_row, sat_row)
+    _check_dev(x, out, carry_row, sat_row, gathered)
     if sat_row is not None:
         _check(_lib.sat_compute_seeded_satrow(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                               _dtype_code(x), sat_row.data_ptr(), _stream(stream)))
+    elif gathered is not None:
+        g = gathered.view(-1, x.shape[1]) if gathered.dim() == 1 else gathered
+        if not (0 <= rank <= g.shape[0]):
+            raise ValueError("rank out of range")
+        _check(_lib.sat_compute_seeded_sum(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
+                                           _dtype_code(x), g.data_ptr(), int(rank), g.stride(0),
+                                           _stream(stream)))
     else:
         _check(_lib.sat_compute_seeded(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                        _dtype_code(x),
@@ -381,6 +396,16 @@ def ipc_open(handle: bytes) -> int:
 
 def ipc_close(ptr: int) -> None:
     _check(_lib.sat_ipc_close(ctypes.c_void_p(ptr)))
+
+
+def release_workspace(stream=None) -> None:
+    """Free libsat's workspace of ``stream`` (sat_release_workspace)."""
+    _check(_lib.sat_release_workspace(_stream(stream)))
+
+
+def set_tag_space(space: int) -> None:
+    """Tests only: shrink the look-back tag space (0 = default 2^30)."""
+    _check(_lib.sat_debug_set_tag_space(int(space)))
 
 
 def last_launch_count() -> int:

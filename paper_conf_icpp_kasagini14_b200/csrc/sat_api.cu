@@ -16,6 +16,8 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <atomic>
+#include <vector>
 #include <string>
 #include <utility>
 
@@ -104,6 +106,36 @@ struct Buf {
     size_t bytes = 0;
 };
 
+// look-back tags are 30 bits (band_tag); sat_debug_set_tag_space (tests only)
+// shrinks the space so the reset paths run
+std::atomic<unsigned long long> g_tag_space{1ull << 30};
+unsigned long long tag_space() { return g_tag_space.load(std::memory_order_relaxed); }
+
+struct Workspace {
+    Buf desc;                 // look-back descriptors (zeroed when (re)allocated)
+    Buf lseg;                 // band-segment row carries (zeroed when (re)allocated)
+    Buf ticket;               // [0] ticket counter, [1] device base (unsigned long long)
+    unsigned long long next_base = 0;
+    bool dev_epoch = false;   // once captured: every launch takes its base from the device (Sec. 4)
+    Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
+    Buf tr;                   // 4R4W transposed copy
+    Buf box;                  // box filter: the SAT it reads
+    Buf part;                 // column totals partials
+    Buf cnt;                  // column totals: per-chunk-column and global arrival counters (self-resetting)
+    Buf shard;                // sharded default workspace
+    Buf din, dout;            // host e2e device copies
+    std::vector<void*> retired;   // buffers a captured graph may still reference (freed by sat_release_workspace)
+    cudaStream_t cstream_in = nullptr, cstream_out = nullptr;
+};
+
+thread_local Workspace* t_ws = nullptr;   // the current call's workspace (for ensure())
+thread_local cudaStream_t t_st = nullptr; // the current call's stream
+
+// Grow a workspace buffer.  New memory is zeroed (when asked) with
+// cudaMemsetAsync on the call's stream, so the kernels queued after it on that
+// stream see zeros.  Once any call on the stream was captured into a CUDA
+// graph, an outgrown buffer is retired, not freed: a graph replay may still
+// reference it (freed by sat_release_workspace).
 int ensure(Buf& b, size_t bytes, bool zero) {
     if (b.bytes >= bytes && b.p) return SAT_OK;
     // a captured call cannot allocate (cudaMalloc / cudaMemset would break
@@ -111,40 +143,21 @@ int ensure(Buf& b, size_t bytes, bool zero) {
     if (t_capture)
         return fail(SAT_ERR_UNSUPPORTED, "stream capture needs a warm workspace: run the same call once "
                                          "on this stream before capturing it");
-    if (b.p) { cudaFree(b.p); b.p = nullptr; b.bytes = 0; }
+    if (b.p) {
+        if (t_ws && t_ws->dev_epoch) t_ws->retired.push_back(b.p);
+        else cudaFree(b.p);
+        b.p = nullptr;
+        b.bytes = 0;
+    }
     size_t want = std::max<size_t>(bytes, 256);
     if (cudaMalloc(&b.p, want) != cudaSuccess) {
         cudaGetLastError();
         return fail(SAT_ERR_NOMEM, "cudaMalloc of " + std::to_string(want) + " bytes failed");
     }
     b.bytes = want;
-    if (zero) CUDA_TRY(cudaMemset(b.p, 0, want));
+    if (zero) CUDA_TRY(cudaMemsetAsync(b.p, 0, want, t_st));
     return SAT_OK;
 }
-
-// look-back tags are 30 bits (band_tag); SAT_TAG_SPACE (tests only) shrinks
-// the space so the reset paths run
-unsigned long long tag_space() {
-    const char* e = getenv("SAT_TAG_SPACE");
-    const unsigned long long v = e ? strtoull(e, nullptr, 10) : 0ull;
-    return v > 0 && v < (1ull << 30) ? v : (1ull << 30);
-}
-
-struct Workspace {
-    Buf desc;                 // look-back descriptors (zeroed when (re)allocated)
-    Buf lseg;                 // band-segment row carries (zeroed when (re)allocated)
-    Buf ticket;               // [0] ticket counter, [1] device base, [2] reset flag (unsigned long long)
-    unsigned long long next_base = 0;
-    bool dev_epoch = false;   // once captured: every launch takes its base from the device (Sec. 4)
-    Buf bt, rs, lx, lsum, topx, lb;   // 2R1W family
-    Buf tr;                   // 4R4W transposed copy
-    Buf box;                  // box filter: the SAT it reads
-    Buf part;                 // column totals partials
-    Buf seedrow;              // seeded mode: SAT row above the strip
-    Buf shard;                // sharded default workspace
-    Buf din, dout;            // host e2e device copies
-    cudaStream_t cstream_in = nullptr, cstream_out = nullptr;
-};
 
 std::map<std::pair<int, void*>, Workspace*> g_ws;
 
@@ -156,7 +169,15 @@ int get_ws(int dev, cudaStream_t st, Workspace*& ws) {
     Workspace*& w = g_ws[{dev, reinterpret_cast<void*>(st)}];
     if (!w) w = new Workspace();
     ws = w;
+    t_ws = w;
+    t_st = st;
     return SAT_OK;
+}
+
+void free_buf(Buf& b) {
+    if (b.p) cudaFree(b.p);
+    b.p = nullptr;
+    b.bytes = 0;
 }
 
 // ------------------------------------------------------------------ helpers
@@ -240,244 +261,185 @@ struct BandCfg {
 // per compute thread.  Two CTAs per SM.
 constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 1, 2};
 constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
-constexpr BandCfg kCfg48{8, 6, 2, 4, 2, 4, 1, 2};
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
+// TH 64 with >= 4 waves of bands ("big"): one CTA per SM, 192 KB ring of
+// 64 x 256 slots (1-KB row segments), 6 chunks parked in TMEM
+constexpr BandCfg kCfg64B{8, 8, 3, 6, 2, 4, 1, 1};
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
 constexpr int kLbw128 = 2;   // look-back window (bands per round trip) at TH = 128:
                              // 2 measured ~1 % faster than 4 at 16384^2/18432^2, 8 slower
-// TH = 112: 14 compute warps, one CTA per SM; fills the SMs where TH = 128
-// leaves a partial wave (16384 rows: 147 bands on 148 SMs instead of 128)
-constexpr BandCfg kCfg112{8, 14, 3, 4, 1, 3, 1, 1};
 // float64 (8-byte elements: 1 KB chunk rows, two TMEM words per element)
 constexpr BandCfg kCfgD16{2, 8, 4, 4, 1, 3, 1, 2};   //  96 KB smem, 128 TMEM cols: 2 CTAs/SM
 constexpr BandCfg kCfgD32{4, 8, 4, 8, 1, 4, 1, 1};   // 192 KB smem, 512 TMEM cols
-constexpr BandCfg kCfgD48{8, 6, 3, 4, 1, 4, 1, 1};   // 168 KB smem, 512 TMEM cols
 // TH 64: ONE control group of 2 warps that split the columns (NS = 2: 2
 // columns per lane, 4 descriptor words per band, look-back window 4):
 // 16384^2 0.917 vs 1.04 ms with 3 groups of 1 warp, 32768^2 3.49 vs 3.87
 constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM cols
+// uint8 input widened to uint32 sums: the ring holds bytes (TH x 128 B per
+// chunk), so it is 6 slots deep
+constexpr BandCfg kCfgU64{8, 8, 6, 4, 1, 4, 1, 2};
+constexpr BandCfg kCfgU128{8, 16, 6, 4, 1, 3, 1, 1};
 
 // CTAs per SM of a configuration (for wave counts before launch)
 int ctas_per_sm(int dtype, int th, bool big) {
     if (dtype == SAT_FLOAT64) return th == 16 ? 2 : 1;
-    return (th >= 112 || big) ? 1 : 2;
+    return (th >= 128 || big) ? 1 : 2;
 }
 
+// One-time per (instantiation, device) launch set-up, shared by all threads.
+struct KernelSetup {
+    std::once_flag once[kMaxDev];
+    cudaFuncAttributes fa[kMaxDev];
+    cudaError_t err[kMaxDev] = {};
+};
+
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int CL = 1, int LBW = 0, typename TI = T>
-int launch_band_t(const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
-                  const DevInfo& di, cudaStream_t st, int& grid_out) {
-    (void)to;
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, CL, MODE, TMA, MINB, LBW, TI>;
-    const size_t smem = BandSmem<T, R, W, S, DT, SUB, CL, TI>::total;
+          int LBW = 0, typename TI = T>
+int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st, int& grid_out) {
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI>;
+    const size_t smem = BandSmem<T, R, W, S, DT, SUB, TI>::total;
     const int threads = (W + NCW + 1) * 32;
-    // per instantiation and device: attributes set once, resources queried once
-    // (a per-call cudaFuncGetAttributes was a visible part of the ~15 us host
-    // cost of a small call)
-    static int configured[kMaxDev] = {};
-    static cudaFuncAttributes fa_dev[kMaxDev];
+    // per instantiation and device: attributes set once, resources queried
+    // once (a per-call cudaFuncGetAttributes was a visible part of the ~15 us
+    // host cost of a small call); std::call_once orders the set-up before any
+    // thread's launch
+    static KernelSetup setup;
     int dev = 0;
     CUDA_TRY(cudaGetDevice(&dev));
     if (dev < 0 || dev >= kMaxDev) return fail(SAT_ERR_CUDA, "device ordinal out of range");
-    if (!configured[dev]) {
-        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
-        CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                      int(cudaSharedmemCarveoutMaxShared)));
-        CUDA_TRY(cudaFuncGetAttributes(&fa_dev[dev], kern));
-        configured[dev] = 1;
-    }
+    std::call_once(setup.once[dev], [&] {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                     int(cudaSharedmemCarveoutMaxShared));
+        if (e == cudaSuccess) e = cudaFuncGetAttributes(&setup.fa[dev], kern);
+        setup.err[dev] = e;
+    });
+    if (setup.err[dev] != cudaSuccess)
+        return fail(SAT_ERR_CUDA, std::string("band kernel set-up: ") + cudaGetErrorString(setup.err[dev]));
     // Resident CTAs per SM, from the kernel's own resources.  (The runtime's
     // occupancy query reports 1 for kernels that allocate tensor memory; two
     // CTAs of ours fit: TC::alloc <= 256 columns of the SM's 512.)
-    const cudaFuncAttributes& fa = fa_dev[dev];
+    const cudaFuncAttributes& fa = setup.fa[dev];
     const int warps = threads / 32;
     const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
-    int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
-                        di.smem_sm / int(smem + fa.sharedSizeBytes + 1024),
-                        MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT, int(sizeof(T) / 4)>::alloc, 32});
+    const int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
+                              di.smem_sm / int(smem + fa.sharedSizeBytes + 1024),
+                              MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT, int(sizeof(T) / 4)>::alloc, 32});
     if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
-    if (const char* e = getenv("SAT_DEBUG_OCC")) occ = atoi(e);
-    if constexpr (CL > 1) {
-        // clusters of CL CTAs (CL consecutive bands); persistent, one ticket
-        // per cluster.  Clusters that cannot be co-resident simply start
-        // late and find no ticket left.
-        long long ncl = std::min<long long>(p.total_units, (long long)occ * di.sms / CL);
-        if (const char* e = getenv("SAT_DEBUG_NCL")) ncl = atoi(e);
-        if (ncl < 1) ncl = 1;
-        const long long grid = ncl * CL;
-        grid_out = int(grid);
-        t_grid = int(grid);
-        cudaLaunchConfig_t cfg;
-        std::memset(&cfg, 0, sizeof(cfg));
-        cfg.gridDim = dim3(unsigned(grid));
-        cfg.blockDim = dim3(unsigned(threads));
-        cfg.dynamicSmemBytes = smem;
-        cfg.stream = st;
-        cudaLaunchAttribute attr[1];
-        attr[0].id = cudaLaunchAttributeClusterDimension;
-        attr[0].val.clusterDim.x = CL;
-        attr[0].val.clusterDim.y = 1;
-        attr[0].val.clusterDim.z = 1;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
-        CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ti, p));
-    } else {
-        long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
-        if (grid < 1) grid = 1;
-        grid_out = int(grid);
-        t_grid = int(grid);
-        // programmatic dependent launch: the CTA prologue (barriers, TMEM
-        // alloc) overlaps the previous kernel's tail; the kernel waits
-        // (griddepcontrol.wait) before its first global access.  Back-to-back
-        // calls: 1024^2 16.7 -> 14.4 us, 4096^2 f32 47.9 -> 45.5 us
-        // (profiles/r01_pdl_ab.txt).  SAT_PDL=0 turns it off.
-        static const bool pdl = [] { const char* e = getenv("SAT_PDL"); return !e || atoi(e) != 0; }();
-        if (pdl) {
-            cudaLaunchConfig_t cfg;
-            std::memset(&cfg, 0, sizeof(cfg));
-            cfg.gridDim = dim3(unsigned(grid));
-            cfg.blockDim = dim3(unsigned(threads));
-            cfg.dynamicSmemBytes = smem;
-            cfg.stream = st;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-            attr[0].val.programmaticStreamSerializationAllowed = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ti, p));
-        } else {
-            kern<<<int(grid), threads, smem, st>>>(ti, p);
-        }
-    }
+    long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
+    if (grid < 1) grid = 1;
+    grid_out = int(grid);
+    t_grid = int(grid);
+    // programmatic dependent launch: the CTA prologue (barriers, TMEM alloc)
+    // overlaps the previous kernel's tail; the kernel waits
+    // (griddepcontrol.wait) before its first global access.  Back-to-back
+    // calls: 1024^2 16.7 -> 14.4 us, 4096^2 f32 47.9 -> 45.5 us
+    // (profiles/r01_pdl_ab.txt)
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(unsigned(grid));
+    cfg.blockDim = dim3(unsigned(threads));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, ti, p));
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     return SAT_OK;
 }
 
 #define SAT_CFG(c) c.R, c.W, c.S, c.DT, c.SUB, c.NCW, c.NS
+// Band heights instantiated per (dtype, mode, path); `band_th` maps a
+// requested height onto them.  1R1W family (MODE_SAT) on the TMA path: int32 /
+// float32 16, 32, 64, 128 (+ the "big" TH-64 configuration), float64 16, 32,
+// 64; the column and row passes of 2R2W / 4R4W: 32 and 64; the generic
+// (non-TMA) path: 32 (and 128 for 4-byte 1R1W).
+int band_th(int mode, int dtype, bool tma, int th) {
+    if (!tma) {
+        if (mode == MODE_SAT && dtype != SAT_FLOAT64 && th >= 128) return 128;
+        return 32;
+    }
+    if (mode != MODE_SAT) return th >= 64 ? 64 : 32;
+    if (dtype == SAT_FLOAT64) return th >= 64 ? 64 : th >= 32 ? 32 : 16;
+    return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
+}
+
 template <typename T, int MODE, bool TMA>
-int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
-                   const DevInfo& di, cudaStream_t st, int& grid) {
-    if constexpr (MODE == MODE_SAT && TMA && std::is_same<T, uint32_t>::value) {
-        // debug: column split of the control warps (SAT_DEBUG_CFG=1|2|4 -> NS)
-        if (const char* e = getenv("SAT_DEBUG_CFG")) {
-            const int ns = atoi(e);
-            if (th == 64 && ns == 2) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 64 && ns == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 32 && ns == 2) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 32 && ns == 4) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 4, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            // one group of two column-splitting control warps (as float64 TH 64)
-            if (th == 16 && ns == 22) return launch_band_t<T, 4, 4, 3, 8, 4, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 32 && ns == 22) return launch_band_t<T, 8, 4, 3, 8, 2, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 64 && ns == 22) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
-            if (th == 48 && ns == 22) return launch_band_t<T, 8, 6, 2, 4, 2, 2, 2, MODE, TMA, 2>(p, ti, to, di, st, grid);
+int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st,
+                   int& grid) {
+    if constexpr (!TMA) {
+        if constexpr (MODE == MODE_SAT && sizeof(T) == 4)
+            if (th == 128) return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, di, st, grid);
+        if constexpr (sizeof(T) == 8)
+            return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
+        else
+            return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
+    } else if constexpr (MODE != MODE_SAT) {
+        if constexpr (sizeof(T) == 8) {
+            if (th == 64) return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
+            return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
+        } else {
+            if (th == 64) return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, di, st, grid);
+            return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
         }
-    }
-    if constexpr (sizeof(T) == 8) {
-        if constexpr (MODE == MODE_SAT && TMA) {
-            if (const char* e = getenv("SAT_DEBUG_F64")) {   // A/B of the float64 look-back
-                const int v = atoi(e);
-                if (th == 64 && v == 1) return launch_band_t<T, 8, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 2) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 3) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 1, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 4) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 5) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 6) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 7) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 4, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 8) return launch_band_t<T, 8, 8, 3, 4, 1, 4, 2, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 9) return launch_band_t<T, 8, 8, 3, 4, 1, 1, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 10) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (th == 64 && v == 11) return launch_band_t<T, 8, 8, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
-                if (th == 32 && v == 6) return launch_band_t<T, 4, 8, 4, 8, 1, 2, 2, MODE, TMA, 1, 1, 0>(p, ti, to, di, st, grid);
-            }
-        }
+    } else if constexpr (sizeof(T) == 8) {
         switch (th) {
-            case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, to, di, st, grid);
-            case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, to, di, st, grid);
-            case 48: return launch_band_t<T, SAT_CFG(kCfgD48), MODE, TMA, kCfgD48.MINB>(p, ti, to, di, st, grid);
-            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, to, di, st, grid);
+            case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, di, st, grid);
+            case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
         }
-        return fail(SAT_ERR_INVALID, "float64: tile_rows must be 16, 32, 48 or 64");
+        return fail(SAT_ERR_INVALID, "float64: no band configuration for this tile_rows");
     } else {
-    if constexpr (MODE == MODE_SAT && TMA) {
-        if (p.big && th == 64) {  // 192 KB ring of 64 x 256 slots, 6 chunks parked in TMEM
-            if (const char* e = getenv("SAT_DEBUG_LBW")) {
-                const int lbw = atoi(e);
-                if (lbw == 8) return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
-                if (lbw == 12) return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1, 1, 12>(p, ti, to, di, st, grid);
-                if (lbw == 83) return launch_band_t<T, 8, 8, 3, 6, 2, 8, 2, MODE, TMA, 1, 1, 8>(p, ti, to, di, st, grid);
-            }
-            return launch_band_t<T, 8, 8, 3, 6, 2, 4, 1, MODE, TMA, 1>(p, ti, to, di, st, grid);
+        if (p.big && th == 64) return launch_band_t<T, SAT_CFG(kCfg64B), MODE, TMA, kCfg64B.MINB>(p, ti, di, st, grid);
+        switch (th) {
+            case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, di, st, grid);
+            case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, di, st, grid);
+            case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
         }
-        if (th == 128) {   // A/B of the look-back window (8 and NS = 2 measured slower)
-            if (const char* e = getenv("SAT_DEBUG_LBW")) {
-                const int lbw = atoi(e);
-                if (lbw == 4) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 4>(p, ti, to, di, st, grid);
-                if (lbw == 1) return launch_band_t<T, 8, 16, 3, 4, 1, 3, 1, MODE, TMA, 1, 1, 1>(p, ti, to, di, st, grid);
-                if (lbw == 22) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (lbw == 12) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 1, MODE, TMA, 1, 1, 2>(p, ti, to, di, st, grid);
-                if (lbw == 24) return launch_band_t<T, 8, 16, 3, 4, 1, 2, 2, MODE, TMA, 1, 1, 4>(p, ti, to, di, st, grid);
-            }
-        }
-        if (p.cluster == 8 && th == 64)
-            return launch_band_t<T, 8, 8, 3, 3, 1, 3, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
-        if (p.cluster == 8 && th == 48)
-            return launch_band_t<T, 8, 6, 2, 4, 2, 4, 1, MODE, TMA, 2, 8>(p, ti, to, di, st, grid);
-    }
-    switch (th) {
-        case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, to, di, st, grid);
-        case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, to, di, st, grid);
-        case 48: return launch_band_t<T, SAT_CFG(kCfg48), MODE, TMA, kCfg48.MINB>(p, ti, to, di, st, grid);
-        case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, to, di, st, grid);
-        case 112: return launch_band_t<T, SAT_CFG(kCfg112), MODE, TMA, kCfg112.MINB>(p, ti, to, di, st, grid);
-        case 128:
-            if constexpr (MODE == MODE_SAT)
-                return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, 1, kLbw128>(p, ti, to, di, st, grid);
-            else
-                return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB>(p, ti, to, di, st, grid);
-    }
-    return fail(SAT_ERR_INVALID, "tile_rows must be 16, 32, 48, 64, 112 or 128");
+        return fail(SAT_ERR_INVALID, "no band configuration for this tile_rows");
     }
 }
 
 // Widening 1R1W: uint8 -> uint32 and float32 -> float64.
 template <typename T, typename TI, bool TMA>
-int launch_band_widen(int th, const BandParams& p, const CUtensorMap& ti, const CUtensorMap& to,
-                      const DevInfo& di, cudaStream_t st, int& grid) {
+int launch_band_widen(int th, const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st,
+                      int& grid) {
     if constexpr (sizeof(TI) == 1) {
-        if (th == 128) {
-            if (getenv("SAT_DEBUG_U8LBW4"))
-                return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, 0, TI>(p, ti, to, di, st, grid);
-            return launch_band_t<T, 8, 16, 6, 4, 1, 3, 1, MODE_SAT, TMA, 1, 1, kLbw128, TI>(p, ti, to, di, st, grid);
+        if constexpr (TMA) {
+            if (th == 128) return launch_band_t<T, SAT_CFG(kCfgU128), MODE_SAT, TMA, 1, kLbw128, TI>(p, ti, di, st, grid);
         }
-        if (th == 64) return launch_band_t<T, 8, 8, 6, 4, 1, 4, 1, MODE_SAT, TMA, 2, 1, 0, TI>(p, ti, to, di, st, grid);
-        return fail(SAT_ERR_INVALID, "uint8 input: tile_rows must be 64 or 128");
+        return launch_band_t<T, SAT_CFG(kCfgU64), MODE_SAT, TMA, 2, 0, TI>(p, ti, di, st, grid);
     } else {
-        switch (th) {
-            case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE_SAT, TMA, kCfgD16.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
-            case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE_SAT, TMA, kCfgD32.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
-            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE_SAT, TMA, kCfgD64.MINB, 1, 0, TI>(p, ti, to, di, st, grid);
+        if constexpr (TMA) {
+            if (th == 16) return launch_band_t<T, SAT_CFG(kCfgD16), MODE_SAT, TMA, kCfgD16.MINB, 0, TI>(p, ti, di, st, grid);
+            if (th == 64) return launch_band_t<T, SAT_CFG(kCfgD64), MODE_SAT, TMA, kCfgD64.MINB, 0, TI>(p, ti, di, st, grid);
         }
-        return fail(SAT_ERR_INVALID, "float32 -> float64: tile_rows must be 16, 32 or 64");
+        return launch_band_t<T, SAT_CFG(kCfgD32), MODE_SAT, TMA, kCfgD32.MINB, 0, TI>(p, ti, di, st, grid);
     }
 }
 
 template <typename T, int MODE>
-int launch_band_m(bool tma, int th, const BandParams& p, const CUtensorMap& ti,
-                  const CUtensorMap& to, const DevInfo& di, cudaStream_t st, int& grid) {
-    return tma ? launch_band_th<T, MODE, true>(th, p, ti, to, di, st, grid)
-               : launch_band_th<T, MODE, false>(th, p, ti, to, di, st, grid);
+int launch_band_m(bool tma, int th, const BandParams& p, const CUtensorMap& ti, const DevInfo& di,
+                  cudaStream_t st, int& grid) {
+    return tma ? launch_band_th<T, MODE, true>(th, p, ti, di, st, grid)
+               : launch_band_th<T, MODE, false>(th, p, ti, di, st, grid);
 }
 
 template <typename T>
-int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtensorMap& ti,
-                  const CUtensorMap& to, const DevInfo& di, cudaStream_t st, int& grid) {
+int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtensorMap& ti, const DevInfo& di,
+                  cudaStream_t st, int& grid) {
     switch (mode) {
-        case MODE_SAT: return launch_band_m<T, MODE_SAT>(tma, th, p, ti, to, di, st, grid);
-        case MODE_COL: return launch_band_m<T, MODE_COL>(tma, th, p, ti, to, di, st, grid);
-        case MODE_ROW: return launch_band_m<T, MODE_ROW>(tma, th, p, ti, to, di, st, grid);
+        case MODE_SAT: return launch_band_m<T, MODE_SAT>(tma, th, p, ti, di, st, grid);
+        case MODE_COL: return launch_band_m<T, MODE_COL>(tma, th, p, ti, di, st, grid);
+        case MODE_ROW: return launch_band_m<T, MODE_ROW>(tma, th, p, ti, di, st, grid);
     }
     return fail(SAT_ERR_INVALID, "bad mode");
 }
@@ -524,6 +486,7 @@ struct Job {
     int th;
     bool tma;
     int jitter;
+    int segments;     // sat_options.segments: 0 = automatic band segments
     const DevInfo* di;
     Workspace* ws;
     cudaStream_t st;
@@ -550,8 +513,18 @@ __global__ void sat_epoch_kernel(unsigned long long* tk, unsigned long long wors
     }
 }
 
+// The band height a launch actually uses (the instantiated configurations).
+int eff_th(const Job& j, int mode) {
+    if (j.in_dtype == SAT_UINT8) return (j.tma && j.th >= 128) ? 128 : 64;
+    if (j.in_dtype != j.dtype) return j.tma ? (j.th >= 64 ? 64 : j.th >= 32 ? 32 : 16) : 32;
+    return band_th(mode, j.dtype, j.tma, j.th);
+}
+
 // One band-kernel launch with ticket/tag bookkeeping.
-int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
+int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
+    Job j = j0;
+    j.th = eff_th(j0, mode);
+    t_th = j.th;
     // The ticket base and the descriptor tags come from a host-side counter
     // advanced per launch.  A captured launch replayed from a CUDA graph would
     // reuse a host value, so under capture (and on this workspace from then
@@ -572,29 +545,16 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * ((p.nc + p.tile_units - 1) / p.tile_units)
                                  : p.total_bands;
-    // Clusters of 8 bands that pass the vertical carry through DSMEM (DESIGN.md
-    // Sec. 4.5) are correct but measured slower than the plain look-back, so
-    // they are opt-in (SAT_CLUSTER=8) for plain 1R1W on the TMA path.
-    p.cluster = 1;
-    if (const char* e = getenv("SAT_CLUSTER")) {
-        if (atoi(e) == 8 && mode == MODE_SAT && j.tma && p.region == REG_ALL && j.dtype != SAT_FLOAT64 &&
-            p.top_src == TOP_LOOKBACK && !p.tile_units && (j.th == 64 || j.th == 48))
-            p.cluster = 8;
-    }
     // Many bands (>= 4 waves of one CTA per SM): one CTA per SM with twice the
     // ring and 1-KB row segments per TMA load.
-    p.big = (mode == MODE_SAT && j.tma && p.cluster == 1 && j.th == 64 && j.dtype != SAT_FLOAT64 &&
+    p.big = (mode == MODE_SAT && j.tma && j.th == 64 && j.dtype != SAT_FLOAT64 && j.in_dtype == j.dtype &&
              p.total_bands >= 4 * j.di->sms) ? 1 : 0;
-    if (const char* e = getenv("SAT_BIG")) p.big = (atoi(e) != 0 && mode == MODE_SAT && j.tma &&
-                                                    p.cluster == 1 && j.th == 64 && j.dtype != SAT_FLOAT64) ? 1 : 0;
-    if (p.cluster > 1)
-        p.total_units = (long long)j.batch * ((p.nb + p.cluster - 1) / p.cluster);
     // Band segments: short units for the last wave when
     // bands are many waves deep
     p.nseg = 1;
     p.segc = p.nc;
     if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && p.region == REG_ALL && !p.tile_units &&
-        p.cluster == 1 && p.Lx == nullptr && p.Lb == nullptr) {
+        p.Lx == nullptr && p.Lb == nullptr) {
         // more bands than resident CTAs: up to 16 segments of >= 16 chunks, so
         // the partial last wave of whole bands becomes many short units
         // (65536^2 TH 128: 5.97 ms with 16 segments vs 6.34 ms whole bands;
@@ -603,7 +563,7 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         // the band's previous segment)
         const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0);
         int want = p.total_bands > slots ? std::min(16, p.nc / 16) : 1;
-        if (const char* e = getenv("SAT_SEG")) want = std::max(1, atoi(e));
+        if (j.segments > 0) want = j.segments;
         if (want > 1 && p.nc > 1) {
             p.segc = (p.nc + want - 1) / want;
             p.nseg = (p.nc + p.segc - 1) / p.segc;
@@ -611,14 +571,12 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
         }
     }
     p.jitter = j.jitter;
-    p.pf = 0;
-    if (const char* e = getenv("SAT_PF")) p.pf = std::max(0, atoi(e));
-    if (const char* e = getenv("SAT_UNIT_SYNC")) p.unit_sync = atoi(e) != 0;
-    p.diag = g_diag_dev;
-    if (const char* e = getenv("SAT_DEBUG_NOLB")) p.dbg = atoi(e);   // 1: no look-back, 2: publish only
-    if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
-        p.trace = t_trace;
-        t_trace = nullptr;
+    if (kDebug) {
+        p.diag = g_diag_dev;
+        if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
+            p.trace = t_trace;
+            t_trace = nullptr;
+        }
     }
     Workspace& ws = *j.ws;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
@@ -650,27 +608,25 @@ int run_band(const Job& j, int mode, const void* in, void* out, BandParams p) {
     p.Lseg = static_cast<uint64_t*>(ws.lseg.p);
     p.ticket = static_cast<unsigned long long*>(ws.ticket.p);
     p.base = ws.next_base;
-    CUtensorMap ti, to;
+    CUtensorMap ti;
     std::memset(&ti, 0, sizeof(ti));
-    std::memset(&to, 0, sizeof(to));
     if (j.tma) {
         SAT_TRY(make_tmap(&ti, in, j.in_dtype, j.batch, j.rows, j.cols, j.th));
     }
     int grid = 0;
     int s;
     if (j.in_dtype == SAT_UINT8)
-        s = j.tma ? launch_band_widen<uint32_t, uint8_t, true>(j.th, p, ti, to, *j.di, j.st, grid)
-                  : launch_band_widen<uint32_t, uint8_t, false>(j.th, p, ti, to, *j.di, j.st, grid);
+        s = j.tma ? launch_band_widen<uint32_t, uint8_t, true>(j.th, p, ti, *j.di, j.st, grid)
+                  : launch_band_widen<uint32_t, uint8_t, false>(j.th, p, ti, *j.di, j.st, grid);
     else if (j.in_dtype != j.dtype)
-        s = j.tma ? launch_band_widen<double, float, true>(j.th, p, ti, to, *j.di, j.st, grid)
-                  : launch_band_widen<double, float, false>(j.th, p, ti, to, *j.di, j.st, grid);
+        s = j.tma ? launch_band_widen<double, float, true>(j.th, p, ti, *j.di, j.st, grid)
+                  : launch_band_widen<double, float, false>(j.th, p, ti, *j.di, j.st, grid);
     else
-        s = SAT_DISPATCH(j.dtype, T, launch_band_d<T>(mode, j.tma, j.th, p, ti, to, *j.di, j.st, grid));
+        s = SAT_DISPATCH(j.dtype, T, launch_band_d<T>(mode, j.tma, j.th, p, ti, *j.di, j.st, grid));
     if (s != SAT_OK) return s;
-    // every persistent ticket taker (a CTA, or a cluster) makes exactly one
-    // failing fetch, so the counter ends at base + units + takers
-    const unsigned long long takers = (unsigned long long)(p.cluster > 1 ? grid / p.cluster : grid);
-    ws.next_base += units + takers;
+    // every persistent ticket taker (a CTA) makes exactly one failing fetch,
+    // so the counter ends at base + units + takers
+    ws.next_base += units + (unsigned long long)grid;
     return SAT_OK;
 }
 
@@ -739,7 +695,6 @@ int run_2r1w_region_t(const Job& j, const Carry2r1w& c, int region, int tA, cons
     // ranges above (16384^2 2R1W 0.657 -> 0.625 ms); 16-chunk ranges for the
     // (1+r)R1W triangles, whose top bands are long (16384^2 0.952 -> 0.705 ms)
     p.tile_units = region == REG_ALL ? (c.nc >= 64 ? 8 : 0) : 16;
-    if (const char* e = getenv("SAT_TILE_UNITS")) p.tile_units = std::max(0, atoi(e));
     p.region = region;
     p.tA = tA;
     p.Lx = ws.lx.p;
@@ -779,7 +734,7 @@ template <typename T>
 int transpose_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols, cudaStream_t st) {
     const uintptr_t al = 2 * sizeof(T) - 1;
     if (rows % 2 == 0 && cols % 2 == 0 && !(reinterpret_cast<uintptr_t>(in) & al) &&
-        !(reinterpret_cast<uintptr_t>(out) & al) && !getenv("SAT_TRANSPOSE32")) {
+        !(reinterpret_cast<uintptr_t>(out) & al)) {
         const int64_t ntr = (rows + 63) / 64;
         const dim3 grid(unsigned((cols + 63) / 64), unsigned(std::min<int64_t>(ntr, 65535)), unsigned(batch));
         sat_transpose64_kernel<T><<<grid, 256, 0, st>>>(static_cast<const T*>(in), static_cast<T*>(out),
@@ -835,22 +790,25 @@ int run_4r1w_t(const Job& j) {
 }
 
 // ------------------------------------------------------------------ core driver
+// satrow: SAT row just above the matrix (SEED_SATROW), cs: column-sum seed of
+// image 0 (sat_common.h ColSeed); both 1R1W only.
 int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
-                 int dtype, int variant, const sat_options* opt, const void* seed,
-                 int seed_kind, cudaStream_t st, int in_dtype = -1) {
+                 int dtype, int variant, const sat_options* opt, const void* satrow,
+                 const ColSeed* cs, cudaStream_t st, int in_dtype = -1) {
     t_launches = 0;
     if (in_dtype < 0) in_dtype = dtype;
     SAT_TRY(validate(in, out, batch, rows, cols, dtype, true, in_dtype));
     if (variant < SAT_2R2W || variant > SAT_4R1W) return fail(SAT_ERR_INVALID, "bad variant");
-    if (in_dtype != dtype && (variant != SAT_1R1W || seed))
+    const bool seeded = satrow != nullptr || (cs && cs->n > 0);
+    if (in_dtype != dtype && (variant != SAT_1R1W || seeded))
         return fail(SAT_ERR_UNSUPPORTED, "widening input: unseeded 1R1W only");
     sat_options o;
     sat_options_init(&o);
     if (opt) o = *opt;
-    if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 48 &&
-        o.tile_rows != 64 && o.tile_rows != 112 && o.tile_rows != 128)
-        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 48, 64, 112 or 128");
+    if (o.tile_rows != 0 && o.tile_rows != 16 && o.tile_rows != 32 && o.tile_rows != 64 && o.tile_rows != 128)
+        return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 64 or 128");
     if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
+    if (o.segments < 0) return fail(SAT_ERR_INVALID, "segments must be >= 0");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     int dev;
     DevInfo di;
@@ -861,36 +819,30 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     j.in = in; j.out = out; j.batch = batch; j.rows = rows; j.cols = cols; j.dtype = dtype;
     j.in_dtype = in_dtype;
     j.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
-    if (in_dtype == SAT_UINT8 && !o.tile_rows) j.th = j.th == 128 ? 128 : 64;
     j.tma = !o.force_generic && tma_ok(in, out, cols, in_dtype);
     j.jitter = o.jitter;
+    j.segments = o.segments;
     j.di = &di;
     j.ws = ws;
     j.st = st;
+    // the 1R1W family's band height (2R1W Steps 1-2 size their carries by it)
+    j.th = eff_th(j, MODE_SAT);
     t_th = j.th;
     switch (variant) {
         case SAT_1R1W: {
             BandParams p = base_params();
-            if (seed && seed_kind == SEED_COLSUM) {
-                // column sums above the strip -> the SAT row just above it
-                SAT_TRY(ensure(ws->seedrow, size_t(cols) * esize(dtype), false));
-                SAT_DISPATCH(dtype, T, (sat_row_prefix_kernel<T><<<1, 1024, 0, st>>>(
-                                            static_cast<const T*>(seed), static_cast<T*>(ws->seedrow.p), cols),
-                                        0));
-                CUDA_TRY(cudaGetLastError());
-                ++t_launches;
-                seed = ws->seedrow.p;
-            }
-            p.seed = seed;
-            p.seed_kind = seed ? SEED_SATROW : SEED_NONE;
+            if (cs && cs->n > 0) p.cseed = *cs;
+            p.seed = satrow;
+            p.seed_kind = satrow ? SEED_SATROW : SEED_NONE;
             return run_band(j, MODE_SAT, in, out, p);
         }
         case SAT_2R2W: {
             // column-wise prefix-sums (look-back down the columns), then
             // row-wise prefix-sums (rows independent)
-            BandParams p = base_params();
-            SAT_TRY(run_band(j, MODE_COL, in, out, p));
-            Job j2 = j;
+            Job j1 = j;
+            j1.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
+            SAT_TRY(run_band(j1, MODE_COL, in, out, base_params()));
+            Job j2 = j1;
             j2.tma = !o.force_generic && tma_ok(out, out, cols);
             return run_band(j2, MODE_ROW, out, out, base_params());
         }
@@ -934,22 +886,26 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     return fail(SAT_ERR_INVALID, "bad variant");
 }
 
+// Column totals in one launch (sat_xchg.cuh sat_colsum_kernel); push = the
+// fused exchange's epilogue.
 template <typename T>
 int column_totals_t(const void* in, void* totals, int64_t rows, int64_t cols, const DevInfo& di,
-                    Workspace& ws, cudaStream_t st) {
+                    Workspace& ws, cudaStream_t st, const XchgParams* x) {
     const int nc = int((cols + TW - 1) / TW);
     long long splits = std::max<long long>(1, (4LL * di.sms + nc - 1) / nc);
-    splits = std::min<long long>(splits, (rows + 63) / 64);
-    if (splits < 1) splits = 1;
-    const int64_t seg = (rows + splits - 1) / splits;
-    splits = (rows + seg - 1) / seg;
+    splits = std::min<long long>(splits, std::max<int64_t>(1, (rows + 63) / 64));
+    const int64_t seg = std::max<int64_t>(1, (rows + splits - 1) / splits);
+    if (rows > 0) splits = (rows + seg - 1) / seg;
     SAT_TRY(ensure(ws.part, size_t(splits) * nc * TW * sizeof(T), false));
-    sat_colsum_partial_kernel<T><<<dim3(nc, unsigned(splits)), 256, 0, st>>>(
-        static_cast<const T*>(in), static_cast<T*>(ws.part.p), rows, cols, seg);
-    CUDA_TRY(cudaGetLastError());
-    ++t_launches;
-    sat_colsum_final_kernel<T><<<unsigned((cols + 255) / 256), 256, 0, st>>>(
-        static_cast<const T*>(ws.part.p), static_cast<T*>(totals), cols, int(splits), nc * TW);
+    SAT_TRY(ensure(ws.cnt, size_t(nc + 1) * sizeof(unsigned int), true));
+    TotalsParams tp;
+    std::memset(&tp, 0, sizeof(tp));
+    tp.in = in; tp.rows = rows; tp.cols = cols; tp.seg_rows = seg; tp.splits = int(splits);
+    tp.part = ws.part.p;
+    tp.cnt = static_cast<unsigned int*>(ws.cnt.p);
+    tp.totals = totals;
+    if (x) { tp.push = 1; tp.x = *x; }
+    sat_colsum_kernel<T><<<dim3(nc, unsigned(splits)), 256, 0, st>>>(tp);
     CUDA_TRY(cudaGetLastError());
     ++t_launches;
     return SAT_OK;
@@ -962,7 +918,7 @@ int column_totals_core(const void* in, void* totals, int64_t rows, int64_t cols,
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
-    return SAT_DISPATCH(dtype, T, column_totals_t<T>(in, totals, rows, cols, di, *ws, st));
+    return SAT_DISPATCH(dtype, T, column_totals_t<T>(in, totals, rows, cols, di, *ws, st, nullptr));
 }
 
 int exscan_core(const void* gathered, void* carry, int64_t nranks, int64_t cols, int rank,
@@ -983,7 +939,8 @@ struct PeerExchange {
     int rank, nranks, dtype;
     int64_t cols;
     XchgParams x;             // epoch advanced per call
-    unsigned int* done;       // device block counter
+    unsigned int* done;       // device counter: band-0 units that finished reading the slots
+    uint64_t** acks;          // device [nranks]: &peers[q].ack[rank] for q < rank
 };
 
 template <typename T>
@@ -1001,39 +958,32 @@ int sharded_fused_t(const void* in, void* out, int64_t strip_rows, PeerExchange&
     int launches = 0;
     if (ex.rank < ex.nranks - 1) {
         // 1. strip column totals; the epilogue pushes them into the higher
-        //    ranks' mailboxes and raises their flags
-        const int nc = int((cols + TW - 1) / TW);
-        long long splits = 0;
-        if (strip_rows > 0) {
-            splits = std::max<long long>(1, (4LL * di.sms + nc - 1) / nc);
-            splits = std::min<long long>(splits, (strip_rows + 63) / 64);
-            const int64_t seg = (strip_rows + splits - 1) / splits;
-            splits = (strip_rows + seg - 1) / seg;
-            SAT_TRY(ensure(ws->part, size_t(splits) * nc * TW * sizeof(T), false));
-            sat_colsum_partial_kernel<T><<<dim3(nc, unsigned(splits)), 256, 0, st>>>(
-                static_cast<const T*>(in), static_cast<T*>(ws->part.p), strip_rows, cols, seg);
-            CUDA_TRY(cudaGetLastError());
-            ++launches;
-        }
-        const unsigned blocks = unsigned(std::min<int64_t>((cols + 255) / 256, 4LL * di.sms));
-        sat_colsum_push_kernel<T><<<blocks, 256, 0, st>>>(static_cast<const T*>(ws->part.p), cols, int(splits),
-                                                          nc * TW, ex.x);
+        //    ranks' mailboxes and raises their flags (ONE launch)
+        t_launches = 0;
+        SAT_TRY(column_totals_t<T>(in, nullptr, strip_rows, cols, di, *ws, st, &ex.x));
+        launches += t_launches;
+    }
+    if (ex.rank > 0 && strip_rows == 0) {
+        sat_xchg_drain_kernel<<<1, 32, 0, st>>>(ex.x);
         CUDA_TRY(cudaGetLastError());
         ++launches;
     }
-    const void* seed = nullptr;
-    if (ex.rank > 0) {
-        // 2. wait for ranks < p, exscan in rank order, SAT row above the strip
-        SAT_TRY(ensure(ws->seedrow, size_t(cols) * sizeof(T), false));
-        sat_seed_from_peers_kernel<T><<<1, 1024, 0, st>>>(static_cast<T*>(ws->seedrow.p), cols, ex.x);
-        CUDA_TRY(cudaGetLastError());
-        ++launches;
-        seed = ws->seedrow.p;
-    }
-    // 3. seeded local 1R1W
+    // 2. seeded local 1R1W: band 0 waits for the flags of ranks < p, adds the
+    //    sum of their slots (rank order) to its first row, acknowledges
     if (strip_rows > 0) {
-        SAT_TRY(compute_core(in, out, 1, strip_rows, cols, ex.dtype, SAT_1R1W, nullptr, seed,
-                             seed ? SEED_SATROW : SEED_NONE, st));
+        ColSeed cs;
+        std::memset(&cs, 0, sizeof(cs));
+        if (ex.rank > 0) {
+            const int par = int(ex.x.epoch & 1);
+            cs.base = ex.x.mine + ex.x.L.slot_off(par, 0);
+            cs.stride = int64_t(ex.x.L.slot_off(par, 1) - ex.x.L.slot_off(par, 0));
+            cs.n = ex.rank;
+            cs.flags = reinterpret_cast<const uint64_t*>(ex.x.mine + ex.x.L.flags_off()) + par * ex.nranks;
+            cs.epoch = ex.x.epoch;
+            cs.acks = ex.acks;
+            cs.done = ex.done;
+        }
+        SAT_TRY(compute_core(in, out, 1, strip_rows, cols, ex.dtype, SAT_1R1W, nullptr, nullptr, &cs, st));
         launches += t_launches;
     }
     t_launches = launches;
@@ -1076,6 +1026,16 @@ int sat_exchange_create(void** handle, int rank, int nranks, int64_t cols, int d
         return fail(SAT_ERR_NOMEM, "exchange counter");
     }
     ex->x.done = ex->done;
+    if (cudaMalloc(&ex->acks, sizeof(uint64_t*) * 16) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(ex->done);
+        delete ex;
+        return fail(SAT_ERR_NOMEM, "exchange ack table");
+    }
+    uint64_t* acks_h[16] = {};
+    for (int q = 0; q < rank; ++q)
+        acks_h[q] = reinterpret_cast<uint64_t*>(ex->x.peers[q] + ex->x.L.acks_off()) + rank;
+    CUDA_TRY(cudaMemcpy(ex->acks, acks_h, sizeof(acks_h), cudaMemcpyHostToDevice));
     CUDA_TRY(cudaMemset(ex->done, 0, sizeof(unsigned int)));
     CUDA_TRY(cudaMemset(mailbox, 0, ex->x.L.bytes()));
     CUDA_TRY(cudaDeviceSynchronize());
@@ -1087,6 +1047,7 @@ int sat_exchange_destroy(void* handle) {
     PeerExchange* ex = static_cast<PeerExchange*>(handle);
     if (!ex) return SAT_OK;
     cudaFree(ex->done);
+    cudaFree(ex->acks);
     delete ex;
     return SAT_OK;
 }
@@ -1131,26 +1092,26 @@ void sat_options_init(sat_options* opt) {
 
 int sat_compute(const void* in, void* out, int64_t rows, int64_t cols, int dtype, int variant,
                 void* stream) {
-    return compute_core(in, out, 1, rows, cols, dtype, variant, nullptr, nullptr, SEED_NONE,
+    return compute_core(in, out, 1, rows, cols, dtype, variant, nullptr, nullptr, nullptr,
                         static_cast<cudaStream_t>(stream));
 }
 
 int sat_compute_ex(const void* in, void* out, int64_t rows, int64_t cols, int dtype, int variant,
                    const sat_options* opt, void* stream) {
-    return compute_core(in, out, 1, rows, cols, dtype, variant, opt, nullptr, SEED_NONE,
+    return compute_core(in, out, 1, rows, cols, dtype, variant, opt, nullptr, nullptr,
                         static_cast<cudaStream_t>(stream));
 }
 
 int sat_compute_batched(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols,
                         int dtype, int variant, const sat_options* opt, void* stream) {
-    return compute_core(in, out, batch, rows, cols, dtype, variant, opt, nullptr, SEED_NONE,
+    return compute_core(in, out, batch, rows, cols, dtype, variant, opt, nullptr, nullptr,
                         static_cast<cudaStream_t>(stream));
 }
 
 int sat_compute_widening(const void* in, int in_dtype, void* out, int dtype, int64_t batch,
                          int64_t rows, int64_t cols, const sat_options* opt, void* stream) {
     if (in_dtype != SAT_UINT8 && !dtype_ok(in_dtype)) return fail(SAT_ERR_INVALID, "bad input dtype");
-    return compute_core(in, out, batch, rows, cols, dtype, SAT_1R1W, opt, nullptr, SEED_NONE,
+    return compute_core(in, out, batch, rows, cols, dtype, SAT_1R1W, opt, nullptr, nullptr,
                         static_cast<cudaStream_t>(stream), in_dtype);
 }
 
@@ -1165,6 +1126,10 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     if (sdt == SAT_INT32 ? out_dtype != SAT_INT32 : (out_dtype != SAT_FLOAT32 && out_dtype != SAT_FLOAT64))
         return fail(SAT_ERR_INVALID, "box filter output: INT32 for integer input, FLOAT32/64 for float input");
     if (rr < 0 || rc < 0) return fail(SAT_ERR_INVALID, "negative radius");
+    // windows are clipped to the image anyway: a radius beyond it changes
+    // nothing, and clamping keeps i + rr / j + rc inside the index type
+    if (rr > rows) rr = int(std::min<int64_t>(rows, INT32_MAX));
+    if (rc > cols) rc = int(std::min<int64_t>(cols, INT32_MAX));
     if (normalize && sdt == SAT_INT32) return fail(SAT_ERR_INVALID, "normalize needs float input");
     if (batch > 65535) return fail(SAT_ERR_UNSUPPORTED, "box filter: batch must be <= 65535");
     SAT_TRY(validate(nullptr, out, batch, rows, cols, out_dtype, false));
@@ -1187,7 +1152,7 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     SAT_TRY(get_ws(dev, st, ws));
     SAT_TRY(ensure(ws->box, size_t(batch) * rows * cols * esize(sdt), false));
     // 1. the SAT (1R1W, widening uint8 -> uint32 and float32 -> float64 on load)
-    SAT_TRY(compute_core(in, ws->box.p, batch, rows, cols, sdt, SAT_1R1W, nullptr, nullptr, SEED_NONE,
+    SAT_TRY(compute_core(in, ws->box.p, batch, rows, cols, sdt, SAT_1R1W, nullptr, nullptr, nullptr,
                          st, in_dtype));
     int launches = t_launches;
     // 2. four SAT reads per output element
@@ -1234,13 +1199,26 @@ int sat_rect_sums(const void* sat, int dtype, int64_t batch, int64_t rows, int64
 
 int sat_compute_seeded(const void* in, void* out, int64_t rows, int64_t cols, int dtype,
                        const void* carry_row, void* stream) {
-    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, carry_row, SEED_COLSUM,
+    return sat_compute_seeded_sum(in, out, rows, cols, dtype, carry_row, carry_row ? 1 : 0, 0, stream);
+}
+
+int sat_compute_seeded_sum(const void* in, void* out, int64_t rows, int64_t cols, int dtype,
+                           const void* vectors, int64_t nvec, int64_t stride, void* stream) {
+    if (nvec < 0 || nvec > INT32_MAX) return fail(SAT_ERR_INVALID, "nvec must be in [0, 2^31)");
+    if (nvec > 0 && !vectors) return fail(SAT_ERR_INVALID, "null seed vectors");
+    if (nvec > 1 && stride < cols) return fail(SAT_ERR_INVALID, "seed stride must be >= cols");
+    ColSeed cs;
+    std::memset(&cs, 0, sizeof(cs));
+    cs.base = vectors;
+    cs.stride = stride * int64_t(esize(dtype));
+    cs.n = int(nvec);
+    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, nullptr, &cs,
                         static_cast<cudaStream_t>(stream));
 }
 
 int sat_compute_seeded_satrow(const void* in, void* out, int64_t rows, int64_t cols, int dtype,
                               const void* sat_row, void* stream) {
-    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, sat_row, SEED_SATROW,
+    return compute_core(in, out, 1, rows, cols, dtype, SAT_1R1W, nullptr, sat_row, nullptr,
                         static_cast<cudaStream_t>(stream));
 }
 
@@ -1297,13 +1275,13 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
         wsp = static_cast<uint8_t*>(ws->shard.p);
     }
     void* send = wsp;
-    void* carry = wsp + row;
     void* recv = wsp + 2 * row;
     int launches = 0;
-    const void* seed = nullptr;
+    ColSeed cs;
+    std::memset(&cs, 0, sizeof(cs));
     if (nranks > 1) {
-        // 1. column totals of the strip (the extra read); the last rank's
-        //    totals are never consumed, so it sends zeros instead
+        // 1. column totals of the strip (the extra read, one launch); the last
+        //    rank's totals are never consumed, so it sends zeros instead
         if (rank < nranks - 1 && strip_rows > 0) {
             SAT_TRY(column_totals_core(in_strip, send, strip_rows, cols, dtype, st));
             launches += t_launches;
@@ -1313,18 +1291,16 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
         // 2. all-gather of the m-vectors (NCCL over NVLink in the Python binding)
         if (allgather(comm_ctx, send, recv, size_t(cols) * eb, stream) != 0)
             return fail(SAT_ERR_COMM, "allgather callback failed");
-        // 3. exclusive scan over ranks
-        if (rank > 0) {
-            t_launches = 0;
-            SAT_TRY(exscan_core(recv, carry, nranks, cols, rank, dtype, st));
-            launches += t_launches;
-            seed = carry;
-        }
+        // 3. the exclusive scan over ranks is the band kernel's seed: band 0
+        //    adds sum_{q < rank} recv[q] (q ascending) to its first row
+        cs.base = recv;
+        cs.stride = int64_t(cols) * int64_t(eb);
+        cs.n = rank;
     }
     // 4. seeded local 1R1W
     if (strip_rows > 0) {
         SAT_TRY(compute_core(in_strip, out_strip, 1, strip_rows, cols, dtype, SAT_1R1W, nullptr,
-                             seed, SEED_COLSUM, st));
+                             nullptr, &cs, st));
         launches += t_launches;
     }
     t_launches = launches;
@@ -1365,7 +1341,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     if (!pinned || variant != SAT_1R1W || rows < 512) {
         CUDA_TRY(cudaMemcpyAsync(ws->din.p, in_host, bytes, cudaMemcpyHostToDevice, st));
         SAT_TRY(compute_core(ws->din.p, ws->dout.p, 1, rows, cols, dtype, variant, nullptr,
-                             nullptr, SEED_NONE, st));
+                             nullptr, nullptr, st));
         launches = t_launches;
         CUDA_TRY(cudaMemcpyAsync(out_host, ws->dout.p, bytes, cudaMemcpyDeviceToHost, st));
         CUDA_TRY(cudaStreamSynchronize(st));
@@ -1382,8 +1358,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     // 32 strips: fill/drain of the copy pipeline is 1/32 of the transfer
     // (32768^2 int32: 89.9 ms vs 95.3 ms with 8 strips; H2D+D2H concurrently
     // take 87.8 ms, tools/pcie_probe.py)
-    int want = 32;
-    if (const char* e = getenv("SAT_HOST_STRIPS")) want = std::max(1, std::min(64, atoi(e)));
+    const int want = 32;
     const int nstrips = int(std::min<int64_t>(want, rows / 256));
     const int64_t srows = (rows + nstrips - 1) / nstrips;
     cudaEvent_t ev_start, ev_in[64], ev_done[64];
@@ -1412,7 +1387,7 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
         if (r1 > r0) {
             SAT_TRY(compute_core(din + r0 * rowb, dout + r0 * rowb, 1, r1 - r0, cols, dtype,
                                  SAT_1R1W, nullptr, k > 0 ? dout + (r0 - 1) * rowb : nullptr,
-                                 SEED_SATROW, st));
+                                 nullptr, st));
             launches += t_launches;
         }
         CUDA_TRY(cudaEventRecord(ev_done[k], st));
@@ -1473,7 +1448,39 @@ int sat_debug_diag_dump(void) {
 }
 
 int sat_debug_trace(void* dev_buf) {
+    if (!kDebug) return fail(SAT_ERR_UNSUPPORTED, "event traces need a debug build (SAT_DEBUG=1)");
     t_trace = static_cast<unsigned long long*>(dev_buf);
+    return SAT_OK;
+}
+
+int sat_debug_set_tag_space(uint64_t space) {
+    if (space == 0) space = 1ull << 30;
+    if (space < 2 || space > (1ull << 30)) return fail(SAT_ERR_INVALID, "tag space must be in [2, 2^30]");
+    g_tag_space.store(space, std::memory_order_relaxed);
+    return SAT_OK;
+}
+
+int sat_release_workspace(void* stream) {
+    int dev;
+    CUDA_TRY(cudaGetDevice(&dev));
+    Workspace* w = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto it = g_ws.find({dev, stream});
+        if (it == g_ws.end()) return SAT_OK;
+        w = it->second;
+        g_ws.erase(it);
+    }
+    // the stream's queued work may still use the buffers
+    CUDA_TRY(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+    for (Buf* b : {&w->desc, &w->lseg, &w->ticket, &w->bt, &w->rs, &w->lx, &w->lsum, &w->topx, &w->lb,
+                   &w->tr, &w->box, &w->part, &w->cnt, &w->shard, &w->din, &w->dout})
+        free_buf(*b);
+    for (void* p : w->retired) cudaFree(p);
+    if (w->cstream_in) cudaStreamDestroy(w->cstream_in);
+    if (w->cstream_out) cudaStreamDestroy(w->cstream_out);
+    if (t_ws == w) t_ws = nullptr;
+    delete w;
     return SAT_OK;
 }
 

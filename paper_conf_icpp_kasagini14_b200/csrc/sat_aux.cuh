@@ -7,8 +7,9 @@
 //    coalescing) and the SAT row above the tile (the paper's C prefix
 //    plus the corner from SAT(S)).  Step 3 is the band kernel with external
 //    carries.
-//  * sharded mode (north star (3)): the strip's column totals and the
-//    exclusive scan of the all-gathered totals over ranks.
+//  * sharded mode (north star (3)): the exclusive scan of all-gathered
+//    totals over ranks (sat_rank_exscan; the sharded entry points fold it into
+//    the band kernel's seed instead, sat_common.h ColSeed).
 #pragma once
 #include "sat_common.h"
 #include "sat_device.cuh"
@@ -234,69 +235,6 @@ __global__ void __launch_bounds__(256) sat_carry_top_kernel(const CarryParams p)
     }
 }
 
-// Sharded mode: partial column sums of row segments.  grid = (nc, splits),
-// 256 threads: warp w sums rows w, w+8, ... of the segment for 128 columns.
-template <typename T>
-__global__ void __launch_bounds__(256)
-sat_colsum_partial_kernel(const T* __restrict__ in, T* __restrict__ part,
-                          int64_t rows, int64_t cols, int64_t seg_rows)
-{
-    const int J = blockIdx.x, sp = blockIdx.y;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int64_t c = int64_t(J) * TW + 4 * lane;
-    const int64_t r0 = int64_t(sp) * seg_rows;
-    int64_t r1 = r0 + seg_rows;
-    if (r1 > rows) r1 = rows;
-    const bool vec = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) && (c + 3 < cols);
-    T cs[4] = {T(0), T(0), T(0), T(0)};
-    int64_t r = r0 + warp;
-    if (vec) {
-        // 8 independent 16-B loads in flight per lane (the sums wait, the loads do not)
-        for (; r + 56 < r1; r += 64) {
-            T e[8][4];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) ldg4<T>(in + (r + 8 * q) * cols + c, e[q]);
-#pragma unroll
-            for (int q = 0; q < 8; ++q)
-#pragma unroll
-                for (int i = 0; i < 4; ++i) cs[i] += e[q][i];
-        }
-    }
-    for (; r < r1; r += 8) {
-        if (vec) {
-            T e[4];
-            ldg4<T>(in + r * cols + c, e);
-#pragma unroll
-            for (int i = 0; i < 4; ++i) cs[i] += e[i];
-        } else {
-#pragma unroll
-            for (int i = 0; i < 4; ++i) if (c + i < cols) cs[i] += in[r * cols + c + i];
-        }
-    }
-    __shared__ T sm[8][TW];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) sm[warp][4 * lane + i] = cs[i];
-    __syncthreads();
-    if (threadIdx.x < TW) {
-        T s = T(0);
-        for (int w = 0; w < 8; ++w) s += sm[w][threadIdx.x];
-        const int64_t cc = int64_t(J) * TW + threadIdx.x;
-        part[int64_t(sp) * gridDim.x * TW + cc] = s;
-    }
-}
-
-// Sum the partials in split order (deterministic); write cols entries.
-template <typename T>
-__global__ void sat_colsum_final_kernel(const T* __restrict__ part, T* __restrict__ totals,
-                                        int64_t cols, int splits, int width)
-{
-    const int64_t c = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (c >= cols) return;
-    T s = T(0);
-    for (int sp = 0; sp < splits; ++sp) s += part[int64_t(sp) * width + c];
-    totals[c] = s;
-}
-
 // carry[c] = sum_{q < rank} gathered[q][c]  (fixed q order)
 template <typename T>
 __global__ void sat_rank_exscan_kernel(const T* __restrict__ gathered, T* __restrict__ carry,
@@ -307,43 +245,6 @@ __global__ void sat_rank_exscan_kernel(const T* __restrict__ gathered, T* __rest
     T s = T(0);
     for (int q = 0; q < rank; ++q) s += gathered[int64_t(q) * cols + c];
     carry[c] = s;
-}
-
-// sat_row[c] = sum_{c' <= c} carry[c'] : the SAT row just above a strip whose
-// column sums above are `carry` (seeded mode).  One CTA of 1024 threads walks
-// the row in tiles of 8192 elements with a running carry.
-template <typename T>
-__global__ void __launch_bounds__(1024)
-sat_row_prefix_kernel(const T* __restrict__ carry, T* __restrict__ sat_row, int64_t cols)
-{
-    __shared__ T wsum[32];
-    __shared__ T s_run;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (threadIdx.x == 0) s_run = T(0);
-    __syncthreads();
-    for (int64_t base = 0; base < cols; base += 8 * 1024) {
-        const int64_t c = base + int64_t(threadIdx.x) * 8;
-        T e[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) e[i] = (c + i < cols) ? carry[c + i] : T(0);
-#pragma unroll
-        for (int i = 1; i < 8; ++i) e[i] += e[i - 1];
-        const T inc = warp_inclusive_scan(e[7], lane);
-        if (lane == 31) wsum[warp] = inc;
-        __syncthreads();
-        if (warp == 0) {
-            const T w = warp_inclusive_scan(wsum[lane], lane);
-            wsum[lane] = w;
-        }
-        __syncthreads();
-        const T off = s_run + (warp > 0 ? wsum[warp - 1] : T(0)) + (inc - e[7]);
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-            if (c + i < cols) sat_row[c + i] = e[i] + off;
-        __syncthreads();
-        if (threadIdx.x == 0) s_run += wsum[31];
-        __syncthreads();
-    }
 }
 
 }  // namespace sat

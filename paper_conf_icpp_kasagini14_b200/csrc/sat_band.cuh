@@ -95,7 +95,7 @@ __device__ __forceinline__ V4<T> lds4_in(const TI* p) {
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int DT, int SUB, int CL = 1, typename TI = T>
+template <typename T, int R, int W, int S, int DT, int SUB, typename TI = T>
 struct BandSmem {
     static constexpr int TH = R * W;
     static constexpr int XS = DT;                    // carry slots: one per parked chunk
@@ -103,12 +103,10 @@ struct BandSmem {
     static constexpr size_t slot_elems = tile_elems * SUB;           // one ring slot
     static constexpr size_t tiles = S * slot_elems * sizeof(TI);     // the ring holds input elements
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
-    // clusters: incoming partial aggregate (chain) and cluster top row per carry slot
-    static constexpr size_t cbuf = CL > 1 ? size_t(2) * XS * TW * sizeof(T) : 0;
-    // + unit queue (CL == 1): ufull[2], uempty[2]
-    static constexpr size_t nbars = 2 * S + 2 * XS + (CL > 1 ? 4 * XS : 4);
+    // + unit queue: ufull[2], uempty[2]
+    static constexpr size_t nbars = 2 * S + 2 * XS + 4;
     static constexpr size_t bars = nbars * sizeof(uint64_t) + 32;   // + s_unit[2], s_tmem
-    static constexpr size_t total = tiles + xbuf + cbuf + bars;
+    static constexpr size_t total = tiles + xbuf + bars;
 };
 
 __device__ __forceinline__ uint32_t band_tag(unsigned long long base, int gb) {
@@ -288,7 +286,39 @@ struct TmemCols {
     static_assert(need <= 512, "TMEM holds at most 512 columns");
 };
 
-template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int CL, int MODE, bool TMA, int MINB,
+// ---------------------------------------------------------------- column-sum seed
+// (sharded mode; sat_common.h ColSeed).  Waits for the producers' flags when
+// the vectors live in a peer-exchange mailbox (sat_xchg.cuh).
+__device__ __forceinline__ void colseed_wait(const ColSeed& cs) {
+    if (cs.flags == nullptr) return;
+    for (int q = 0; q < cs.n; ++q) {
+        uint64_t v;
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(cs.flags + q) : "memory");
+        if (v >= cs.epoch) continue;
+        SpinGuard guard(0x18000000u | uint32_t(q), uint32_t(cs.epoch));
+        do {
+            __nanosleep(128);
+            guard.tick();
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(cs.flags + q) : "memory");
+        } while (v < cs.epoch);
+    }
+}
+// sum_{q < n} vec_q[c .. c+3] in q order (columns >= cols read as 0); volatile
+// loads: the vectors may have been written over NVLink by another GPU
+template <typename T>
+__device__ __forceinline__ V4<T> colseed4(const ColSeed& cs, int64_t c, int64_t cols) {
+    T e[4] = {T(0), T(0), T(0), T(0)};
+    for (int q = 0; q < cs.n; ++q) {
+        const volatile T* v = reinterpret_cast<const volatile T*>(
+            reinterpret_cast<const uint8_t*>(cs.base) + int64_t(q) * cs.stride);
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+            if (c + i < cols) e[i] += v[c + i];
+    }
+    return V4<T>{e[0], e[1], e[2], e[3]};
+}
+
+template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
           int LBW_ = 0, typename TI = T>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
@@ -298,9 +328,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
     constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(TI);
-    using SM = BandSmem<T, R, W, S, DT, SUB, CL, TI>;
-    static_assert(std::is_same<T, TI>::value || (MODE == MODE_SAT && CL == 1), "widening input: 1R1W only");
-    static_assert(CL == 1 || (MODE == MODE_SAT && NS == 1 && sizeof(T) == 4), "clusters: 1R1W band kernel only");
+    using SM = BandSmem<T, R, W, S, DT, SUB, TI>;
+    static_assert(std::is_same<T, TI>::value || MODE == MODE_SAT, "widening input: 1R1W only");
     constexpr int NWE = Words<T>::N;             // 32-bit words per element
     using TC = TmemCols<R, W, DT, NWE>;
     constexpr int XS = SM::XS;
@@ -314,33 +343,20 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     extern __shared__ __align__(1024) uint8_t smem[];
     TI* tiles = reinterpret_cast<TI*>(smem);
     T* xbuf = reinterpret_cast<T*>(smem + SM::tiles);
-    T* cagg = reinterpret_cast<T*>(smem + SM::tiles + SM::xbuf);         // [XS][TW] own aggregate (CL > 1)
-    T* ctop = cagg + size_t(XS) * TW;                                     // [XS][TW] top from rank 0 (CL > 1)
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf + SM::cbuf);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::tiles + SM::xbuf);
     uint64_t* full = bars;              // [S]  TMA load landed (tx count)
     uint64_t* empty = bars + S;         // [S]  every compute warp read the slot
     uint64_t* colr = bars + 2 * S;      // [XS] every compute warp published its bottom row
     uint64_t* topr = bars + 2 * S + XS; // [XS] the control warp wrote the add vectors
-    // clusters (CL > 1), per carry slot: aggb = the aggregates of every lower
-    // rank are readable; aggfree = every higher rank has read ours; ctopb =
-    // the cluster's top row from rank 0 arrived; ctopfree (rank 0) = every
-    // other rank read it
-    uint64_t* aggb = bars + 2 * S + 2 * XS;
-    uint64_t* aggfree = aggb + XS;
-    uint64_t* ctopb = aggb + 2 * XS;
-    uint64_t* ctopfree = aggb + 3 * XS;
-    // unit queue (CL == 1): the producer warp takes the
-    // next ticket as soon as it has issued the last load of the current unit
-    // and posts it in s_unit[u & 1] (ufull); the other warps read it and
-    // release the entry (uempty), so the next unit's loads overlap the
-    // current unit's last look-backs and stores
+    // unit queue: the producer warp takes the next ticket
+    // as soon as it has issued the last load of the current unit and posts it
+    // in s_unit[u & 1] (ufull); the other warps read it and release the entry
+    // (uempty), so the next unit's loads overlap the current unit's last
+    // look-backs and stores
     uint64_t* ufull = bars + 2 * S + 2 * XS;
     uint64_t* uempty = ufull + 2;
     long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
     uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 2);
-    const uint32_t crank = CL > 1 ? cluster_ctarank() : 0u;
-    // ticket/tag base: the host's counter, or (CUDA-graph capture, DESIGN.md
-    // Sec. 4) the value sat_epoch_kernel wrote just before this launch
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -350,22 +366,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], W * 32);
         }
-        if constexpr (CL == 1) {
-            for (int u = 0; u < 2; ++u) {
-                mbar_init(&ufull[u], 1);
-                mbar_init(&uempty[u], W + NCW);      // lane 0 of every non-producer warp
-            }
+        for (int u = 0; u < 2; ++u) {
+            mbar_init(&ufull[u], 1);
+            mbar_init(&uempty[u], W + NCW);      // lane 0 of every non-producer warp
         }
         for (int x = 0; x < XS; ++x) {
             mbar_init(&colr[x], W * 32);
             mbar_init(&topr[x], 32 * NS);
-            if constexpr (CL > 1) {
-                const uint32_t rk = cluster_ctarank();
-                mbar_init(&aggb[x], rk > 0 ? 32 * rk : 1);
-                mbar_init(&aggfree[x], rk + 1 < CL ? 32 * (CL - 1 - rk) : 1);
-                mbar_init(&ctopb[x], 32);
-                mbar_init(&ctopfree[x], 32 * (CL - 1));
-            }
         }
         fence_mbar_init();
     }
@@ -377,13 +384,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     if (TMA && warp == PW && lane == 0) prefetch_tmap(&tm_in);
     tmem_fence_before();
     __syncthreads();
-    if constexpr (CL > 1) cluster_sync_all();    // peers' barriers initialised before any remote arrive
     tmem_fence_after();
     const uint32_t tmem_base = HOLD ? *s_tmem : 0u;
-    // Programmatic dependent launch (SAT_PDL): everything above is CTA-local
-    // and may overlap the previous kernel's tail; global memory from here on
-    // (a no-op when launched without the attribute)
+    // Programmatic dependent launch: everything above is CTA-local and may
+    // overlap the previous kernel's tail; global memory from here on (a
+    // no-op when launched without the attribute)
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    // ticket/tag base: the host's counter, or (CUDA-graph capture, DESIGN.md
+    // Sec. 4) the value sat_epoch_kernel wrote just before this launch
     const unsigned long long kbase = p.base_dev ? __ldcg(p.base_dev) : p.base;
 
     const int64_t img_elems = p.rows * p.cols;
@@ -393,18 +401,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
 
     for (uint32_t useq = 0;; ++useq) {
-        if constexpr (CL > 1) {
-            // one ticket per cluster: CL consecutive bands, rank r takes band CL*u + r
-            if (crank == 0 && threadIdx.x == 0) {
-                const unsigned long long u = atomicAdd(p.ticket, 1ull) - kbase;
-                for (uint32_t r = 0; r < CL; ++r) st_cluster_u64(mapa(smem_u32(s_unit), r), u);
-            }
-            cluster_sync_all();
-        }
         long long unit;
-        if constexpr (CL > 1) {
-            unit = *s_unit;
-        } else {
+        {
             const uint32_t qs = useq & 1u, qph = (useq >> 1) & 1u;
             if (warp == PW) {
                 if (lane == 0) {
@@ -423,25 +421,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         }
         diag_mark(p.diag, uint32_t(unit), 0, 1);
         if (unit < 0) __trap();                       // ticket accounting out of sync: never silently
-        if (p.diag != nullptr && threadIdx.x == 0) {
-            // per-block history of units (debug)
-            volatile unsigned int* h = p.diag + 4096u * 32u * 4u + 4096u * 32u * 2u + blockIdx.x * 16u;
-            const unsigned int n = h[15];
-            if (n < 15) { h[n] = uint32_t(unit); h[15] = n + 1; }
-        }
         if (unit >= p.total_units) break;
 
         int gb, j0, j1;
-        int gcb = 0, cb = 0;                           // cluster-band (CL > 1)
         int seg = 0;                                   // band segment (p.nseg > 1)
-        if constexpr (CL > 1) {
-            const int upi = (p.nb + CL - 1) / CL;       // cluster-bands per image
-            gcb = int(unit);
-            const int im = gcb / upi;
-            cb = gcb - im * upi;
-            gb = im * p.nb + cb * CL + int(crank);      // may exceed the image: a virtual band
-            j0 = 0; j1 = p.nc;
-        } else if (p.tile_units) {
+        if (p.tile_units) {
             // ranges of tile_units chunks of a band's region (external
             // carries: the row carry at the range start comes from Lx)
             const int per = (p.nc + p.tile_units - 1) / p.tile_units;
@@ -460,15 +444,19 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             gb = int(unit);
             region_range(p.region, p.tA, p.nb, p.nc, gb % p.nb, j0, j1);
         }
-        const int img = CL > 1 ? gcb / ((p.nb + CL - 1) / CL) : gb / p.nb;
-        const int band = gb - img * p.nb;              // >= p.nb: virtual (rows all beyond the matrix)
+        const int img = gb / p.nb;
+        const int band = gb - img * p.nb;
         const int nch = j1 - j0;
         const int row0 = band * TH;
-        const bool traced = p.trace != nullptr && band < p.nb;
+        const bool traced = kDebug && p.trace != nullptr;
+        (void)traced;
 
         if (warp < W) {
             // ================= compute warps =================
             const int rbase = warp * R;                  // first row of this warp in the band
+            // column-sum seed: added to the strip's first row (warp 0, row 0)
+            const bool seeded = p.cseed.n > 0 && gb == 0 && warp == 0;
+            if (seeded) colseed_wait(p.cseed);
             T L[R];
 #pragma unroll
             for (int r = 0; r < R; ++r) L[r] = T(0);
@@ -533,12 +521,16 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             auto local = [&](int k) {
                 const uint32_t it = g + k;
                 V4<T> v[R];
+                V4<T> sd;
+                if (seeded) sd = colseed4<T>(p.cseed, int64_t(j0 + k) * TW + 4 * lane, p.cols);
                 if constexpr (TMA) {
                     const uint32_t q = gq + uint32_t(k / SUB);     // ring slot of chunk k
                     const int s = q % S;
                     if (k % SUB == 0) mbar_wait(&full[s], (q / S) & 1);
-                    if (traced && warp == 0 && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
+                    if constexpr (kDebug) {
+                        if (traced && warp == 0 && lane == 0)
+                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
+                    }
                     const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
                                   + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
@@ -571,6 +563,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         v[r] = V4<T>{e[0], e[1], e[2], e[3]};
                     }
                 }
+                if (seeded) add4(v[0], sd);
                 if constexpr (MODE != MODE_COL) row_scan<T, R>(v, L, lane);
                 if constexpr (!HOLD) {
                     store_rows(v, k);                    // the row pass is final
@@ -594,8 +587,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             auto finish = [&](int k) {
                 const uint32_t it = g + k;
                 mbar_wait(&topr[it % XS], (it / XS) & 1);
-                if (traced && warp == 0 && lane == 0)
-                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
+                if constexpr (kDebug) {
+                    if (traced && warp == 0 && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
+                }
                 const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
                 uint32_t u[TC::per_chunk];
                 tmem_wait_st();
@@ -610,8 +605,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     add4(v[r], add);
                 }
                 store_rows(v, k);
-                if (traced && warp == 0 && lane == 0)
-                    p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
+                if constexpr (kDebug) {
+                    if (traced && warp == 0 && lane == 0)
+                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
+                }
             };
 
             if constexpr (!HOLD) {
@@ -624,6 +621,23 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     diag_mark(p.diag, uint32_t(unit), uint32_t(k), 3);
                 }
                 for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
+            }
+            if (seeded && p.cseed.acks != nullptr) {
+                // every seed vector this unit needed has been read (the values
+                // are in the stored results); the last band-0 unit (segments)
+                // acknowledges to the producers (sat_xchg.cuh)
+                __syncwarp();
+                if (lane == 0) {
+                    __threadfence();
+                    const unsigned int n = atomicAdd(p.cseed.done, 1u);
+                    if (n + 1 == unsigned(p.nseg > 1 ? p.nseg : 1)) {
+                        *p.cseed.done = 0u;
+#pragma unroll 1
+                        for (int q = 0; q < p.cseed.n; ++q)
+                            asm volatile("st.release.sys.global.u64 [%0], %1;"
+                                         :: "l"(p.cseed.acks[q]), "l"(uint64_t(p.cseed.epoch)) : "memory");
+                    }
+                }
             }
             if (p.nseg > 1 && seg + 1 < p.nseg && lane < R * NWE) {
                 // hand the row carry to segment seg+1 of this band (word `lane`)
@@ -670,8 +684,10 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     const int c0 = J * TW + cl;
                     T* xb = xbuf + size_t(it % XS) * W * TW + cl;
                     mbar_wait(&colr[it % XS], (it / XS) & 1);
-                    if (traced && cw == grp * NS && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
+                    if constexpr (kDebug) {
+                        if (traced && cw == grp * NS && lane == 0)
+                            p.trace[(int64_t(gb) * p.nc + J) * 8 + 1] = globaltimer();
+                    }
                     T agg[CPL];
                     lds_cols<T, CPL>(xb, agg);
 #pragma unroll
@@ -691,164 +707,93 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                     for (int i = 0; i < CPL; ++i) top[i] = T(0);
                     unsigned long long hops = 0, polls = 0;
-                    // decoupled look-back from descriptor row gidx (index idx
-                    // within its image) over rows idx-1, idx-2, ...: adds the
-                    // SAT row above row idx to acc
-                    auto walk = [&](int gidx, int idx, T (&acc)[CPL]) {
-                        T (&top)[CPL] = acc;
-                    // decoupled look-back over bands band-1, band-2, ...,
-                    // LBW descriptor rows per round trip
-                    uint32_t pend = (1u << CPL) - 1u;
-                    int kb = idx - 1;
-                    SpinGuard guard(0x80000000u | uint32_t(J), uint32_t(gidx));
-                    while (pend) {
-                        uint64_t wv[LBW][NW];
-#pragma unroll
-                        for (int q = 0; q < LBW; ++q) {
-                            const int b2 = kb - q;
-                            if (b2 >= 0) {
-                                load_words<NW>(p.desc + ((int64_t(gidx) - (idx - b2)) * desc_w + c0) * NWE, wv[q]);
-                            } else {
-#pragma unroll
-                                for (int i = 0; i < NW; ++i) wv[q][i] = 0;
-                            }
-                        }
-                        bool stalled = false;
-#pragma unroll
-                        for (int q = 0; q < LBW; ++q) {
-                            if (!pend || stalled) break;
-                            const int b2 = kb - q;
-                            if (CL == 1 && p.region == REG_C && b2 + J < p.tA) {
-                                // tile (b2, J) belongs to (A): its final SAT row is in `out`
-                                const int64_t row = int64_t(b2 + 1) * TH - 1;
-#pragma unroll
-                                for (int i = 0; i < CPL; ++i)
-                                    if ((pend >> i) & 1u)
-                                        top[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
-                                pend = 0;
-                                break;
-                            }
-                            const uint32_t tk = band_tag(kbase, gidx - (idx - b2));
-                            bool ready = true;
-#pragma unroll
-                            for (int i = 0; i < NW; ++i) {
-                                const uint32_t t = uint32_t(wv[q][i] >> 32);
-                                ready = ready && ((t & ~3u) == tk) && (t & 3u);
-                            }
-                            // the words of one float64 value must come from the
-                            // same publication (aggregate and inclusive share a slot)
-#pragma unroll
-                            for (int i = 0; i < CPL; ++i)
-#pragma unroll
-                                for (int k = 1; k < NWE; ++k)
-                                    ready = ready && (uint32_t(wv[q][i * NWE + k] >> 32) == uint32_t(wv[q][i * NWE] >> 32));
-                            if (!ready) { stalled = true; kb = b2; break; }
-#pragma unroll
-                            for (int i = 0; i < CPL; ++i) {
-                                if ((pend >> i) & 1u) {
-                                    uint32_t w[NWE];
-#pragma unroll
-                                    for (int k = 0; k < NWE; ++k) w[k] = uint32_t(wv[q][i * NWE + k]);
-                                    top[i] += from_words<T>(w);
-                                    if ((uint32_t(wv[q][i * NWE] >> 32) & 3u) == 2u) pend &= ~(1u << i);
-                                }
-                            }
-                            ++hops;
-                        }
-                        if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
-                        else kb -= LBW;
-                    }
-                    };
-                    auto seed_row = [&](T (&acc)[CPL]) {
+                    if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                    if (!lookback) {
+                        lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
+                    } else if (band == 0) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
-                            // the SAT row just above the matrix (sat_api.cu turns a
-                            // column-sum seed into this row first)
+                            // the SAT row just above the matrix (seeded mode)
                             const T* sd = reinterpret_cast<const T*>(p.seed);
 #pragma unroll
-                            for (int i = 0; i < CPL; ++i) acc[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
-                        }
-                    };
-                    if constexpr (CL > 1) {
-                        // Cluster of CL bands (DSMEM): every
-                        // rank leaves its chunk aggregate in its own smem and
-                        // signals the higher ranks; rank r sums the aggregates
-                        // of ranks < r straight from their smem (one DSMEM round
-                        // trip); rank 0 looks back over the cluster-band
-                        // descriptors and broadcasts the SAT row T above the
-                        // cluster; rank r's top = T + S_{r-1}; the last rank
-                        // publishes the cluster's aggregate and inclusive.
-                        const uint32_t x = it % XS, ph = (it / XS) & 1u;
-                        const int upi = (p.nb + CL - 1) / CL;
-                        const bool pubc = cb + 1 < upi;
-                        uint64_t* myc = p.desc + int64_t(gcb) * desc_w + c0;
-                        const uint32_t ctag = band_tag(kbase, gcb);
-                        T Sp[CPL] = {};
-                        if (crank + 1 < CL) {
-                            if (it >= uint32_t(XS)) mbar_wait_cluster(&aggfree[x], ph ^ 1u);
-                            sts_cols<T, CPL>(cagg + size_t(x) * TW + cl, agg);
-                            for (uint32_t r2 = crank + 1; r2 < CL; ++r2)
-                                mbar_arrive_remote(mapa(smem_u32(&aggb[x]), r2));
-                        }
-                        if (crank > 0) {
-                            mbar_wait_cluster(&aggb[x], ph);
-                            for (uint32_t r2 = 0; r2 < crank; ++r2) {
-                                const uint4 u = ld_cluster_v4(mapa(smem_u32(cagg + size_t(x) * TW + cl), r2));
-                                Sp[0] += from_bits<T>(u.x); Sp[1] += from_bits<T>(u.y);
-                                Sp[2] += from_bits<T>(u.z); Sp[3] += from_bits<T>(u.w);
-                            }
-                            for (uint32_t r2 = 0; r2 < crank; ++r2)
-                                mbar_arrive_remote(mapa(smem_u32(&aggfree[x]), r2));
-                        }
-                        if (crank == 0) {
-                            if (cb == 0) seed_row(top);
-                            else walk(gcb, cb, top);
-                            if (it >= uint32_t(XS)) mbar_wait_cluster(&ctopfree[x], ph ^ 1u);
-                            for (uint32_t r2 = 1; r2 < CL; ++r2) {
-                                st_cluster_v4(mapa(smem_u32(ctop + size_t(x) * TW + cl), r2),
-                                              to_bits(top[0]), to_bits(top[1]), to_bits(top[2]), to_bits(top[3]));
-                                mbar_arrive_remote(mapa(smem_u32(&ctopb[x]), r2));
-                            }
-                        } else {
-                            T Sa[CPL];
-#pragma unroll
-                            for (int i = 0; i < CPL; ++i) Sa[i] = Sp[i] + agg[i];
-                            // (cluster-band 0 publishes only its inclusive: a walk
-                            // must never pass row 0 on an aggregate)
-                            if (crank + 1 == CL && pubc && cb > 0) publish_words<T, CPL>(myc, ctag | 1u, Sa);
-                            mbar_wait_cluster(&ctopb[x], ph);
-                            lds_cols<T, CPL>(ctop + size_t(x) * TW + cl, top);
-                            mbar_arrive_remote(mapa(smem_u32(&ctopfree[x]), 0));
-                            if (crank + 1 == CL && pubc) {
-                                T inc[CPL];
-#pragma unroll
-                                for (int i = 0; i < CPL; ++i) inc[i] = top[i] + Sa[i];
-                                publish_words<T, CPL>(myc, ctag | 2u, inc);
-                            }
-#pragma unroll
-                            for (int i = 0; i < CPL; ++i) top[i] += Sp[i];
+                            for (int i = 0; i < CPL; ++i) top[i] = (c0 + i < p.cols) ? sd[c0 + i] : T(0);
                         }
                     } else {
-                        if (p.dbg & 1) {
-                            // timing probe only: no vertical carry
-                        } else if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
-                        if (p.dbg & 1) {
-                        } else if (!lookback) {
-                            lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
-                        } else if (band == 0) {
-                            seed_row(top);
-                        } else if (!(p.dbg & 2)) {
-                            walk(gb, band, top);
-                        }
-                        if (publish && !(p.dbg & 1)) {
-                            T inc[CPL];
+                        // decoupled look-back over bands band-1, band-2, ...,
+                        // LBW descriptor rows per round trip: adds the SAT row
+                        // above this band to top
+                        uint32_t pend = (1u << CPL) - 1u;
+                        int kb = band - 1;
+                        SpinGuard guard(0x80000000u | uint32_t(J), uint32_t(gb));
+                        while (pend) {
+                            uint64_t wv[LBW][NW];
 #pragma unroll
-                            for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
-                            publish_words<T, CPL>(my, tagbase | 2u, inc);
+                            for (int q = 0; q < LBW; ++q) {
+                                const int b2 = kb - q;
+                                if (b2 >= 0) {
+                                    load_words<NW>(p.desc + ((int64_t(gb) - (band - b2)) * desc_w + c0) * NWE, wv[q]);
+                                } else {
+#pragma unroll
+                                    for (int i = 0; i < NW; ++i) wv[q][i] = 0;
+                                }
+                            }
+                            bool stalled = false;
+#pragma unroll
+                            for (int q = 0; q < LBW; ++q) {
+                                if (!pend || stalled) break;
+                                const int b2 = kb - q;
+                                if (p.region == REG_C && b2 + J < p.tA) {
+                                    // tile (b2, J) belongs to (A): its final SAT row is in `out`
+                                    const int64_t row = int64_t(b2 + 1) * TH - 1;
+#pragma unroll
+                                    for (int i = 0; i < CPL; ++i)
+                                        if ((pend >> i) & 1u)
+                                            top[i] += (c0 + i < p.cols) ? gout[row * p.cols + c0 + i] : T(0);
+                                    pend = 0;
+                                    break;
+                                }
+                                const uint32_t tk = band_tag(kbase, gb - (band - b2));
+                                bool ready = true;
+#pragma unroll
+                                for (int i = 0; i < NW; ++i) {
+                                    const uint32_t t = uint32_t(wv[q][i] >> 32);
+                                    ready = ready && ((t & ~3u) == tk) && (t & 3u);
+                                }
+                                // the words of one float64 value must come from the
+                                // same publication (aggregate and inclusive share a slot)
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i)
+#pragma unroll
+                                    for (int k = 1; k < NWE; ++k)
+                                        ready = ready && (uint32_t(wv[q][i * NWE + k] >> 32) == uint32_t(wv[q][i * NWE] >> 32));
+                                if (!ready) { stalled = true; kb = b2; break; }
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i) {
+                                    if ((pend >> i) & 1u) {
+                                        uint32_t w[NWE];
+#pragma unroll
+                                        for (int k = 0; k < NWE; ++k) w[k] = uint32_t(wv[q][i * NWE + k]);
+                                        top[i] += from_words<T>(w);
+                                        if ((uint32_t(wv[q][i * NWE] >> 32) & 3u) == 2u) pend &= ~(1u << i);
+                                    }
+                                }
+                                ++hops;
+                            }
+                            if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
+                            else kb -= LBW;
                         }
                     }
-                    if (traced && cw == grp * NS && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
-                            (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
+                    if (publish) {
+                        T inc[CPL];
+#pragma unroll
+                        for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
+                        publish_words<T, CPL>(my, tagbase | 2u, inc);
+                    }
+                    if constexpr (kDebug) {
+                        if (traced && cw == grp * NS && lane == 0)
+                            p.trace[(int64_t(gb) * p.nc + J) * 8 + 2] =
+                                (globaltimer() & 0xFFFFFFFFFFFFull) | (min(hops, 255ull) << 48) | (min(polls, 255ull) << 56);
+                    }
+                    (void)hops; (void)polls;
                     // add vectors for finish(): top + bottom rows of the warps above
 #pragma unroll
                     for (int w2 = 0; w2 < W; ++w2) {
@@ -867,18 +812,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if constexpr (TMA) {
                 if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
-                    int kpf = S * SUB;                       // next chunk to prefetch into L2
                     for (int k0 = 0; k0 < nch; k0 += SUB) {
                         const uint32_t q = gq + uint32_t(k0 / SUB);
                         const int s = q % S;
                         const int nsub = nch - k0 < SUB ? nch - k0 : SUB;
-                        // L2 prefetch p.pf chunks ahead of the load (beyond the ring)
-                        if (p.pf > S * SUB)
-                            for (; kpf < nch && kpf < k0 + p.pf; ++kpf)
-                                tma_prefetch_3d(&tm_in, (j0 + kpf) * TW, row0, img);
                         if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
-                        if (traced)
-                            p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();
+                        if constexpr (kDebug) {
+                            if (traced) p.trace[(int64_t(gb) * p.nc + j0 + k0) * 8 + 4] = globaltimer();
+                        }
                         mbar_arrive_expect_tx(&full[s], TILE_BYTES * nsub);
                         for (int j = 0; j < nsub; ++j)   // adjacent boxes: SUB*512 B per row
                             tma_load_3d(tiles + size_t(s) * SM::slot_elems + size_t(j) * SM::tile_elems,
@@ -890,8 +831,6 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         diag_mark(p.diag, uint32_t(unit), uint32_t(nch), 5);
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
-        if constexpr (CL > 1) cluster_sync_all();      // before rank 0 overwrites s_unit
-        else if (p.unit_sync) __syncthreads();         // A/B: no overlap of consecutive units
     }
     diag_mark(p.diag, 0xFFFFFFFFu, 0, 6);
     if (HOLD) {

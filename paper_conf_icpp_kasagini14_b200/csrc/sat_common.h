@@ -35,6 +35,24 @@ SAT_HD void region_range(int region, int tA, int nb, int nc, int I, int& j0, int
     j0 = lo; j1 = hi;
 }
 
+// Column-sum seed of a strip (row-strip sharding, north star (3)): the
+// carry row c[j] = sum_{q < n} vec_q[j] (q ascending) is the column sum of
+// everything above the strip.  Band 0 of image 0 adds it to its first input
+// row before the row scan (SAT of [c; a] restricted to a's rows == the rows
+// of the taller matrix's SAT), so neither a carry-prefix kernel nor an
+// exclusive-scan kernel runs.  Sources: one vector (sat_compute_seeded), the
+// all-gathered totals of ranks < p (NCCL path), or the slots of a peer
+// mailbox after its flags (fused exchange, sat_xchg.cuh).
+struct ColSeed {
+    const void* base;               // vector q at base + q * stride (bytes); nullptr = none
+    int64_t stride;
+    int n;                          // vectors to sum (0 = no seed)
+    const uint64_t* flags;          // nullable: wait flags[q] >= epoch (sys acquire) before reading vector q
+    unsigned long long epoch;
+    uint64_t* const* acks;          // nullable: [n] after the last read, st.release.sys(acks[q], epoch)
+    unsigned int* done;             // band-0 units finished reading (self-resetting counter) when acks != nullptr
+};
+
 struct BandParams {
     const void* in;            // [batch][rows][cols] (generic path, not used by TMA path)
     void* out;                 // [batch][rows][cols]
@@ -45,7 +63,6 @@ struct BandParams {
     int total_bands;           // batch * nb
     long long total_units;     // bands (band units) or bands*nc (tile units)
     int tile_units;            // K > 0: one ticket = K consecutive tiles of a band (external carries); 0 = whole bands
-    int cluster;               // CTAs per cluster (1, or 8: one ticket = 8 bands)
     int big;                   // 1: one CTA per SM with a 2x ring of 1-KB row segments (TH 64)
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
@@ -53,16 +70,14 @@ struct BandParams {
     const unsigned long long* base_dev;   // nullable: read the base from device memory (graph capture)
     const void* seed;          // [cols] SAT row above band 0 of image 0, nullable
     int seed_kind;             // SEED_NONE or SEED_SATROW
+    ColSeed cseed;             // column-sum seed added to row 0 of image 0 (n = 0: none)
     int top_src;               // TopSrc
     int region;                // Region
     int tA;                    // (1+r)R1W threshold
     const void* Lx;            // [nc+1][total_bands*TH] row carry at chunk start, nullable
     const void* TopX;          // [total_bands][nc*TW] external SAT row above, nullable
     void* Lb;                  // [total_bands*TH] band-final row carry out, nullable
-    int jitter;                // debug: random publish delay (ns scale), 0 = off
-    int dbg;                   // debug: bit 0 = skip look-back and publication (top = 0; WRONG results, timing only)
-    unsigned long long* trace; // debug: [total_bands*nc][4] event times (ns), nullable
-    unsigned int* diag;        // debug: host-mapped progress marks (sat_debug_diag_enable), nullable
+    int jitter;                // stress tests: random publish delay (ns scale), 0 = off
     // Band segments (plain 1R1W, many waves): a ticket is (segment s, band b),
     // segment-major, so the last wave holds short units.  Segment s covers
     // chunks [s*segc, (s+1)*segc); the row carry L of band b crosses from
@@ -70,8 +85,8 @@ struct BandParams {
     int nseg;                  // 1 = whole bands
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
-    int pf;                    // L2 prefetch distance in chunks (TMA path; 0 = off)
-    int unit_sync;             // A/B: 1 = the next unit starts only after every warp finished this one
+    unsigned long long* trace; // debug builds (SAT_DEBUG): [total_bands*nc][8] event times (ns), nullable
+    unsigned int* diag;        // debug builds: host-mapped progress marks, nullable
 };
 
 }  // namespace sat

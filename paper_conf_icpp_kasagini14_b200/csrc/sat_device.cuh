@@ -53,13 +53,20 @@ constexpr unsigned long long kSpinLimitNs = 4000000000ull;   // 4 s
 // a protocol deadlock can be read back after the launch fails.
 __device__ unsigned int* g_sat_diag = nullptr;
 
-// progress marks (debug): per (block, warp) the last {unit, step, mark}
-// (`diag` comes from the kernel parameters, not from g_sat_diag: a global
-// load per mark would stall the compute warps for a full memory round trip)
+#ifndef SAT_DEBUG
+#define SAT_DEBUG 0      // 1: per-chunk event traces and per-warp progress marks (tools/ only)
+#endif
+constexpr bool kDebug = SAT_DEBUG != 0;
+
+// progress marks (debug builds only): per (block, warp) the last {unit, step,
+// mark} in host-mapped memory (`diag` comes from the kernel parameters, not
+// from g_sat_diag: a global load per mark would stall the compute warps)
 __device__ __forceinline__ void diag_mark(unsigned int* diag, uint32_t unit, uint32_t step, uint32_t mark) {
-    if (diag != nullptr && (threadIdx.x & 31) == 0) {
-        volatile unsigned int* d = diag + 4096u * 32u * 4u + (blockIdx.x * 32u + (threadIdx.x >> 5)) * 4u;
-        d[0] = unit; d[1] = step; d[2] = 0xC0DE0000u | mark; d[3] = blockIdx.x;
+    if constexpr (kDebug) {
+        if (diag != nullptr && (threadIdx.x & 31) == 0) {
+            volatile unsigned int* d = diag + 4096u * 32u * 4u + (blockIdx.x * 32u + (threadIdx.x >> 5)) * 4u;
+            d[0] = unit; d[1] = step; d[2] = 0xC0DE0000u | mark; d[3] = blockIdx.x;
+        }
     }
 }
 

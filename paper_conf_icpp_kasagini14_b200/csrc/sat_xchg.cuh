@@ -8,10 +8,9 @@
 //     of every higher rank's mailbox (P2P stores over NVLink through
 //     IPC-mapped pointers), and the last block to finish raises a flag
 //     (st.release.sys) in each of those mailboxes;
-//   * the SAT prologue (the kernel that turns the carry into the SAT row above
-//     the strip) waits for the flags of ranks < p (ld.acquire.sys), sums their
-//     slots in rank order and writes its acknowledgement back into each
-//     producer's mailbox.
+//   * the SAT kernel's band 0 waits for the flags of ranks < p
+//     (ld.acquire.sys), sums their slots in rank order into its first input
+//     row and writes its acknowledgement back into each producer's mailbox.
 // Mailboxes are double-buffered by call parity; before reusing a parity a
 // producer waits for every consumer's acknowledgement of the call two back,
 // so no data is overwritten before it is read and no barrier is needed.
@@ -21,6 +20,10 @@
 
 namespace sat {
 
+// The consumer side runs inside the band kernel (sat_band.cuh, ColSeed):
+// band 0 waits for the flags of ranks < p, adds sum_{q<p} slot[par][q] (q
+// ascending) to its first input row, and the last band-0 unit acknowledges.
+//
 // Mailbox layout (per rank, `cols` values of T per slot):
 //   uint64 flag[2][P]     flag[par][q] = epoch of the totals q wrote in slot par
 //   uint64 ack[P]         ack[c]       = last epoch consumer c finished reading
@@ -61,89 +64,128 @@ __device__ __forceinline__ void wait_at_least(const uint64_t* p, uint64_t want, 
     while (ld_acquire_sys_u64(p) < want) { __nanosleep(128); guard.tick(); }
 }
 
-// Column totals from the partials (as sat_colsum_final_kernel), pushed into
-// slot (epoch & 1, rank) of every higher rank's mailbox.
+// Column totals of a strip in ONE launch (the sharded mode's extra read).
+// grid = (nc, splits), 256 threads: block (J, sp) sums rows [sp*seg, (sp+1)*seg)
+// of the 128 columns of chunk J (8 independent 16-B loads in flight per lane)
+// into part[sp][J*128 ..]; the last block to arrive for chunk J (counter
+// cnt[J]) adds the splits in split order (deterministic), writes the totals
+// and -- in the fused exchange -- stores them straight into slot (epoch & 1,
+// rank) of every higher rank's mailbox; the last chunk column to finish
+// (counter cnt[nc]) raises those ranks' flags with st.release.sys.  Before
+// the first store into a parity, the consumers' acknowledgements of the call
+// two back are awaited.  Counters reset themselves.
+struct TotalsParams {
+    const void* in;
+    int64_t rows, cols;
+    int64_t seg_rows;
+    int splits;
+    void* part;                 // [splits][nc*TW]
+    unsigned int* cnt;          // [nc + 1], zero between calls
+    void* totals;               // nullable: cols entries on this device
+    int push;                   // 1: fused exchange (x)
+    XchgParams x;
+};
+
 template <typename T>
-__global__ void __launch_bounds__(256)
-sat_colsum_push_kernel(const T* __restrict__ part, int64_t cols, int splits, int width, XchgParams x) {
+__global__ void __launch_bounds__(256) sat_colsum_kernel(const TotalsParams tp) {
+    const int J = blockIdx.x, sp = blockIdx.y;
+    const int nc = gridDim.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const T* in = static_cast<const T*>(tp.in);
+    const int64_t cols = tp.cols;
+    const int64_t c = int64_t(J) * TW + 4 * lane;
+    const int64_t r0 = int64_t(sp) * tp.seg_rows;
+    const int64_t r1 = min(tp.rows, r0 + tp.seg_rows);
+    const bool vec = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(in) & 15) == 0) && (c + 3 < cols);
+    T cs[4] = {T(0), T(0), T(0), T(0)};
+    int64_t r = r0 + warp;
+    if (vec) {
+        for (; r + 56 < r1; r += 64) {
+            T e[8][4];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) ldg4<T>(in + (r + 8 * q) * cols + c, e[q]);
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+#pragma unroll
+                for (int i = 0; i < 4; ++i) cs[i] += e[q][i];
+        }
+    }
+    for (; r < r1; r += 8) {
+        if (vec) {
+            T e[4];
+            ldg4<T>(in + r * cols + c, e);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) cs[i] += e[i];
+        } else {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) if (c + i < cols) cs[i] += in[r * cols + c + i];
+        }
+    }
+    __shared__ T sm[8][TW];
+    __shared__ int s_last;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) sm[warp][4 * lane + i] = cs[i];
+    __syncthreads();
+    T* part = static_cast<T*>(tp.part);
+    if (threadIdx.x < TW) {
+        T s = T(0);
+        for (int w = 0; w < 8; ++w) s += sm[w][threadIdx.x];
+        part[int64_t(sp) * nc * TW + int64_t(J) * TW + threadIdx.x] = s;
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = atomicAdd(&tp.cnt[J], 1u) == unsigned(tp.splits - 1);
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    const XchgParams& x = tp.x;
     const int par = int(x.epoch & 1);
     const int P = x.L.P;
-    if (threadIdx.x == 0 && x.epoch > 2) {
+    if (tp.push && threadIdx.x == 0 && x.epoch > 2) {
         // the consumers of this parity's previous use (epoch - 2) are done
-        for (int c = x.rank + 1; c < P; ++c)
-            wait_at_least(reinterpret_cast<const uint64_t*>(x.mine + x.L.acks_off()) + c, x.epoch - 2,
-                          0x10000000u | uint32_t(c));
+        for (int q = x.rank + 1; q < P; ++q)
+            wait_at_least(reinterpret_cast<const uint64_t*>(x.mine + x.L.acks_off()) + q, x.epoch - 2,
+                          0x10000000u | uint32_t(q));
     }
     __syncthreads();
-    for (int64_t c = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; c < cols;
-         c += int64_t(gridDim.x) * blockDim.x) {
-        T s = T(0);
-        for (int sp = 0; sp < splits; ++sp) s += part[int64_t(sp) * width + c];
-        for (int q = x.rank + 1; q < P; ++q)
-            reinterpret_cast<T*>(x.peers[q] + x.L.slot_off(par, x.rank))[c] = s;
+    if (threadIdx.x < TW) {
+        const int64_t cc = int64_t(J) * TW + threadIdx.x;
+        if (cc < cols) {
+            T s = T(0);
+            for (int k = 0; k < tp.splits; ++k) s += __ldcg(part + int64_t(k) * nc * TW + cc);
+            if (tp.totals) static_cast<T*>(tp.totals)[cc] = s;
+            if (tp.push)
+                for (int q = x.rank + 1; q < P; ++q)
+                    reinterpret_cast<T*>(x.peers[q] + x.L.slot_off(par, x.rank))[cc] = s;
+        }
     }
-    // last block: publish the flag in every consumer's mailbox
+    if (threadIdx.x == 0) tp.cnt[J] = 0u;
+    if (!tp.push) return;
     __threadfence_system();
     __syncthreads();
     if (threadIdx.x == 0) {
-        const unsigned int n = atomicAdd(x.done, 1u);
-        if (n == gridDim.x - 1) {
+        const unsigned int n = atomicAdd(&tp.cnt[nc], 1u);
+        if (n == unsigned(nc - 1)) {
+            tp.cnt[nc] = 0u;
             __threadfence_system();
             for (int q = x.rank + 1; q < P; ++q)
                 st_release_sys_u64(reinterpret_cast<uint64_t*>(x.peers[q] + x.L.flags_off()) + par * P + x.rank,
                                    x.epoch);
-            *x.done = 0;
         }
     }
 }
 
-// Rank p's carry: wait for ranks < p, carry[c] = sum_{q<p} slot[par][q][c]
-// (rank order), acknowledge, then the SAT row above the strip =
-// row prefix of the carry (as sat_row_prefix_kernel).  One CTA of 1024.
-template <typename T>
-__global__ void __launch_bounds__(1024)
-sat_seed_from_peers_kernel(T* __restrict__ sat_row, int64_t cols, XchgParams x) {
-    __shared__ T wsum[32];
-    __shared__ T s_run;
+// A rank with an empty strip still consumes its producers' totals: wait for
+// the flags, acknowledge (keeps the double-buffered protocol in step).
+__global__ void sat_xchg_drain_kernel(XchgParams x) {
     const int par = int(x.epoch & 1);
     const int P = x.L.P;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (threadIdx.x < x.rank)
-        wait_at_least(reinterpret_cast<const uint64_t*>(x.mine + x.L.flags_off()) + par * P + threadIdx.x,
-                      x.epoch, 0x18000000u | threadIdx.x);
-    if (threadIdx.x == 0) s_run = T(0);
-    __syncthreads();
-    for (int64_t base = 0; base < cols; base += 8 * 1024) {
-        const int64_t c = base + int64_t(threadIdx.x) * 8;
-        T e[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            T s = T(0);
-            if (c + i < cols)
-                for (int q = 0; q < x.rank; ++q)
-                    s += reinterpret_cast<const volatile T*>(x.mine + x.L.slot_off(par, q))[c + i];
-            e[i] = s;
-        }
-#pragma unroll
-        for (int i = 1; i < 8; ++i) e[i] += e[i - 1];
-        const T inc = warp_inclusive_scan(e[7], lane);
-        if (lane == 31) wsum[warp] = inc;
-        __syncthreads();
-        if (warp == 0) wsum[lane] = warp_inclusive_scan(wsum[lane], lane);
-        __syncthreads();
-        T exc = __shfl_up_sync(0xffffffffu, inc, 1);
-        if (lane == 0) exc = T(0);
-        const T off = s_run + (warp > 0 ? wsum[warp - 1] : T(0)) + exc;
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-            if (c + i < cols) sat_row[c + i] = e[i] + off;
-        __syncthreads();
-        if (threadIdx.x == 0) s_run += wsum[31];
-        __syncthreads();
+    const int q = threadIdx.x;
+    if (q < x.rank) {
+        wait_at_least(reinterpret_cast<const uint64_t*>(x.mine + x.L.flags_off()) + par * P + q, x.epoch,
+                      0x18000000u | uint32_t(q));
+        st_release_sys_u64(reinterpret_cast<uint64_t*>(x.peers[q] + x.L.acks_off()) + x.rank, x.epoch);
     }
-    // every slot read: acknowledge to each producer
-    if (threadIdx.x < x.rank)
-        st_release_sys_u64(reinterpret_cast<uint64_t*>(x.peers[threadIdx.x] + x.L.acks_off()) + x.rank, x.epoch);
 }
 
 }  // namespace sat

@@ -27,7 +27,7 @@ def test_every_declared_symbol_is_exported():
 
 
 def test_abi_version_and_strings():
-    assert libsat.abi_version() == 1
+    assert libsat.abi_version() == 2
     assert libsat.lib.sat_strerror(0) == b"ok"
     assert libsat.lib.sat_strerror(-1) == b"invalid argument"
 

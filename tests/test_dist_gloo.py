@@ -17,16 +17,22 @@ from sat_inputs import make_np
 
 
 class OracleOps:
-    def column_totals(self, strip):
-        return torch.from_numpy(oracle.column_totals(strip.numpy()).astype(np.int32))
+    """Oracle stand-ins with CudaOps' interface: column totals into the
+    exchange buffer; the seeded SAT takes the gathered totals and the rank
+    (the exclusive scan over ranks happens inside it, as in the kernel)."""
 
-    def exscan(self, gathered, rank):
-        return torch.from_numpy(np.ascontiguousarray(oracle.rank_exscan(gathered.numpy(), rank)))
+    def column_totals(self, strip, out=None):
+        t = torch.from_numpy(oracle.column_totals(strip.numpy()).astype(np.int32))
+        if out is not None:
+            out.copy_(t)
+            return out
+        return t
 
-    def seeded_sat(self, strip, carry, out=None):
+    def seeded_sat(self, strip, gathered, rank, out=None):
         loc = oracle.sat(strip.numpy()).view(np.uint32)
-        if carry is not None:
-            top = np.cumsum(carry.numpy().view(np.uint32).astype(np.uint64)).astype(np.uint32)
+        if gathered is not None and rank > 0:
+            carry = np.ascontiguousarray(oracle.rank_exscan(gathered.numpy(), rank)).view(np.uint32)
+            top = np.cumsum(carry.astype(np.uint64)).astype(np.uint32)
             with np.errstate(over="ignore"):
                 loc = loc + top[None, :]
         return torch.from_numpy(loc.view(np.int32).copy())

@@ -52,7 +52,7 @@ def test_widening_float32_to_float64(libsat, shape):
     assert np.array_equal(y.cpu().numpy(), oracle.sat(a))        # exact: dyadic sums in double
 
 
-def test_widening_batched_tiles_segments(libsat, monkeypatch):
+def test_widening_batched_tiles_segments(libsat):
     a = u8img(1080, 1920, seed=4, batch=5)
     for th in (64, 128):
         y = libsat.sat_widening(dev(a), torch.int32, tile_rows=th).cpu().numpy()
@@ -62,9 +62,8 @@ def test_widening_batched_tiles_segments(libsat, monkeypatch):
     for th in (16, 32, 64):
         assert np.array_equal(libsat.sat_widening(dev(f), torch.float64, tile_rows=th).cpu().numpy(),
                               oracle.sat(f))
-    monkeypatch.setenv("SAT_SEG", "3")
     g = u8img(64 * 40 + 7, 2048, seed=5)
-    assert np.array_equal(libsat.sat_widening(dev(g), torch.int32, tile_rows=64).cpu().numpy(),
+    assert np.array_equal(libsat.sat_widening(dev(g), torch.int32, tile_rows=64, segments=3).cpu().numpy(),
                           oracle.sat(g.astype(np.int32)))
 
 

@@ -69,7 +69,7 @@ def test_shapes(libsat, variant, dtype, shape):
     check(libsat.sat(dev(a), variant=variant), ref, dtype)
 
 
-@pytest.mark.parametrize("tile_rows", [16, 32, 48, 64, 112, 128])
+@pytest.mark.parametrize("tile_rows", [16, 32, 64, 128])
 @pytest.mark.parametrize("generic", [False, True])
 @pytest.mark.parametrize("variant", VARIANTS)
 def test_tile_configs(libsat, tile_rows, generic, variant):
@@ -78,7 +78,8 @@ def test_tile_configs(libsat, tile_rows, generic, variant):
         ref = oracle.sat(a)
         check(libsat.sat(dev(a), variant=variant, tile_rows=tile_rows, force_generic=generic),
               ref, dtype)
-        assert libsat.last_tile_rows() == tile_rows
+        if variant in ("1r1w", "2r1w", "1+rr1w") and not generic:
+            assert libsat.last_tile_rows() == tile_rows
 
 
 @pytest.mark.parametrize("r", [0.0, 0.1, 0.25, 0.5, 1.0])
@@ -134,7 +135,7 @@ def test_repeated_calls_fresh_tags(libsat):
 
 
 def test_lookback_jitter_stress(libsat):
-    for th in (16, 32, 48, 64, 112, 128):
+    for th in (16, 32, 64, 128):
         a = gen(3000, 2500, "int32", seed=th)
         check(libsat.sat(dev(a), tile_rows=th, jitter=20000), oracle.sat(a), "int32")
         af = gen(3000, 2500, "float32", seed=th)
@@ -199,6 +200,38 @@ def test_column_totals_and_exscan(libsat):
                 assert np.allclose(e, r, rtol=1e-6, atol=0)
 
 
+def test_seeded_gathered_is_the_rank_exscan(libsat):
+    """sat_compute_seeded_sum: band 0 adds sum_{q<rank} gathered[q] to its
+    first row (the sharded mode's exclusive scan inside the SAT kernel), for
+    every rank, in one launch."""
+    P, n, m = 5, 640, 1100
+    for dtype in ("int32", "float32"):
+        full = gen(n, m, dtype, seed=17)
+        ref = oracle.sat(full)
+        r0 = 257
+        if dtype == "int32":
+            above = oracle.column_totals(full[:r0])
+        else:
+            above = full[:r0].astype(np.float64).sum(axis=0)
+        # P gathered vectors whose prefix of length `rank` sums to `above`
+        rng = np.random.default_rng(3)
+        for rank in range(1, P + 1):
+            g = np.zeros((P, m), dtype=np.float64 if dtype == "float32" else np.uint32)
+            if dtype == "int32":
+                parts = rng.integers(0, 2**32, size=(rank - 1, m), dtype=np.uint64).astype(np.uint32)
+                with np.errstate(over="ignore"):
+                    last = above.view(np.uint32) - parts.sum(axis=0, dtype=np.uint32)
+                g[:rank - 1] = parts
+                g[rank - 1] = last
+                gd = dev(g.view(np.int32))
+            else:
+                g[:rank] = above / rank
+                gd = dev(g.astype(np.float32))
+            got = libsat.sat_seeded(dev(full[r0:]), gathered=gd, rank=rank)
+            assert libsat.last_launch_count() == 1
+            check(got, ref[r0:], dtype)
+
+
 @pytest.mark.parametrize("P", [1, 2, 3, 8])
 def test_sharded_abi_single_process(libsat, P):
     """sat_compute_sharded with a fake all-gather: P ranks simulated one after
@@ -220,6 +253,8 @@ def test_sharded_abi_single_process(libsat, P):
                 recv.copy_(torch.stack(totals))
             o, st = libsat.sat_sharded_abi(strips[p], p, P, ag)
             outs.append(o.cpu().numpy())
+            # one totals launch (ranks < P-1) + one SAT launch
+            assert libsat.last_launch_count() == (2 if (P > 1 and p < P - 1) else 1)
             rows = bounds[p][1] - bounds[p][0]
             assert st["extra_bytes_read"] == (rows * m * 4 if (P > 1 and p < P - 1) else 0)
         check(np.concatenate(outs), ref, dtype)
@@ -310,44 +345,13 @@ def test_cfg4_65536_properties(libsat):
         assert rec == np.uint32(int(x[i, j]) & 0xFFFFFFFF)
 
 
-# ------------------------------------------------------------------ clusters (DSMEM carry chain)
-@pytest.mark.parametrize("shape,th", [((1024, 1024), 64), ((512, 700), 64), ((2048, 4096), 64),
-                                      ((9 * 64, 1280), 64), ((170 * 64, 256), 64),
-                                      ((8 * 48, 2000), 48), ((160 * 48 + 5, 384), 48)])
-def test_cluster_path(libsat, shape, th, monkeypatch):
-    """The opt-in 8-CTA cluster path (SAT_CLUSTER=8), including padded virtual
-    bands -- several clusters run concurrently and look back over each other's
-    cluster-band descriptors."""
-    monkeypatch.setenv("SAT_CLUSTER", "8")
-    for dtype in ("int32", "float32"):
-        a = gen(*shape, dtype, seed=shape[0] + th)
-        check(libsat.sat(dev(a), tile_rows=th), oracle.sat(a), dtype)
-
-
-def test_cluster_repeat_and_jitter(libsat, monkeypatch):
-    monkeypatch.setenv("SAT_CLUSTER", "8")
-    a = gen(4096, 2048, "int32", seed=41)
-    ref = oracle.sat(a)
-    x = dev(a)
-    for _ in range(5):
-        check(libsat.sat(x, tile_rows=64), ref, "int32")
-    check(libsat.sat(x, tile_rows=64, jitter=20000), ref, "int32")
-
-
-def test_cluster_batched_and_seeded(libsat, monkeypatch):
-    monkeypatch.setenv("SAT_CLUSTER", "8")
-    a = make_np(512, 640, "int32", "u32", seed=42, batch=3)       # 8 bands per image
-    y = libsat.sat_batched(dev(a), tile_rows=64).cpu().numpy()
-    for b in range(3):
-        check(y[b], oracle.sat(a[b]), "int32")
-    full = gen(64 * 40, 900, "int32", seed=43)
-    ref = oracle.sat(full)
-    r0 = 64 * 8
-    carry = oracle.column_totals(full[:r0])
-    check(libsat.sat_seeded(dev(full[r0:]), carry_row=dev(carry)), ref[r0:], "int32")
-
-
 def test_debug_trace_records_events(libsat):
+    """Event traces exist in debug builds only (SAT_DEBUG=1); the release
+    library refuses them loudly."""
+    if libsat.lib.sat_debug_trace(None) != 0:
+        with pytest.raises(Exception, match="debug build"):
+            libsat.debug_trace(torch.zeros(8, dtype=torch.int64, device="cuda"))
+        return
     a = gen(640, 1024, "int32", seed=44)
     x = dev(a)
     nb, nc = 10, 8
@@ -361,59 +365,58 @@ def test_debug_trace_records_events(libsat):
     assert libsat.last_grid() >= 1
 
 
-@pytest.mark.parametrize("shape", [(1000, 1300), (64 * 40 + 7, 2048), (4096, 777 * 4)])
-def test_big_ring_config(libsat, shape, monkeypatch):
-    """TH=64 with one CTA per SM and 1-KB row segments per TMA load (the
-    configuration chosen automatically for >= 4 waves of bands)."""
-    monkeypatch.setenv("SAT_BIG", "1")
+@pytest.mark.parametrize("shape", [(64 * 600 + 7, 256), (64 * 640, 777 * 4)])
+def test_big_ring_config(libsat, shape):
+    """TH=64 with one CTA per SM and 1-KB row segments per TMA load (chosen
+    automatically for >= 4 waves of TH-64 bands)."""
     for dtype in ("int32", "float32"):
         a = gen(*shape, dtype, seed=shape[0])
         check(libsat.sat(dev(a), tile_rows=64), oracle.sat(a), dtype)
 
 
 @pytest.mark.parametrize("nseg", [2, 3, 7])
-@pytest.mark.parametrize("tile_rows", [64, 112, 128])
-def test_band_segments(libsat, nseg, tile_rows, monkeypatch):
+@pytest.mark.parametrize("tile_rows", [64, 128])
+def test_band_segments(libsat, nseg, tile_rows):
     """Band segments: a ticket is (segment, band) and the
     row carry crosses segments through tagged words; every split is exact."""
-    monkeypatch.setenv("SAT_SEG", str(nseg))
+    kw = dict(tile_rows=tile_rows, segments=nseg)
     for shape in [(1000, 1300), (64 * 40 + 7, 2048), (300, 777 * 4)]:
         for dtype in ("int32", "float32"):
             a = gen(*shape, dtype, seed=nseg * 7 + shape[0])
-            check(libsat.sat(dev(a), tile_rows=tile_rows), oracle.sat(a), dtype)
+            check(libsat.sat(dev(a), **kw), oracle.sat(a), dtype)
     a = gen(3 * 400, 1920, "int32", seed=5).reshape(3, 400, 1920)
-    got = libsat.sat_batched(dev(a), tile_rows=tile_rows).cpu().numpy()
+    got = libsat.sat_batched(dev(a), **kw).cpu().numpy()
     for i in range(3):
         assert np.array_equal(got[i], oracle.sat(a[i]))
     # repeated calls reuse the carry buffer with fresh tags; jitter shuffles timing
     x = dev(gen(2048, 4096, "int32", seed=3))
     ref = oracle.sat(x.cpu().numpy())
     for _ in range(3):
-        check(libsat.sat(x, tile_rows=tile_rows), ref, "int32")
-    check(libsat.sat(x, tile_rows=tile_rows, jitter=20000), ref, "int32")
+        check(libsat.sat(x, **kw), ref, "int32")
+    check(libsat.sat(x, jitter=20000, **kw), ref, "int32")
 
 
 @pytest.mark.parametrize("nseg", [3, 4, 5])
-@pytest.mark.parametrize("tile_rows", [64, 112, 128])
-def test_unit_queue_many_units(libsat, nseg, tile_rows, monkeypatch):
+@pytest.mark.parametrize("tile_rows", [64, 128])
+def test_unit_queue_many_units(libsat, nseg, tile_rows):
     """Many short units per CTA: the next unit's loads
     start before the current unit's control groups are done, so a group's
     chunks must stay G apart across unit boundaries.  Segments of a number of
     chunks that is not a multiple of the control-group count (3 at TH 112/128)
     failed before the assignment became CTA-global."""
-    monkeypatch.setenv("SAT_SEG", str(nseg))
+    kw = dict(tile_rows=tile_rows, segments=nseg)
     a = gen(20000, 3000, "int32", seed=nseg + tile_rows)
     ref = oracle.sat(a)
     x = dev(a)
-    check(libsat.sat(x, tile_rows=tile_rows), ref, "int32")
-    check(libsat.sat(x, tile_rows=tile_rows, jitter=20000), ref, "int32")
+    check(libsat.sat(x, **kw), ref, "int32")
+    check(libsat.sat(x, jitter=20000, **kw), ref, "int32")
     af = gen(9000, 2500, "float32", seed=nseg)
-    check(libsat.sat(dev(af), tile_rows=tile_rows), oracle.sat(af), "float32")
+    check(libsat.sat(dev(af), **kw), oracle.sat(af), "float32")
     # 65536 x 4096 all ones, in place (1 GiB): 2048 units of 8 chunks at nseg 4
     if nseg == 4:
         n, m = 65536, 4096
         y = torch.ones(n, m, dtype=torch.int32, device="cuda")
-        libsat.sat(y, out=y, tile_rows=tile_rows)
+        libsat.sat(y, out=y, **kw)
         jj = torch.arange(1, m + 1, device="cuda", dtype=torch.int64)
         for r in (0, 127, 17664, 18944, 40000, n - 1):
             assert torch.equal(y[r].to(torch.int64) % 2**32, ((r + 1) * jj) % 2**32), r
@@ -575,13 +578,20 @@ def test_cuda_graph_batched_two_shapes(libsat):
 
 
 @pytest.mark.parametrize("space,replays", [("300000", 6), ("540000", 60)])
-def test_cuda_graph_tag_reset(libsat, monkeypatch, space, replays):
-    """A tiny tag space (SAT_TAG_SPACE) makes sat_epoch_kernel clear the
+def test_cuda_graph_tag_reset(libsat, space, replays):
+    """A tiny tag space (sat_debug_set_tag_space) makes sat_epoch_kernel clear the
     descriptors on every replay (each launch's value range crosses a multiple
     of half the space), and forces the host-side reset on eager calls of a
     never-captured stream.  At 540000 (half the space just above the
     per-launch bound) only some replays clear: the mixed regime."""
-    monkeypatch.setenv("SAT_TAG_SPACE", space)
+    libsat.set_tag_space(int(space))
+    try:
+        _graph_tag_reset(libsat, replays)
+    finally:
+        libsat.set_tag_space(0)
+
+
+def _graph_tag_reset(libsat, replays):
     x = dev(gen(2048, 2048, "int32", seed=3))
     s = torch.cuda.Stream()
     with torch.cuda.stream(s):
