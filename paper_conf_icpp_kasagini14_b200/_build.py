@@ -9,6 +9,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libsat.so")
+LIB_DEBUG = os.path.join(PKG, "libsat_debug.so")   # tools only: event traces (SAT_DEBUG=1)
 NVCC_FLAGS = [
     "-O3", "-std=c++17", "-lineinfo",
     "-gencode", "arch=compute_100a,code=sm_100a",
@@ -21,25 +22,29 @@ def _sources():
             + glob.glob(os.path.join(CSRC, "*.h")) + [os.path.join(ROOT, "include", "sat.h")])
 
 
-def stale() -> bool:
-    if not os.path.exists(LIB):
+def stale(lib: str = LIB) -> bool:
+    if not os.path.exists(lib):
         return True
-    t = os.path.getmtime(LIB)
+    t = os.path.getmtime(lib)
     return any(os.path.getmtime(s) > t for s in _sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
-        return LIB
+def build(force: bool = False, verbose: bool = False, debug: bool = False) -> str:
+    """Build libsat.so (release), or libsat_debug.so (debug=True: per-chunk
+    event traces and progress marks for tools/; load it with LIBSAT_SO)."""
+    lib = LIB_DEBUG if debug else LIB
+    if not force and not stale(lib):
+        return lib
     nvcc = os.environ.get("NVCC", "nvcc")
-    tmp = LIB + ".tmp%d" % os.getpid()
-    cmd = [nvcc] + NVCC_FLAGS + ["-o", tmp, os.path.join(CSRC, "sat_api.cu")]
+    tmp = lib + ".tmp%d" % os.getpid()
+    cmd = [nvcc] + NVCC_FLAGS + (["-DSAT_DEBUG=1"] if debug else []) + ["-o", tmp, os.path.join(CSRC, "sat_api.cu")]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force=True, verbose=True))
+    import sys
+    print(build(force=True, verbose=True, debug="--debug" in sys.argv))

@@ -122,6 +122,8 @@ struct Workspace {
     Buf box;                  // box filter: the SAT it reads
     Buf part;                 // column totals partials
     Buf cnt;                  // column totals: per-chunk-column and global arrival counters (self-resetting)
+    Buf order;                // segment-unit ticket order (int2 per unit), for order_key
+    unsigned long long order_key = 0;
     Buf shard;                // sharded default workspace
     Buf din, dout;            // host e2e device copies
     std::vector<void*> retired;   // buffers a captured graph may still reference (freed by sat_release_workspace)
@@ -296,9 +298,9 @@ struct KernelSetup {
 };
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW = 0, typename TI = T>
+          int LBW = 0, typename TI = T, bool BULK = false>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI>;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI, BULK>;
     const size_t smem = BandSmem<T, R, W, S, DT, SUB, TI>::total;
     const int threads = (W + NCW + 1) * 32;
     // per instantiation and device: attributes set once, resources queried
@@ -397,6 +399,16 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
         }
         return fail(SAT_ERR_INVALID, "float64: no band configuration for this tile_rows");
     } else {
+        if (p.xcfg == 1 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 0, T, true>(p, ti, di, st, grid);
+        if (p.xcfg == 2 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 0, T, false>(p, ti, di, st, grid);
+        if (p.xcfg == 4 && th == 32) return launch_band_t<T, 8, 4, 3, 8, 4, 4, 1, MODE, TMA, 1, 0, T, true>(p, ti, di, st, grid);
+        if (p.xcfg == 5 && th == 32) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 1, MODE, TMA, 2, 0, T, true>(p, ti, di, st, grid);
+        if (p.xcfg == 7 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 8>(p, ti, di, st, grid);
+        if (p.xcfg == 8 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 8>(p, ti, di, st, grid);
+        if (p.xcfg == 9 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 4>(p, ti, di, st, grid);
+        if (p.xcfg == 10 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 2>(p, ti, di, st, grid);
+        if (p.xcfg == 11 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 12>(p, ti, di, st, grid);
+        if (p.xcfg == 6 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 2, T, true>(p, ti, di, st, grid);
         if (p.big && th == 64) return launch_band_t<T, SAT_CFG(kCfg64B), MODE, TMA, kCfg64B.MINB>(p, ti, di, st, grid);
         switch (th) {
             case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, di, st, grid);
@@ -487,6 +499,7 @@ struct Job {
     bool tma;
     int jitter;
     int segments;     // sat_options.segments: 0 = automatic band segments
+    int xcfg;         // development A/B (sat_options.reserved[0])
     const DevInfo* di;
     Workspace* ws;
     cudaStream_t st;
@@ -548,7 +561,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     // Many bands (>= 4 waves of one CTA per SM): one CTA per SM with twice the
     // ring and 1-KB row segments per TMA load.
     p.big = (mode == MODE_SAT && j.tma && j.th == 64 && j.dtype != SAT_FLOAT64 && j.in_dtype == j.dtype &&
-             p.total_bands >= 4 * j.di->sms) ? 1 : 0;
+             p.total_bands >= 4 * j.di->sms && !j.xcfg) ? 1 : 0;
     // Band segments: short units for the last wave when
     // bands are many waves deep
     p.nseg = 1;
@@ -561,7 +574,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         // 20480^2: 0.614 ms with 8-10 vs 0.887 ms; 12288^2 float64: 0.608 vs
         // 0.785 ms); at most one wave: whole bands (a segment would wait for
         // the band's previous segment)
-        const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0);
+        const int slots = j.di->sms * (j.xcfg == 5 ? 2 : (j.xcfg && j.th != 128) ? 1 : ctas_per_sm(j.dtype, j.th, p.big != 0));
         int want = p.total_bands > slots ? std::min(16, p.nc / 16) : 1;
         if (j.segments > 0) want = j.segments;
         if (want > 1 && p.nc > 1) {
@@ -570,7 +583,30 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
             p.total_units = (long long)p.total_bands * p.nseg;
         }
     }
+    // skewed ticket order of the segment units
+    p.order = nullptr;
+    if (p.nseg > 1 && (j.xcfg == 40 || j.xcfg == 41)) {
+        const int K = std::max(1, (j.xcfg == 41 ? 4 : 2) * j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0) / p.nseg);
+        const unsigned long long key = (unsigned long long)p.total_bands | ((unsigned long long)p.nseg << 32) |
+                                       ((unsigned long long)K << 44);
+        Workspace& w = *j.ws;
+        if (w.order_key != key || !w.order.p) {
+            std::vector<int2> ord;
+            ord.reserve(size_t(p.total_bands) * p.nseg);
+            const long long kmax = (long long)p.total_bands - 1 + (long long)K * (p.nseg - 1);
+            for (long long d = 0; d <= kmax; ++d)
+                for (int sg = 0; sg < p.nseg; ++sg) {
+                    const long long b = d - (long long)K * sg;
+                    if (b >= 0 && b < p.total_bands) ord.push_back(make_int2(sg, int(b)));
+                }
+            SAT_TRY(ensure(w.order, ord.size() * sizeof(int2), false));
+            CUDA_TRY(cudaMemcpy(w.order.p, ord.data(), ord.size() * sizeof(int2), cudaMemcpyHostToDevice));
+            w.order_key = key;
+        }
+        p.order = static_cast<const int2*>(w.order.p);
+    }
     p.jitter = j.jitter;
+    p.xcfg = (mode == MODE_SAT && j.tma && j.dtype != SAT_FLOAT64 && j.in_dtype == j.dtype) ? j.xcfg : 0;
     if (kDebug) {
         p.diag = g_diag_dev;
         if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
@@ -822,6 +858,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     j.tma = !o.force_generic && tma_ok(in, out, cols, in_dtype);
     j.jitter = o.jitter;
     j.segments = o.segments;
+    j.xcfg = o.reserved[0];
     j.di = &di;
     j.ws = ws;
     j.st = st;
@@ -1474,7 +1511,7 @@ int sat_release_workspace(void* stream) {
     // the stream's queued work may still use the buffers
     CUDA_TRY(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     for (Buf* b : {&w->desc, &w->lseg, &w->ticket, &w->bt, &w->rs, &w->lx, &w->lsum, &w->topx, &w->lb,
-                   &w->tr, &w->box, &w->part, &w->cnt, &w->shard, &w->din, &w->dout})
+                   &w->tr, &w->box, &w->part, &w->cnt, &w->order, &w->shard, &w->din, &w->dout})
         free_buf(*b);
     for (void* p : w->retired) cudaFree(p);
     if (w->cstream_in) cudaStreamDestroy(w->cstream_in);

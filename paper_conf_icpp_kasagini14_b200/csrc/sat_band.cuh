@@ -105,7 +105,9 @@ struct BandSmem {
     static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
     // + unit queue: ufull[2], uempty[2]
     static constexpr size_t nbars = 2 * S + 2 * XS + 4;
-    static constexpr size_t bars = nbars * sizeof(uint64_t) + 32;   // + s_unit[2], s_tmem
+    // + s_unit[2], s_tmem, and per compute warp the (band, chunk) of each
+    // parked chunk (finish() may run after the chunk's unit ended)
+    static constexpr size_t bars = nbars * sizeof(uint64_t) + 32 + size_t(W) * DT * 8;
     static constexpr size_t total = tiles + xbuf + bars;
 };
 
@@ -319,7 +321,7 @@ __device__ __forceinline__ V4<T> colseed4(const ColSeed& cs, int64_t c, int64_t 
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW_ = 0, typename TI = T>
+          int LBW_ = 0, typename TI = T, bool BULK = false>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -357,6 +359,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     uint64_t* uempty = ufull + 2;
     long long* s_unit = reinterpret_cast<long long*>(bars + SM::nbars);
     uint32_t* s_tmem = reinterpret_cast<uint32_t*>(s_unit + 2);
+    int2* meta = reinterpret_cast<int2*>(s_unit + 4);   // [W][DT]
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -399,6 +402,56 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     const int64_t lx_stride = int64_t(p.total_bands) * TH;
     uint32_t g = 0;                              // CTA-local chunk counter (carry / TMEM slots)
     uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
+    // compute warps: this warp's rows in a band, TMEM lanes (32*(warp%4) ..)
+    // and column range, parked-chunk metadata
+    const int rbase = warp * R;
+    const uint32_t tm_warp = tmem_base + ((uint32_t(32 * (warp & 3))) << 16)
+                             + uint32_t((warp >> 2) * TC::per_warp);
+    int2* wmeta = meta + (warp < W ? warp : 0) * DT;
+    // finish(it) of the CTA-global chunk stream: + (SAT row above the band +
+    // bottom rows of the warps above), from the add vector the control warp
+    // left in xbuf, then the 1W.  Runs DT-1 chunks after local(it) -- across
+    // unit boundaries, so the look-back of a unit's last chunks overlaps the
+    // next unit's first chunks instead of stalling the compute warps.
+    auto finish_it = [&](uint32_t it) {
+        const int2 md = wmeta[it % DT];
+        const int fgb = md.x, fJ = md.y;
+        const int fimg = fgb / p.nb;
+        const int frow0 = (fgb - fimg * p.nb) * TH;
+        T* fout = reinterpret_cast<T*>(p.out) + int64_t(fimg) * (p.rows * p.cols);
+        mbar_wait(&topr[it % XS], (it / XS) & 1);
+        if constexpr (kDebug) {
+            if (p.trace != nullptr && warp == 0 && lane == 0)
+                p.trace[(int64_t(fgb) * p.nc + fJ) * 8 + 6] = globaltimer();
+        }
+        const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
+        uint32_t u[TC::per_chunk];
+        tmem_wait_st();
+        tmem_ld<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
+        tmem_wait_ld();
+        const int64_t c = int64_t(fJ) * TW + 4 * lane;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const uint32_t* q = u + 4 * r * NWE;
+            V4<T> v{from_words<T>(q), from_words<T>(q + NWE), from_words<T>(q + 2 * NWE), from_words<T>(q + 3 * NWE)};
+            add4(v, add);
+            const int64_t row = frow0 + rbase + r;
+            if (row < p.rows) {
+                if constexpr (TMA) {
+                    if (c < p.cols) st_global_v4(fout + row * p.cols + c, v);
+                } else {
+                    const T e[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+                        if (c + i < p.cols) fout[row * p.cols + c + i] = e[i];
+                }
+            }
+        }
+        if constexpr (kDebug) {
+            if (p.trace != nullptr && warp == 0 && lane == 0)
+                p.trace[(int64_t(fgb) * p.nc + fJ) * 8 + 3] = globaltimer();
+        }
+    };
 
     for (uint32_t useq = 0;; ++useq) {
         long long unit;
@@ -436,8 +489,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             j0 = min(r1, r0 + sr * p.tile_units);
             j1 = min(r1, j0 + p.tile_units);
         } else if (p.nseg > 1) {
-            seg = int(unit / p.total_bands);
-            gb = int(unit - (long long)seg * p.total_bands);
+            if (p.order != nullptr) {
+                const int2 u = __ldg(p.order + unit);
+                seg = u.x;
+                gb = u.y;
+            } else {
+                seg = int(unit / p.total_bands);
+                gb = int(unit - (long long)seg * p.total_bands);
+            }
             j0 = seg * p.segc;
             j1 = min(p.nc, j0 + p.segc);
         } else {
@@ -453,7 +512,6 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 
         if (warp < W) {
             // ================= compute warps =================
-            const int rbase = warp * R;                  // first row of this warp in the band
             // column-sum seed: added to the strip's first row (warp 0, row 0)
             const bool seeded = p.cseed.n > 0 && gb == 0 && warp == 0;
             if (seeded) colseed_wait(p.cseed);
@@ -492,9 +550,6 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             }
             const TI* gin = reinterpret_cast<const TI*>(p.in) + int64_t(img) * img_elems;
             T* gout = reinterpret_cast<T*>(p.out) + int64_t(img) * img_elems;
-            // this warp's TMEM lanes (32*(warp%4) ..) and column range
-            const uint32_t tm_warp = tmem_base + ((uint32_t(32 * (warp & 3))) << 16)
-                                     + uint32_t((warp >> 2) * TC::per_warp);
 
             // store R rows of 4 values to the output (16-B vectors on the TMA
             // path, where cols % 4 == 0; guarded scalars otherwise)
@@ -531,10 +586,24 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         if (traced && warp == 0 && lane == 0)
                             p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
                     }
-                    const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
-                                  + size_t(rbase) * TW + 4 * lane;
+                    if constexpr (BULK) {
+                        // slot = [TH][SUB*TW] row pieces (1-D bulk copies); rows
+                        // beyond the image and columns beyond the matrix were
+                        // not copied: read as 0
+                        const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(rbase) * (SUB * TW)
+                                      + size_t(k % SUB) * TW + 4 * lane;
+                        const bool cin = int64_t(j0 + k) * TW + 4 * lane < p.cols;
 #pragma unroll
-                    for (int r = 0; r < R; ++r) v[r] = lds4_in<T, TI>(t + r * TW);
+                        for (int r = 0; r < R; ++r) {
+                            v[r] = lds4_in<T, TI>(t + r * (SUB * TW));
+                            if (!cin || row0 + rbase + r >= p.rows) v[r] = V4<T>{T(0), T(0), T(0), T(0)};
+                        }
+                    } else {
+                        const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
+                                      + size_t(rbase) * TW + 4 * lane;
+#pragma unroll
+                        for (int r = 0; r < R; ++r) v[r] = lds4_in<T, TI>(t + r * TW);
+                    }
                     if (k % SUB == SUB - 1 || k == nch - 1) {
                         // release the slot to the next TMA write only once the
                         // generic-proxy reads have landed in registers (the
@@ -579,48 +648,19 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     }
                     tmem_st<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
                     sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
+                    if (lane == 0) wmeta[it % DT] = make_int2(gb, j0 + k);
                     mbar_arrive(&colr[it % XS]);
                 }
             };
-            // finish(k): + (SAT row above the band + bottom rows of the warps
-            // above), from the add vector the control warp left in xbuf
-            auto finish = [&](int k) {
-                const uint32_t it = g + k;
-                mbar_wait(&topr[it % XS], (it / XS) & 1);
-                if constexpr (kDebug) {
-                    if (traced && warp == 0 && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 6] = globaltimer();
-                }
-                const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
-                uint32_t u[TC::per_chunk];
-                tmem_wait_st();
-                tmem_ld<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
-                tmem_wait_ld();
-                V4<T> v[R];
-#pragma unroll
-                for (int r = 0; r < R; ++r) {
-                    const uint32_t* q = u + 4 * r * NWE;
-                    v[r] = V4<T>{from_words<T>(q), from_words<T>(q + NWE), from_words<T>(q + 2 * NWE),
-                                 from_words<T>(q + 3 * NWE)};
-                    add4(v[r], add);
-                }
-                store_rows(v, k);
-                if constexpr (kDebug) {
-                    if (traced && warp == 0 && lane == 0)
-                        p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 3] = globaltimer();
-                }
-            };
-
             if constexpr (!HOLD) {
                 for (int k = 0; k < nch; ++k) local(k);
             } else {
                 for (int k = 0; k < nch; ++k) {
                     local(k);
                     diag_mark(p.diag, uint32_t(unit), uint32_t(k), 2);
-                    if (k >= DT - 1) finish(k - (DT - 1));
+                    if (g + k >= uint32_t(DT - 1)) finish_it(g + k - (DT - 1));
                     diag_mark(p.diag, uint32_t(unit), uint32_t(k), 3);
                 }
-                for (int k = (nch > DT - 1 ? nch - (DT - 1) : 0); k < nch; ++k) finish(k);
             }
             if (seeded && p.cseed.acks != nullptr) {
                 // every seed vector this unit needed has been read (the values
@@ -707,8 +747,15 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                     for (int i = 0; i < CPL; ++i) top[i] = T(0);
                     unsigned long long hops = 0, polls = 0;
-                    if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
-                    if (!lookback) {
+                    const bool xnopub = p.xcfg == 31, xnowalk = p.xcfg >= 30 && p.xcfg < 40;   // dev timing probes (wrong results)
+                    if (publish && band > 0 && !xnopub) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                    if (p.xcfg >= 32 && p.xcfg < 40) {
+                        // fake walk: the look-back's latency without its loads
+                        const unsigned long long t0 = globaltimer();
+                        const unsigned long long wait = (p.xcfg - 31) * 2000ull;   // 32: 2 us, 33: 4 us, 35: 8 us
+                        while (globaltimer() - t0 < wait) __nanosleep(200);
+                    } else if (xnowalk) {
+                    } else if (!lookback) {
                         lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
                     } else if (band == 0) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
@@ -782,7 +829,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             else kb -= LBW;
                         }
                     }
-                    if (publish) {
+                    if (publish && !xnopub) {
                         T inc[CPL];
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
@@ -809,7 +856,26 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             }
         } else {
             // ================= producer warp: TMA load ring =================
-            if constexpr (TMA) {
+            if constexpr (TMA && BULK) {
+                // every lane issues 1-D bulk copies of whole row pieces
+                // (SUB*TW elements, >= 1 KB): long contiguous DRAM runs
+                const uint64_t pol = policy_evict_first();
+                const TI* gin = reinterpret_cast<const TI*>(p.in) + int64_t(img) * img_elems;
+                const int nrows = int(min(int64_t(TH), p.rows - int64_t(row0)));
+                for (int k0 = 0; k0 < nch; k0 += SUB) {
+                    const uint32_t q = gq + uint32_t(k0 / SUB);
+                    const int s = q % S;
+                    const int64_t c0 = int64_t(j0 + k0) * TW;
+                    const uint32_t bytes = uint32_t(min(int64_t(SUB) * TW, p.cols - c0) * int64_t(sizeof(TI)));
+                    if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
+                    if (lane == 0) mbar_arrive_expect_tx(&full[s], bytes * uint32_t(nrows));
+                    __syncwarp();
+                    TI* dst = tiles + size_t(s) * SM::slot_elems;
+                    for (int r = lane; r < nrows; r += 32)
+                        bulk_load(dst + size_t(r) * (SUB * TW), gin + (int64_t(row0) + r) * p.cols + c0, bytes,
+                                  &full[s], pol);
+                }
+            } else if constexpr (TMA) {
                 if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
                     for (int k0 = 0; k0 < nch; k0 += SUB) {
@@ -831,6 +897,11 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
         diag_mark(p.diag, uint32_t(unit), uint32_t(nch), 5);
         g += nch;
         gq += uint32_t((nch + SUB - 1) / SUB);
+    }
+    if constexpr (HOLD) {
+        // the last DT-1 parked chunks of the stream
+        if (warp < W)
+            for (uint32_t it = g > uint32_t(DT - 1) ? g - (DT - 1) : 0u; it < g; ++it) finish_it(it);
     }
     diag_mark(p.diag, 0xFFFFFFFFu, 0, 6);
     if (HOLD) {

@@ -85,6 +85,14 @@ struct BandParams {
     int nseg;                  // 1 = whole bands
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
+    // Ticket order of the segment units (nullable = segment-major): order[t]
+    // = (segment, band) of ticket t, sorted by band + K * segment (DESIGN.md
+    // Sec. 4.6): both predecessors of a unit -- the same segment of the band
+    // above (vertical carry) and the previous segment of the same band (row
+    // carry) -- hold earlier tickets, and consecutive bands of one segment
+    // run ~nseg tickets apart instead of adjacent (no look-back lockstep).
+    const int2* order;
+    int xcfg;                  // development A/B: alternative band configuration (0 = default)
     unsigned long long* trace; // debug builds (SAT_DEBUG): [total_bands*nc][8] event times (ns), nullable
     unsigned int* diag;        // debug builds: host-mapped progress marks, nullable
 };

@@ -160,6 +160,16 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* m, uin
            "r"(smem_u32(bar)), "l"(policy)
         : "memory");
 }
+// 1-D bulk copy global -> shared (contiguous `bytes`, a multiple of 16, both
+// addresses 16-B aligned), completing tx bytes on `bar`
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                          uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1], %2, [%3], %4;"
+        :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy)
+        : "memory");
+}
 // HBM -> L2 only (no shared memory, no barrier): raises the bytes in flight
 // per SM beyond the shared-memory ring
 __device__ __forceinline__ void tma_prefetch_3d(const CUtensorMap* m, int c0, int c1, int c2) {

@@ -1,0 +1,62 @@
+"""A/B of 1R1W band configurations (development): for each config
+(tile_rows, xcfg, segments) first a parity gate against the CPU oracle on a
+3000 x 4096 int32 matrix, then kernel-only timing of each shape (median of
+reps CUDA-event launches, L2 flushed before each), configs interleaved in
+rounds to cancel clock drift.
+
+python tools/ab_sat.py "16384x16384,65536x65536" "128:0:0,64:1:0,64:2:0" [reps] [rounds] [dtype]
+"""
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import oracle
+import paper_conf_icpp_kasagini14_b200 as libsat
+from sat_inputs import make_np, make_torch
+
+shapes = [tuple(int(v) for v in s.split("x")) for s in sys.argv[1].split(",")]
+cfgs = [tuple(int(v) for v in c.split(":")) for c in sys.argv[2].split(",")]
+reps = int(sys.argv[3]) if len(sys.argv) > 3 else 10
+rounds = int(sys.argv[4]) if len(sys.argv) > 4 else 3
+dtype = sys.argv[5] if len(sys.argv) > 5 else "int32"
+dist = "u32" if dtype == "int32" else "unit"
+
+ok = {}
+a = make_np(3000, 4096, dtype, dist, seed=5)
+ref = oracle.sat(a)
+xa = torch.from_numpy(a).cuda()
+for c in cfgs:
+    th, xc, seg = c
+    got = libsat.sat(xa, tile_rows=th, xcfg=xc, segments=seg).cpu().numpy()
+    ok[c] = bool(np.array_equal(got, ref)) if dtype == "int32" else oracle.max_rel_err(got, ref) <= 1e-5
+    print(f"parity th={th} xcfg={xc} seg={seg}: {ok[c]} (th used {libsat.last_tile_rows()})", flush=True)
+
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+for (n, m) in shapes:
+    x = make_torch(n, m, dtype, dist, seed=1, device="cuda")
+    y = torch.empty_like(x)
+    res = {c: [] for c in cfgs}
+    for c in cfgs:
+        for _ in range(2):
+            libsat.sat(x, out=y, tile_rows=c[0], xcfg=c[1], segments=c[2])
+    for _ in range(rounds):
+        for c in cfgs:
+            for _ in range(reps):
+                flush.fill_(1)
+                s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s.record()
+                libsat.sat(x, out=y, tile_rows=c[0], xcfg=c[1], segments=c[2])
+                e.record()
+                e.synchronize()
+                res[c].append(s.elapsed_time(e))
+    nb = 2 * x.numel() * x.element_size()
+    for c in cfgs:
+        ms = statistics.median(res[c])
+        print(f"{n}x{m} {dtype} th={c[0]} xcfg={c[1]} seg={c[2]} median {ms:.4f} ms min {min(res[c]):.4f} "
+              f"{nb / ms / 1e6:.0f} GB/s frac {nb / ms / 1e6 / 6550.1:.3f} parity={ok[c]}", flush=True)
+    del x, y
+    torch.cuda.empty_cache()

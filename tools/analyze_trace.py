@@ -40,3 +40,18 @@ print("hops: mean %.2f max %d; share of chunks with hops>1: %.3f; polls mean %.2
 bi = np.arange(nb)
 for q in (0, 1, 2, nb // 4, nb // 2, nb - 1):
     print("  band %4d: lb med %.2f hops %.1f polls %.1f end %.1f" % (q, np.median(t[q, :, 2] - t[q, :, 1]), hops[q].mean(), polls[q].mean(), t[q, -1, 3]))
+# compute-warp stall at finish(J): the add vector arrived (t6) after the
+# compute warps had finished local(J + DT - 1) (t1 of that chunk)
+DT = int(sys.argv[2]) if len(sys.argv) > 2 else 4
+if nc > DT:
+    stall = t[:, :nc - DT + 1, 6] - t[:, DT - 1:, 1]
+    stall = np.maximum(stall, 0)
+    print("finish stall per chunk (us): mean %.2f p50 %.2f p90 %.2f; total per band mean %.1f max %.1f" % (
+        stall.mean(), np.median(stall), np.percentile(stall, 90), stall.sum(1).mean(), stall.sum(1).max()))
+    for q in (0, 1, 8, nb // 4, nb // 2, 3 * nb // 4, nb - 1):
+        print("  band %4d: stall total %.1f us, lb med %.2f, arrival period med %.2f" % (
+            q, stall[q].sum(), np.median(t[q, :, 2] - t[q, :, 1]), np.median(np.diff(t[q, :, 0]))))
+# propagation of the inclusive down the bands for a middle chunk
+J = nc // 2
+print("chunk %d: local done (t1) by band: " % J + " ".join("%.1f" % v for v in t[::max(1, nb // 16), J, 1]))
+print("chunk %d: look-back done (t2) by band: " % J + " ".join("%.1f" % v for v in t[::max(1, nb // 16), J, 2]))
