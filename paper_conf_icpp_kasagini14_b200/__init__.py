@@ -134,10 +134,9 @@ def _check_dev(*ts):
 
 
 def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
-            jitter: int = 0, segments: int = 0, xcfg: int = 0) -> SatOptions:
+            jitter: int = 0, segments: int = 0) -> SatOptions:
     o = SatOptions()
     _lib.sat_options_init(ctypes.byref(o))
-    o.reserved[0] = int(xcfg)
     o.r = float(r)
     o.tile_rows = int(tile_rows)
     o.force_generic = int(bool(force_generic))
@@ -147,7 +146,7 @@ def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
 
 
 def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
-        force_generic: bool = False, jitter: int = 0, segments: int = 0, stream=None, xcfg: int = 0):
+        force_generic: bool = False, jitter: int = 0, segments: int = 0, stream=None):
     """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32/float64 IEEE).
 
     ``out`` may be ``x`` itself (in place).  ``variant`` in
@@ -161,7 +160,7 @@ def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
     _check_dev(x, out)
     if out.shape != x.shape or out.dtype != x.dtype:
         raise ValueError("out must match x in shape and dtype")
-    o = options(r, tile_rows, force_generic, jitter, segments, xcfg)
+    o = options(r, tile_rows, force_generic, jitter, segments)
     _check(_lib.sat_compute_ex(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                _dtype_code(x), VARIANTS[variant], ctypes.byref(o), _stream(stream)))
     return out

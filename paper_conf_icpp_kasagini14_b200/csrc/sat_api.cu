@@ -69,6 +69,7 @@ constexpr int kMaxDev = 64;
 
 struct DevInfo {
     int sms = 0;
+    int l2 = 0;
     int smem_optin = 0;
     int smem_sm = 0;
     bool ok = false;
@@ -86,6 +87,7 @@ int get_dev(int& dev, DevInfo& info) {
         CUDA_TRY(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
         CUDA_TRY(cudaDeviceGetAttribute(&d.smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
         CUDA_TRY(cudaDeviceGetAttribute(&d.smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+        CUDA_TRY(cudaDeviceGetAttribute(&d.l2, cudaDevAttrL2CacheSize, dev));
         d.ok = true;
     }
     if (!g_encode) {
@@ -122,8 +124,6 @@ struct Workspace {
     Buf box;                  // box filter: the SAT it reads
     Buf part;                 // column totals partials
     Buf cnt;                  // column totals: per-chunk-column and global arrival counters (self-resetting)
-    Buf order;                // segment-unit ticket order (int2 per unit), for order_key
-    unsigned long long order_key = 0;
     Buf shard;                // sharded default workspace
     Buf din, dout;            // host e2e device copies
     std::vector<void*> retired;   // buffers a captured graph may still reference (freed by sat_release_workspace)
@@ -263,10 +263,15 @@ struct BandCfg {
 // per compute thread.  Two CTAs per SM.
 constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 1, 2};
 constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
+// column / row passes (2R2W, 4R4W) at TH 64: two CTAs per SM
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
-// TH 64 with >= 4 waves of bands ("big"): one CTA per SM, 192 KB ring of
-// 64 x 256 slots (1-KB row segments), 6 chunks parked in TMEM
-constexpr BandCfg kCfg64B{8, 8, 3, 6, 2, 4, 1, 1};
+// 1R1W at TH 64 ("wide"): one CTA per SM, 192 KB ring of 64 x 256 slots
+// (1-KB row segments per TMA load pair), 8 chunks parked in TMEM (all 512
+// columns).  Between one half and two thirds of a wave of 128-row bands it
+// beats both TH 32 and TH 128: 6144^2 int32 0.084 vs 0.094 ms (TH 32),
+// 8192^2 0.127 vs 0.143, 10240^2 0.179 vs 0.198 (TH 128); the two-CTA TH-64
+// configuration was 20-30 % slower (profiles/r02_ab_th.txt)
+constexpr BandCfg kCfg64W{8, 8, 3, 8, 2, 4, 1, 1};
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
@@ -284,10 +289,10 @@ constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM co
 constexpr BandCfg kCfgU64{8, 8, 6, 4, 1, 4, 1, 2};
 constexpr BandCfg kCfgU128{8, 16, 6, 4, 1, 3, 1, 1};
 
-// CTAs per SM of a configuration (for wave counts before launch)
-int ctas_per_sm(int dtype, int th, bool big) {
+// CTAs per SM of a 1R1W-family configuration (for wave counts before launch)
+int ctas_per_sm(int dtype, int th) {
     if (dtype == SAT_FLOAT64) return th == 16 ? 2 : 1;
-    return (th >= 128 || big) ? 1 : 2;
+    return th >= 64 ? 1 : 2;
 }
 
 // One-time per (instantiation, device) launch set-up, shared by all threads.
@@ -298,9 +303,9 @@ struct KernelSetup {
 };
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW = 0, typename TI = T, bool BULK = false>
+          int LBW = 0, typename TI = T>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI, BULK>;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI>;
     const size_t smem = BandSmem<T, R, W, S, DT, SUB, TI>::total;
     const int threads = (W + NCW + 1) * 32;
     // per instantiation and device: attributes set once, resources queried
@@ -360,7 +365,7 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di,
 #define SAT_CFG(c) c.R, c.W, c.S, c.DT, c.SUB, c.NCW, c.NS
 // Band heights instantiated per (dtype, mode, path); `band_th` maps a
 // requested height onto them.  1R1W family (MODE_SAT) on the TMA path: int32 /
-// float32 16, 32, 64, 128 (+ the "big" TH-64 configuration), float64 16, 32,
+// float32 16, 32, 64 ("wide", one CTA per SM), 128, float64 16, 32,
 // 64; the column and row passes of 2R2W / 4R4W: 32 and 64; the generic
 // (non-TMA) path: 32 (and 128 for 4-byte 1R1W).
 int band_th(int mode, int dtype, bool tma, int th) {
@@ -399,21 +404,10 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
         }
         return fail(SAT_ERR_INVALID, "float64: no band configuration for this tile_rows");
     } else {
-        if (p.xcfg == 1 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 0, T, true>(p, ti, di, st, grid);
-        if (p.xcfg == 2 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 0, T, false>(p, ti, di, st, grid);
-        if (p.xcfg == 4 && th == 32) return launch_band_t<T, 8, 4, 3, 8, 4, 4, 1, MODE, TMA, 1, 0, T, true>(p, ti, di, st, grid);
-        if (p.xcfg == 5 && th == 32) return launch_band_t<T, 8, 4, 3, 8, 2, 4, 1, MODE, TMA, 2, 0, T, true>(p, ti, di, st, grid);
-        if (p.xcfg == 7 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 8>(p, ti, di, st, grid);
-        if (p.xcfg == 8 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 8>(p, ti, di, st, grid);
-        if (p.xcfg == 9 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 4>(p, ti, di, st, grid);
-        if (p.xcfg == 10 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 3, 1, MODE, TMA, 1, 2>(p, ti, di, st, grid);
-        if (p.xcfg == 11 && th == 128) return launch_band_t<T, 16, 8, 3, 4, 1, 4, 1, MODE, TMA, 1, 12>(p, ti, di, st, grid);
-        if (p.xcfg == 6 && th == 64) return launch_band_t<T, 8, 8, 3, 8, 2, 4, 1, MODE, TMA, 1, 2, T, true>(p, ti, di, st, grid);
-        if (p.big && th == 64) return launch_band_t<T, SAT_CFG(kCfg64B), MODE, TMA, kCfg64B.MINB>(p, ti, di, st, grid);
         switch (th) {
             case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, di, st, grid);
             case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
-            case 64: return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfg64W), MODE, TMA, kCfg64W.MINB>(p, ti, di, st, grid);
             case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
         }
         return fail(SAT_ERR_INVALID, "no band configuration for this tile_rows");
@@ -470,15 +464,16 @@ int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dty
         }
         return rows * batch >= 1024 ? 32 : 16;
     }
-    // 1R1W: TH = 128 (one CTA per SM) once its bands fill half the SMs: in
-    // the one-wave regime the look-back chain (one hop per band) costs more
-    // than idle SMs (A/B sweep, int32: 10240^2 0.200 ms vs 0.224 for TH 32,
-    // 12288^2 0.254 vs 0.313, 14336^2 0.327 vs 0.417; 16K^2+: 5.3-5.4 TB/s vs
-    // 5.0 for TH 64); below that TH 32 from 1536 rows (2048^2-8192^2: 15-25 %
-    // faster than TH 16), else TH 16.
+    // 1R1W (one CTA per SM for TH 64 and 128; r02 sweep, profiles/r02_ab_th.txt):
+    // TH = 128 once its bands fill about two thirds of the SMs (the look-back
+    // chain is one hop per band; 16K^2+: 5.3-5.4 TB/s); the wide TH 64 below
+    // that while its bands fill 60 % of the SMs (6144^2-10240^2: 9-11 %
+    // faster than TH 32 or 128); then TH 32 from 1536 rows (2048^2-4096^2:
+    // 15-25 % faster than TH 16), else TH 16.
     if (variant == SAT_1R1W || variant == SAT_1PLUSR_R1W) {   // (1+r): its band C is 1R1W
-        const long long b128 = batch * ((rows + 127) / 128);
-        if (b128 * 2 >= di.sms) return 128;
+        const long long b128 = batch * ((rows + 127) / 128), b64 = batch * ((rows + 63) / 64);
+        if (b128 * 100 >= 65LL * di.sms) return 128;
+        if (b64 * 10 >= 6LL * di.sms) return 64;
         return rows * batch >= 1536 ? 32 : 16;
     }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
@@ -499,7 +494,6 @@ struct Job {
     bool tma;
     int jitter;
     int segments;     // sat_options.segments: 0 = automatic band segments
-    int xcfg;         // development A/B (sat_options.reserved[0])
     const DevInfo* di;
     Workspace* ws;
     cudaStream_t st;
@@ -558,10 +552,6 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * ((p.nc + p.tile_units - 1) / p.tile_units)
                                  : p.total_bands;
-    // Many bands (>= 4 waves of one CTA per SM): one CTA per SM with twice the
-    // ring and 1-KB row segments per TMA load.
-    p.big = (mode == MODE_SAT && j.tma && j.th == 64 && j.dtype != SAT_FLOAT64 && j.in_dtype == j.dtype &&
-             p.total_bands >= 4 * j.di->sms && !j.xcfg) ? 1 : 0;
     // Band segments: short units for the last wave when
     // bands are many waves deep
     p.nseg = 1;
@@ -574,7 +564,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         // 20480^2: 0.614 ms with 8-10 vs 0.887 ms; 12288^2 float64: 0.608 vs
         // 0.785 ms); at most one wave: whole bands (a segment would wait for
         // the band's previous segment)
-        const int slots = j.di->sms * (j.xcfg == 5 ? 2 : (j.xcfg && j.th != 128) ? 1 : ctas_per_sm(j.dtype, j.th, p.big != 0));
+        const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th);
         int want = p.total_bands > slots ? std::min(16, p.nc / 16) : 1;
         if (j.segments > 0) want = j.segments;
         if (want > 1 && p.nc > 1) {
@@ -583,30 +573,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
             p.total_units = (long long)p.total_bands * p.nseg;
         }
     }
-    // skewed ticket order of the segment units
-    p.order = nullptr;
-    if (p.nseg > 1 && (j.xcfg == 40 || j.xcfg == 41)) {
-        const int K = std::max(1, (j.xcfg == 41 ? 4 : 2) * j.di->sms * ctas_per_sm(j.dtype, j.th, p.big != 0) / p.nseg);
-        const unsigned long long key = (unsigned long long)p.total_bands | ((unsigned long long)p.nseg << 32) |
-                                       ((unsigned long long)K << 44);
-        Workspace& w = *j.ws;
-        if (w.order_key != key || !w.order.p) {
-            std::vector<int2> ord;
-            ord.reserve(size_t(p.total_bands) * p.nseg);
-            const long long kmax = (long long)p.total_bands - 1 + (long long)K * (p.nseg - 1);
-            for (long long d = 0; d <= kmax; ++d)
-                for (int sg = 0; sg < p.nseg; ++sg) {
-                    const long long b = d - (long long)K * sg;
-                    if (b >= 0 && b < p.total_bands) ord.push_back(make_int2(sg, int(b)));
-                }
-            SAT_TRY(ensure(w.order, ord.size() * sizeof(int2), false));
-            CUDA_TRY(cudaMemcpy(w.order.p, ord.data(), ord.size() * sizeof(int2), cudaMemcpyHostToDevice));
-            w.order_key = key;
-        }
-        p.order = static_cast<const int2*>(w.order.p);
-    }
     p.jitter = j.jitter;
-    p.xcfg = (mode == MODE_SAT && j.tma && j.dtype != SAT_FLOAT64 && j.in_dtype == j.dtype) ? j.xcfg : 0;
     if (kDebug) {
         p.diag = g_diag_dev;
         if (mode == MODE_SAT && p.top_src == TOP_LOOKBACK && t_trace) {
@@ -858,7 +825,6 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     j.tma = !o.force_generic && tma_ok(in, out, cols, in_dtype);
     j.jitter = o.jitter;
     j.segments = o.segments;
-    j.xcfg = o.reserved[0];
     j.di = &di;
     j.ws = ws;
     j.st = st;
@@ -1511,7 +1477,7 @@ int sat_release_workspace(void* stream) {
     // the stream's queued work may still use the buffers
     CUDA_TRY(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     for (Buf* b : {&w->desc, &w->lseg, &w->ticket, &w->bt, &w->rs, &w->lx, &w->lsum, &w->topx, &w->lb,
-                   &w->tr, &w->box, &w->part, &w->cnt, &w->order, &w->shard, &w->din, &w->dout})
+                   &w->tr, &w->box, &w->part, &w->cnt, &w->shard, &w->din, &w->dout})
         free_buf(*b);
     for (void* p : w->retired) cudaFree(p);
     if (w->cstream_in) cudaStreamDestroy(w->cstream_in);

@@ -321,7 +321,7 @@ __device__ __forceinline__ V4<T> colseed4(const ColSeed& cs, int64_t c, int64_t 
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW_ = 0, typename TI = T, bool BULK = false>
+          int LBW_ = 0, typename TI = T>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
@@ -489,14 +489,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             j0 = min(r1, r0 + sr * p.tile_units);
             j1 = min(r1, j0 + p.tile_units);
         } else if (p.nseg > 1) {
-            if (p.order != nullptr) {
-                const int2 u = __ldg(p.order + unit);
-                seg = u.x;
-                gb = u.y;
-            } else {
-                seg = int(unit / p.total_bands);
-                gb = int(unit - (long long)seg * p.total_bands);
-            }
+            seg = int(unit / p.total_bands);
+            gb = int(unit - (long long)seg * p.total_bands);
             j0 = seg * p.segc;
             j1 = min(p.nc, j0 + p.segc);
         } else {
@@ -586,19 +580,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         if (traced && warp == 0 && lane == 0)
                             p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
                     }
-                    if constexpr (BULK) {
-                        // slot = [TH][SUB*TW] row pieces (1-D bulk copies); rows
-                        // beyond the image and columns beyond the matrix were
-                        // not copied: read as 0
-                        const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(rbase) * (SUB * TW)
-                                      + size_t(k % SUB) * TW + 4 * lane;
-                        const bool cin = int64_t(j0 + k) * TW + 4 * lane < p.cols;
-#pragma unroll
-                        for (int r = 0; r < R; ++r) {
-                            v[r] = lds4_in<T, TI>(t + r * (SUB * TW));
-                            if (!cin || row0 + rbase + r >= p.rows) v[r] = V4<T>{T(0), T(0), T(0), T(0)};
-                        }
-                    } else {
+                    {
                         const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
                                       + size_t(rbase) * TW + 4 * lane;
 #pragma unroll
@@ -747,15 +729,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                     for (int i = 0; i < CPL; ++i) top[i] = T(0);
                     unsigned long long hops = 0, polls = 0;
-                    const bool xnopub = p.xcfg == 31, xnowalk = p.xcfg >= 30 && p.xcfg < 40;   // dev timing probes (wrong results)
-                    if (publish && band > 0 && !xnopub) publish_words<T, CPL>(my, tagbase | 1u, agg);
-                    if (p.xcfg >= 32 && p.xcfg < 40) {
-                        // fake walk: the look-back's latency without its loads
-                        const unsigned long long t0 = globaltimer();
-                        const unsigned long long wait = (p.xcfg - 31) * 2000ull;   // 32: 2 us, 33: 4 us, 35: 8 us
-                        while (globaltimer() - t0 < wait) __nanosleep(200);
-                    } else if (xnowalk) {
-                    } else if (!lookback) {
+                    if (publish && band > 0) publish_words<T, CPL>(my, tagbase | 1u, agg);
+                    if (!lookback) {
                         lds_cols<T, CPL>(reinterpret_cast<const T*>(p.TopX) + int64_t(gb) * desc_w + c0, top);
                     } else if (band == 0) {
                         if (p.seed_kind != SEED_NONE && img == 0) {
@@ -829,7 +804,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             else kb -= LBW;
                         }
                     }
-                    if (publish && !xnopub) {
+                    if (publish) {
                         T inc[CPL];
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
@@ -856,26 +831,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             }
         } else {
             // ================= producer warp: TMA load ring =================
-            if constexpr (TMA && BULK) {
-                // every lane issues 1-D bulk copies of whole row pieces
-                // (SUB*TW elements, >= 1 KB): long contiguous DRAM runs
-                const uint64_t pol = policy_evict_first();
-                const TI* gin = reinterpret_cast<const TI*>(p.in) + int64_t(img) * img_elems;
-                const int nrows = int(min(int64_t(TH), p.rows - int64_t(row0)));
-                for (int k0 = 0; k0 < nch; k0 += SUB) {
-                    const uint32_t q = gq + uint32_t(k0 / SUB);
-                    const int s = q % S;
-                    const int64_t c0 = int64_t(j0 + k0) * TW;
-                    const uint32_t bytes = uint32_t(min(int64_t(SUB) * TW, p.cols - c0) * int64_t(sizeof(TI)));
-                    if (q >= uint32_t(S)) mbar_wait(&empty[s], ((q / S) & 1) ^ 1u);
-                    if (lane == 0) mbar_arrive_expect_tx(&full[s], bytes * uint32_t(nrows));
-                    __syncwarp();
-                    TI* dst = tiles + size_t(s) * SM::slot_elems;
-                    for (int r = lane; r < nrows; r += 32)
-                        bulk_load(dst + size_t(r) * (SUB * TW), gin + (int64_t(row0) + r) * p.cols + c0, bytes,
-                                  &full[s], pol);
-                }
-            } else if constexpr (TMA) {
+            if constexpr (TMA) {
                 if (lane == 0) {
                     const uint64_t pol = policy_evict_first();
                     for (int k0 = 0; k0 < nch; k0 += SUB) {

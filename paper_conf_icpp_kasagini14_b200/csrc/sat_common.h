@@ -63,7 +63,6 @@ struct BandParams {
     int total_bands;           // batch * nb
     long long total_units;     // bands (band units) or bands*nc (tile units)
     int tile_units;            // K > 0: one ticket = K consecutive tiles of a band (external carries); 0 = whole bands
-    int big;                   // 1: one CTA per SM with a 2x ring of 1-KB row segments (TH 64)
     uint64_t* desc;            // [total_bands][nc*TW] look-back descriptor words
     unsigned long long* ticket;
     unsigned long long base;   // ticket base of this launch (also the tag base)
@@ -85,14 +84,6 @@ struct BandParams {
     int nseg;                  // 1 = whole bands
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
-    // Ticket order of the segment units (nullable = segment-major): order[t]
-    // = (segment, band) of ticket t, sorted by band + K * segment (DESIGN.md
-    // Sec. 4.6): both predecessors of a unit -- the same segment of the band
-    // above (vertical carry) and the previous segment of the same band (row
-    // carry) -- hold earlier tickets, and consecutive bands of one segment
-    // run ~nseg tickets apart instead of adjacent (no look-back lockstep).
-    const int2* order;
-    int xcfg;                  // development A/B: alternative band configuration (0 = default)
     unsigned long long* trace; // debug builds (SAT_DEBUG): [total_bands*nc][8] event times (ns), nullable
     unsigned int* diag;        // debug builds: host-mapped progress marks, nullable
 };

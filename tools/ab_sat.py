@@ -1,10 +1,10 @@
 """A/B of 1R1W band configurations (development): for each config
-(tile_rows, xcfg, segments) first a parity gate against the CPU oracle on a
+(tile_rows, segments) first a parity gate against the CPU oracle on a
 3000 x 4096 int32 matrix, then kernel-only timing of each shape (median of
 reps CUDA-event launches, L2 flushed before each), configs interleaved in
 rounds to cancel clock drift.
 
-python tools/ab_sat.py "16384x16384,65536x65536" "128:0:0,64:1:0,64:2:0" [reps] [rounds] [dtype]
+python tools/ab_sat.py "16384x16384,65536x65536" "128:0,64:0" [reps] [rounds] [dtype]
 """
 import os
 import statistics
@@ -30,10 +30,10 @@ a = make_np(3000, 4096, dtype, dist, seed=5)
 ref = oracle.sat(a)
 xa = torch.from_numpy(a).cuda()
 for c in cfgs:
-    th, xc, seg = c
-    got = libsat.sat(xa, tile_rows=th, xcfg=xc, segments=seg).cpu().numpy()
+    th, seg = c
+    got = libsat.sat(xa, tile_rows=th, segments=seg).cpu().numpy()
     ok[c] = bool(np.array_equal(got, ref)) if dtype == "int32" else oracle.max_rel_err(got, ref) <= 1e-5
-    print(f"parity th={th} xcfg={xc} seg={seg}: {ok[c]} (th used {libsat.last_tile_rows()})", flush=True)
+    print(f"parity th={th} seg={seg}: {ok[c]} (th used {libsat.last_tile_rows()})", flush=True)
 
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 for (n, m) in shapes:
@@ -42,21 +42,21 @@ for (n, m) in shapes:
     res = {c: [] for c in cfgs}
     for c in cfgs:
         for _ in range(2):
-            libsat.sat(x, out=y, tile_rows=c[0], xcfg=c[1], segments=c[2])
+            libsat.sat(x, out=y, tile_rows=c[0], segments=c[1])
     for _ in range(rounds):
         for c in cfgs:
             for _ in range(reps):
                 flush.fill_(1)
                 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 s.record()
-                libsat.sat(x, out=y, tile_rows=c[0], xcfg=c[1], segments=c[2])
+                libsat.sat(x, out=y, tile_rows=c[0], segments=c[1])
                 e.record()
                 e.synchronize()
                 res[c].append(s.elapsed_time(e))
     nb = 2 * x.numel() * x.element_size()
     for c in cfgs:
         ms = statistics.median(res[c])
-        print(f"{n}x{m} {dtype} th={c[0]} xcfg={c[1]} seg={c[2]} median {ms:.4f} ms min {min(res[c]):.4f} "
+        print(f"{n}x{m} {dtype} th={c[0]} seg={c[1]} median {ms:.4f} ms min {min(res[c]):.4f} "
               f"{nb / ms / 1e6:.0f} GB/s frac {nb / ms / 1e6 / 6550.1:.3f} parity={ok[c]}", flush=True)
     del x, y
     torch.cuda.empty_cache()
