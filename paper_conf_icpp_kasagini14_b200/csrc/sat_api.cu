@@ -26,6 +26,7 @@
 #include "sat_band.cuh"
 #include "sat_paper.cuh"
 #include "sat_box.cuh"
+#include "sat_boxf.cuh"
 #include "sat_xchg.cuh"
 
 using namespace sat;
@@ -124,6 +125,7 @@ struct Workspace {
     Buf box;                  // box filter: the SAT it reads
     Buf part;                 // column totals partials
     Buf cnt;                  // column totals: per-chunk-column and global arrival counters (self-resetting)
+    Buf bticket;              // fused box filter: unit ticket (zeroed per call on the stream)
     Buf shard;                // sharded default workspace
     Buf din, dout;            // host e2e device copies
     std::vector<void*> retired;   // buffers a captured graph may still reference (freed by sat_release_workspace)
@@ -993,6 +995,53 @@ int sharded_fused_t(const void* in, void* out, int64_t strip_rows, PeerExchange&
     return SAT_OK;
 }
 
+// Fused box filter (sat_boxf.cuh): one launch, the SAT stays on chip.
+template <typename TI, typename TS, typename TO, int TH, int MAXH, int NS, int NWARP = 16>
+int box_fused_t(const void* in, int in_dtype, void* out, int64_t batch, int64_t rows, int64_t cols, int rr, int rc,
+                int normalize, const DevInfo& di, Workspace& ws, cudaStream_t st) {
+    auto kern = sat_boxf_kernel<TI, TS, TO, TH, MAXH, NS, NWARP>;
+    const size_t smem = BoxSmem<MAXH, NS, TI, TS, NWARP>::total;
+    static KernelSetup setup;
+    int dev = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    if (dev < 0 || dev >= kMaxDev) return fail(SAT_ERR_CUDA, "device ordinal out of range");
+    std::call_once(setup.once[dev], [&] {
+        setup.err[dev] = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    });
+    if (setup.err[dev] != cudaSuccess)
+        return fail(SAT_ERR_CUDA, std::string("box kernel set-up: ") + cudaGetErrorString(setup.err[dev]));
+    CUtensorMap tm;
+    std::memset(&tm, 0, sizeof(tm));
+    SAT_TRY(make_tmap(&tm, in, in_dtype, batch, rows, cols, MAXH));
+    SAT_TRY(ensure(ws.bticket, sizeof(unsigned long long), false));
+    CUDA_TRY(cudaMemsetAsync(ws.bticket.p, 0, sizeof(unsigned long long), st));
+    BoxParams bp;
+    bp.in = in; bp.out = out; bp.rows = int(rows); bp.cols = int(cols); bp.batch = int(batch);
+    bp.rr = rr; bp.rc = rc; bp.normalize = normalize;
+    bp.nb = int((rows + TH - 1) / TH);
+    bp.nc = int((cols + TW - 1) / TW);
+    bp.ticket = static_cast<unsigned long long*>(ws.bticket.p);
+    bp.base = 0;
+    const long long units = (long long)batch * bp.nb;
+    const int grid = int(std::min<long long>(units, di.sms));
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(unsigned(grid));
+    cfg.blockDim = dim3(NWARP * 32);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, tm, bp));
+    CUDA_TRY(cudaGetLastError());
+    t_launches = 1;
+    t_grid = grid;
+    return SAT_OK;
+}
+
 }  // namespace
 
 // ====================================================================== C ABI
@@ -1153,6 +1202,29 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
+    // Fused (one launch, the SAT never leaves the chip, sat_boxf.cuh) when the
+    // input is TMA-addressable, out does not alias it (a band's halo rows are
+    // another band's output rows), the halo fits the band buffer and rc < 128.
+    {
+        const bool al = (reinterpret_cast<uintptr_t>(in) & 15) == 0 && (reinterpret_cast<uintptr_t>(out) & 15) == 0;
+        const bool apart = in != out;
+        const bool u8 = in_dtype == SAT_UINT8 && cols % 16 == 0 && 2 * rr <= 32;
+        const bool i32 = in_dtype == SAT_INT32 && cols % 4 == 0 && 2 * rr <= 32;
+        const bool f32 = in_dtype == SAT_FLOAT32 && cols % 4 == 0 && 2 * rr <= 16;
+        if (al && apart && rc <= 127 && rows <= INT32_MAX && cols <= INT32_MAX && (u8 || i32 || f32)) {
+            if (u8)
+                return box_fused_t<uint8_t, uint32_t, int32_t, 64, 96, 4>(in, in_dtype, out, batch, rows, cols, rr, rc, 0,
+                                                                           di, *ws, st);
+            if (i32)
+                return box_fused_t<uint32_t, uint32_t, int32_t, 32, 64, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
+                                                                            0, di, *ws, st);
+            if (out_dtype == SAT_FLOAT32)
+                return box_fused_t<float, double, float, 32, 48, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
+                                                                     normalize, di, *ws, st);
+            return box_fused_t<float, double, double, 32, 48, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
+                                                                  normalize, di, *ws, st);
+        }
+    }
     SAT_TRY(ensure(ws->box, size_t(batch) * rows * cols * esize(sdt), false));
     // 1. the SAT (1R1W, widening uint8 -> uint32 and float32 -> float64 on load)
     SAT_TRY(compute_core(in, ws->box.p, batch, rows, cols, sdt, SAT_1R1W, nullptr, nullptr, nullptr,
@@ -1477,7 +1549,7 @@ int sat_release_workspace(void* stream) {
     // the stream's queued work may still use the buffers
     CUDA_TRY(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     for (Buf* b : {&w->desc, &w->lseg, &w->ticket, &w->bt, &w->rs, &w->lx, &w->lsum, &w->topx, &w->lb,
-                   &w->tr, &w->box, &w->part, &w->cnt, &w->shard, &w->din, &w->dout})
+                   &w->tr, &w->box, &w->part, &w->cnt, &w->bticket, &w->shard, &w->din, &w->dout})
         free_buf(*b);
     for (void* p : w->retired) cudaFree(p);
     if (w->cstream_in) cudaStreamDestroy(w->cstream_in);

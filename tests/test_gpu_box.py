@@ -180,3 +180,62 @@ def test_box_filter_cuda_graph(libsat):
         got = y.cpu().numpy()
         for b in range(B):
             assert np.array_equal(got[b], oracle.box_filter(a[b].astype(np.int32), rr, rc)), (it, b)
+
+
+# ------------------------------------------------------------------ fused box filter (sat_boxf.cuh)
+@pytest.mark.parametrize("shape,rr,rc,batch", [
+    ((1080, 1920), 4, 4, 3),       # the cfg5-style image batch (r = 4)
+    ((1000, 2064), 16, 127, 2),    # largest fused radii; partial last chunk (2064 = 16 x 128 + 16)
+    ((50, 16), 3, 9, 4),           # fewer rows than a band, one 16-column chunk
+    ((64, 256), 0, 0, 1),          # identity
+    ((130, 400), 16, 1, 1),        # window taller than the rows a band owns
+    ((777, 1296), 7, 100, 2),
+], ids=lambda v: str(v))
+def test_box_fused_uint8(libsat, shape, rr, rc, batch):
+    a = u8img(*shape, seed=shape[0] + rr, batch=batch)
+    y = libsat.box_filter(dev(a), rr, rc)
+    assert libsat.last_launch_count() == 1          # fused: one launch, no SAT in HBM
+    got = y.cpu().numpy()
+    for b in range(batch):
+        assert np.array_equal(got[b], oracle.box_filter(a[b].astype(np.int32), rr, rc)), b
+
+
+@pytest.mark.parametrize("rr,rc", [(1, 1), (16, 33), (5, 127)])
+def test_box_fused_int32_wrapping(libsat, rr, rc):
+    a = make_np(700, 1000, "int32", "u32", seed=rr + rc, batch=2)
+    y = libsat.box_filter(dev(a), rr, rc)
+    assert libsat.last_launch_count() == 1
+    got = y.cpu().numpy()
+    for b in range(2):
+        assert np.array_equal(got[b], oracle.box_filter(a[b], rr, rc))
+
+
+@pytest.mark.parametrize("normalize", [False, True])
+@pytest.mark.parametrize("rr,rc", [(4, 6), (8, 127), (0, 2)])
+def test_box_fused_float32(libsat, normalize, rr, rc):
+    """float32 input, float64 SAT on chip; dyadic inputs make every box sum
+    exact, so both output types match the correctly rounded oracle value."""
+    a = make_np(333, 1000, "float32", "unit", seed=rr * 7 + rc, batch=2)
+    for out_dtype in (torch.float32, torch.float64):
+        y = libsat.box_filter(dev(a), rr, rc, normalize=normalize, out_dtype=out_dtype)
+        assert libsat.last_launch_count() == 1
+        got = y.cpu().numpy()
+        for b in range(2):
+            ref = oracle.box_filter(a[b], rr, rc, normalize=normalize)
+            assert np.array_equal(got[b], ref.astype(got.dtype))
+
+
+def test_box_fused_matches_two_pass(libsat):
+    """The fused kernel and the two-pass path (forced by in-place output) agree
+    bit for bit; a radius beyond the fused limit takes the two-pass path."""
+    a = make_np(540, 960, "int32", "u32", seed=3)
+    x = dev(a)
+    fused = libsat.box_filter(x, 5, 9).cpu().numpy()
+    assert libsat.last_launch_count() == 1
+    y = x.clone()
+    libsat.box_filter(y, 5, 9, out=y)
+    assert libsat.last_launch_count() >= 2
+    assert np.array_equal(fused, y.cpu().numpy())
+    big = libsat.box_filter(x, 40, 3).cpu().numpy()
+    assert libsat.last_launch_count() >= 2
+    assert np.array_equal(big, oracle.box_filter(a, 40, 3))

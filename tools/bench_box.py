@@ -5,7 +5,8 @@ python tools/bench_box.py [--images 32] [--radius 4] [--reps 20]
 
 Lines (JSON): widening 1R1W uint8 -> int32 (1 + 4 B per pixel), float32 ->
 float64 (4 + 8 B), the box filter from uint8 pixels (SAT pass 1 + 4 B, box
-pass 4 + 4 B: 13 B per pixel; a fused kernel would need 1 + 4), and
+pass 4 + 4 B: 13 B per pixel in round 1; the fused kernel moves 1 x (1 +
+2r/TH) + 4 B), and
 rectangle-sum queries (random rectangles over the same images).  CUDA events
 around each call, median of --reps, a 512 MB L2 flush before each; bytes are
 algorithmic; peak = MEASURED_PEAKS.json hbm_gbs.
@@ -53,6 +54,7 @@ def main():
     i32 = torch.empty(B, n, m, dtype=torch.int32, device="cuda")
     f64 = torch.empty(B, n, m, dtype=torch.float64, device="cuda")
     box = torch.empty(B, n, m, dtype=torch.int32, device="cuda")
+    f32o = torch.empty(B, n, m, dtype=torch.float32, device="cuda")
     rects = torch.stack([torch.randint(0, B, (1 << 20,)), torch.randint(0, n, (1 << 20,)),
                          torch.randint(0, m, (1 << 20,)), torch.randint(0, n, (1 << 20,)),
                          torch.randint(0, m, (1 << 20,))], 1).to(torch.int32).cuda()
@@ -63,7 +65,10 @@ def main():
         ("widen u8->i32 1R1W", lambda: libsat.sat_widening(u8, torch.int32, out=i32), 5 * px, px),
         ("widen f32->f64 1R1W", lambda: libsat.sat_widening(f32, torch.float64, out=f64), 12 * px, px),
         ("sat i32 1R1W (same images)", lambda: libsat.sat_batched(i32, out=box), 8 * px, px),
-        (f"box filter u8 r={r} (SAT + 4 reads)", lambda: libsat.box_filter(u8, r, r, out=box), 13 * px, px),
+        (f"box filter u8 r={r} fused (1 B in x (1 + 2r/64) + 4 B out)", lambda: libsat.box_filter(u8, r, r, out=box),
+         int((1 + 2 * r / 64) * px) + 4 * px, px),
+        (f"box filter f32->f32 r={r} fused (float64 SAT on chip)", lambda: libsat.box_filter(f32, r, r, out=f32o),
+         int(4 * (1 + 2 * r / 32) * px) + 4 * px, px),
         ("rect sums (1M queries)", lambda: libsat.rect_sums(i32, rects, out=qout), None, 1 << 20),
     ]
     for name, fn, nbytes, units in cases:
