@@ -236,11 +236,11 @@ bool tma_ok(const void* in, const void* out, int64_t cols, int in_dtype = -1) {
 }
 
 int make_tmap(CUtensorMap* m, const void* base, int dtype, int64_t batch, int64_t rows,
-              int64_t cols, int th) {
+              int64_t cols, int th, int tw = TW) {
     cuuint64_t dims[3] = {cuuint64_t(cols), cuuint64_t(rows), cuuint64_t(batch)};
     const cuuint64_t eb = esize(dtype);
     cuuint64_t strides[2] = {cuuint64_t(cols) * eb, cuuint64_t(cols) * cuuint64_t(rows) * eb};
-    cuuint32_t box[3] = {cuuint32_t(TW), cuuint32_t(th), 1};
+    cuuint32_t box[3] = {cuuint32_t(tw), cuuint32_t(th), 1};
     cuuint32_t es[3] = {1, 1, 1};
     CUresult r = g_encode(m, dtype == SAT_INT32     ? CU_TENSOR_MAP_DATA_TYPE_UINT32
                              : dtype == SAT_FLOAT32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
@@ -286,6 +286,12 @@ constexpr BandCfg kCfgD32{4, 8, 4, 8, 1, 4, 1, 1};   // 192 KB smem, 512 TMEM co
 // columns per lane, 4 descriptor words per band, look-back window 4):
 // 16384^2 0.917 vs 1.04 ms with 3 groups of 1 warp, 32768^2 3.49 vs 3.87
 constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM cols
+// TH 128 (plain 1R1W): 64-column chunks, so a lane moves two doubles (16 B)
+// and a chunk is 64 KB -- the int32 TH-128 geometry: 16 compute warps, one CTA
+// per SM, 3 x 64 KB ring, 4 chunks parked (512 TMEM columns), 3 control
+// warps of 2 columns per lane (4 descriptor words per band, window 2)
+constexpr BandCfg kCfgD128{8, 16, 3, 4, 1, 3, 1, 1};
+constexpr int kTwD128 = 64;
 // uint8 input widened to uint32 sums: the ring holds bytes (TH x 128 B per
 // chunk), so it is 6 slots deep
 constexpr BandCfg kCfgU64{8, 8, 6, 4, 1, 4, 1, 2};
@@ -305,10 +311,10 @@ struct KernelSetup {
 };
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW = 0, typename TI = T>
+          int LBW = 0, typename TI = T, int TWK = TW>
 int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di, cudaStream_t st, int& grid_out) {
-    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI>;
-    const size_t smem = BandSmem<T, R, W, S, DT, SUB, TI>::total;
+    auto kern = sat_band_kernel<T, R, W, S, DT, SUB, NCW, NS, MODE, TMA, MINB, LBW, TI, TWK>;
+    const size_t smem = BandSmem<T, R, W, S, DT, SUB, TI, TWK>::total;
     const int threads = (W + NCW + 1) * 32;
     // per instantiation and device: attributes set once, resources queried
     // once (a per-call cudaFuncGetAttributes was a visible part of the ~15 us
@@ -336,7 +342,8 @@ int launch_band_t(const BandParams& p, const CUtensorMap& ti, const DevInfo& di,
     const int regs_warp = ((fa.numRegs * 32 + 255) / 256) * 256;
     const int occ = std::min({2048 / threads, 65536 / (regs_warp * warps),
                               di.smem_sm / int(smem + fa.sharedSizeBytes + 1024),
-                              MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT, int(sizeof(T) / 4)>::alloc, 32});
+                              MODE == MODE_ROW ? 32 : 512 / TmemCols<R, W, DT, int(sizeof(T) / 4), TWK / 32>::alloc,
+                              32});
     if (occ < 1) return fail(SAT_ERR_CUDA, "band kernel does not fit on an SM");
     long long grid = std::min<long long>(p.total_units, (long long)occ * di.sms);
     if (grid < 1) grid = 1;
@@ -376,7 +383,7 @@ int band_th(int mode, int dtype, bool tma, int th) {
         return 32;
     }
     if (mode != MODE_SAT) return th >= 64 ? 64 : 32;
-    if (dtype == SAT_FLOAT64) return th >= 64 ? 64 : th >= 32 ? 32 : 16;
+    if (dtype == SAT_FLOAT64) return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
     return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
 }
 
@@ -400,6 +407,8 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
         }
     } else if constexpr (sizeof(T) == 8) {
         switch (th) {
+            case 128: return launch_band_t<T, SAT_CFG(kCfgD128), MODE, TMA, kCfgD128.MINB, kLbw128, T, kTwD128>(
+                          p, ti, di, st, grid);
             case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, di, st, grid);
             case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
             case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
@@ -457,6 +466,9 @@ int launch_band_d(int mode, bool tma, int th, const BandParams& p, const CUtenso
 // raise parallelism, taller bands cut descriptor traffic).
 int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dtype) {
     if (dtype == SAT_FLOAT64) {
+        // plain 1R1W: TH 128 with 64-column chunks (the int32 TH-128 geometry)
+        // once its bands fill two thirds of the SMs
+        if (variant == SAT_1R1W && batch * ((rows + 127) / 128) * 100 >= 65LL * di.sms) return 128;
         // one CTA per SM for TH 32/64 (1-KB rows): the tallest band with a
         // wave; below that TH 32 from 1024 rows (a shorter look-back chain
         // beats filling the SMs: 1024^2 0.031 vs 0.034 ms, 2048^2 0.054 vs 0.063)
@@ -549,8 +561,11 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     p.rows = j.rows;
     p.cols = j.cols;
     p.batch = int(j.batch);
+    // chunk width: 64 columns for float64 at TH 128 (kCfgD128), else 128
+    const int tw = (mode == MODE_SAT && j.tma && j.dtype == SAT_FLOAT64 && j.in_dtype == j.dtype && j.th == 128)
+                       ? kTwD128 : TW;
     p.nb = int((j.rows + j.th - 1) / j.th);
-    p.nc = int((j.cols + TW - 1) / TW);
+    p.nc = int((j.cols + tw - 1) / tw);
     p.total_bands = int(j.batch * p.nb);
     p.total_units = p.tile_units ? (long long)p.total_bands * ((p.nc + p.tile_units - 1) / p.tile_units)
                                  : p.total_bands;
@@ -585,7 +600,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     }
     Workspace& ws = *j.ws;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
-        const size_t need = size_t(p.total_bands) * size_t(p.nc) * TW * sizeof(uint64_t) * (esize(j.dtype) / 4);
+        const size_t need = size_t(p.total_bands) * size_t(p.nc) * tw * sizeof(uint64_t) * (esize(j.dtype) / 4);
         SAT_TRY(ensure(ws.desc, need, true));
     }
     SAT_TRY(ensure(ws.ticket, 4 * sizeof(unsigned long long), true));
@@ -616,7 +631,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     CUtensorMap ti;
     std::memset(&ti, 0, sizeof(ti));
     if (j.tma) {
-        SAT_TRY(make_tmap(&ti, in, j.in_dtype, j.batch, j.rows, j.cols, j.th));
+        SAT_TRY(make_tmap(&ti, in, j.in_dtype, j.batch, j.rows, j.cols, j.th, tw));
     }
     int grid = 0;
     int s;
@@ -830,7 +845,9 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     j.di = &di;
     j.ws = ws;
     j.st = st;
-    // the 1R1W family's band height (2R1W Steps 1-2 size their carries by it)
+    // the 1R1W family's band height (2R1W Steps 1-2 size their carries by it);
+    // float64 TH 128 (64-column chunks) serves plain 1R1W only
+    if (dtype == SAT_FLOAT64 && variant != SAT_1R1W && j.th > 64) j.th = 64;
     j.th = eff_th(j, MODE_SAT);
     t_th = j.th;
     switch (variant) {

@@ -42,67 +42,80 @@
 
 namespace sat {
 
-template <typename T>
-struct V4 { T x, y, z, w; };
+// The EPL consecutive elements a lane owns in a chunk row (16 B for 4-byte
+// types at 128-column chunks and for float64 at 64-column chunks; 32 B for
+// float64 at 128 columns), moved as whole vectors.
+template <typename T, int N>
+struct Vec { T e[N]; };
 
-// 4 consecutive elements (16 B, or 32 B for float64) as vector accesses
-template <typename T>
-__device__ __forceinline__ void v4_words(const V4<T>& v, uint32_t (&w)[4 * Words<T>::N]) {
-    const T e[4] = {v.x, v.y, v.z, v.w};
-    pack<T, 4>(e, w);
+template <typename T, int N>
+__device__ __forceinline__ void vec_words(const Vec<T, N>& v, uint32_t (&w)[N * Words<T>::N]) {
+    pack<T, N>(v.e, w);
 }
-template <typename T>
-__device__ __forceinline__ V4<T> lds4(const T* p) {
-    uint32_t w[4 * Words<T>::N];
-    ld_words<4 * Words<T>::N>(p, w);
-    T e[4];
-    unpack<T, 4>(w, e);
-    return V4<T>{e[0], e[1], e[2], e[3]};
+template <typename T, int N>
+__device__ __forceinline__ Vec<T, N> ldsv(const T* p) {
+    uint32_t w[N * Words<T>::N];
+    ld_words<N * Words<T>::N>(p, w);
+    Vec<T, N> v;
+    unpack<T, N>(w, v.e);
+    return v;
 }
-template <typename T>
-__device__ __forceinline__ void sts4(T* p, const V4<T>& v) {
-    uint32_t w[4 * Words<T>::N];
-    v4_words(v, w);
-    st_words<4 * Words<T>::N>(p, w);
+template <typename T, int N>
+__device__ __forceinline__ void stsv(T* p, const Vec<T, N>& v) {
+    uint32_t w[N * Words<T>::N];
+    vec_words(v, w);
+    st_words<N * Words<T>::N>(p, w);
 }
 // streaming store (evict-first: the SAT is not re-read by this kernel)
-template <typename T>
-__device__ __forceinline__ void st_global_v4(T* p, const V4<T>& v) {
-    uint32_t w[4 * Words<T>::N];
-    v4_words(v, w);
-    stcs_words<4 * Words<T>::N>(p, w);
+template <typename T, int N>
+__device__ __forceinline__ void stgv(T* p, const Vec<T, N>& v) {
+    uint32_t w[N * Words<T>::N];
+    vec_words(v, w);
+    stcs_words<N * Words<T>::N>(p, w);
 }
-template <typename T>
-__device__ __forceinline__ void add4(V4<T>& a, const V4<T>& b) {
-    a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+template <typename T, int N>
+__device__ __forceinline__ void addv(Vec<T, N>& a, const Vec<T, N>& b) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) a.e[i] += b.e[i];
+}
+template <typename T, int N>
+__device__ __forceinline__ Vec<T, N> zerov() {
+    Vec<T, N> v;
+#pragma unroll
+    for (int i = 0; i < N; ++i) v.e[i] = T(0);
+    return v;
 }
 
-// Input element -> arithmetic element for 4 consecutive columns in shared
-// memory: the same type, or a narrower input widened on load (uint8 pixels ->
-// uint32 sums, the classic integral image; float32 -> float64 sums, an
-// accurate float integral image).  DESIGN.md Sec. 4.8.
-template <typename T, typename TI>
-__device__ __forceinline__ V4<T> lds4_in(const TI* p) {
+// Input element -> arithmetic element for the lane's N consecutive columns
+// in shared memory: the same type, or a narrower input widened on load (uint8
+// pixels -> uint32 sums, the classic integral image; float32 -> float64 sums,
+// an accurate float integral image).  DESIGN.md Sec. 4.8.
+template <typename T, typename TI, int N>
+__device__ __forceinline__ Vec<T, N> ldsv_in(const TI* p) {
     if constexpr (std::is_same<T, TI>::value) {
-        return lds4<T>(p);
+        return ldsv<T, N>(p);
     } else if constexpr (sizeof(TI) == 1) {
+        static_assert(N == 4, "uint8 input: 4 pixels per lane");
         const uint32_t w = *reinterpret_cast<const uint32_t*>(p);
-        return V4<T>{T(w & 255u), T((w >> 8) & 255u), T((w >> 16) & 255u), T(w >> 24)};
+        return Vec<T, N>{{T(w & 255u), T((w >> 8) & 255u), T((w >> 16) & 255u), T(w >> 24)}};
     } else {
-        const V4<TI> a = lds4<TI>(p);
-        return V4<T>{T(a.x), T(a.y), T(a.z), T(a.w)};
+        const Vec<TI, N> a = ldsv<TI, N>(p);
+        Vec<T, N> v;
+#pragma unroll
+        for (int i = 0; i < N; ++i) v.e[i] = T(a.e[i]);
+        return v;
     }
 }
 
 // Shared-memory footprint of one configuration.
-template <typename T, int R, int W, int S, int DT, int SUB, typename TI = T>
+template <typename T, int R, int W, int S, int DT, int SUB, typename TI = T, int TWK = TW>
 struct BandSmem {
     static constexpr int TH = R * W;
     static constexpr int XS = DT;                    // carry slots: one per parked chunk
-    static constexpr size_t tile_elems = size_t(TH) * TW;            // one 128-column chunk
+    static constexpr size_t tile_elems = size_t(TH) * TWK;           // one TWK-column chunk
     static constexpr size_t slot_elems = tile_elems * SUB;           // one ring slot
     static constexpr size_t tiles = S * slot_elems * sizeof(TI);     // the ring holds input elements
-    static constexpr size_t xbuf = size_t(XS) * W * TW * sizeof(T);
+    static constexpr size_t xbuf = size_t(XS) * W * TWK * sizeof(T);
     // + unit queue: ufull[2], uempty[2]
     static constexpr size_t nbars = 2 * S + 2 * XS + 4;
     // + s_unit[2], s_tmem, and per compute warp the (band, chunk) of each
@@ -155,17 +168,18 @@ __device__ __forceinline__ void publish_words(uint64_t* my, uint32_t tag, const 
     }
 }
 
-// Row-wise inclusive prefix-sums of R rows of 128 columns (lane owns 4
+// Row-wise inclusive prefix-sums of R rows of a chunk (lane owns N
 // consecutive columns), continuing from the running row sums L, which are
 // advanced to the end of the chunk.  Rows are interleaved step by step so the
 // shuffles of different rows overlap.
-template <typename T, int R>
-__device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
+template <typename T, int R, int N>
+__device__ __forceinline__ void row_scan(Vec<T, N> (&v)[R], T (&L)[R], int lane) {
     T inc[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        v[r].y += v[r].x; v[r].z += v[r].y; v[r].w += v[r].z;
-        inc[r] = v[r].w;
+#pragma unroll
+        for (int i = 1; i < N; ++i) v[r].e[i] += v[r].e[i - 1];
+        inc[r] = v[r].e[N - 1];
     }
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -179,13 +193,14 @@ __device__ __forceinline__ void row_scan(V4<T> (&v)[R], T (&L)[R], int lane) {
     for (int r = 0; r < R; ++r) {
         T exc;
         if constexpr (std::is_same<T, uint32_t>::value) {
-            exc = inc[r] - v[r].w;                 // exact in Z/2^32
+            exc = inc[r] - v[r].e[N - 1];          // exact in Z/2^32
         } else {
             exc = __shfl_up_sync(0xffffffffu, inc[r], 1);
             if (lane == 0) exc = T(0);
         }
         const T off = L[r] + exc;
-        v[r].x += off; v[r].y += off; v[r].z += off; v[r].w += off;
+#pragma unroll
+        for (int i = 0; i < N; ++i) v[r].e[i] += off;
         L[r] += __shfl_sync(0xffffffffu, inc[r], 31);
     }
 }
@@ -276,11 +291,11 @@ __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.
 __device__ __forceinline__ void tmem_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tmem_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// TMEM columns per CTA for W compute warps holding DT chunks of R x 4
+// TMEM columns per CTA for W compute warps holding DT chunks of R x EPL
 // elements of NWE 32-bit words each.
-template <int R, int W, int DT, int NWE = 1>
+template <int R, int W, int DT, int NWE = 1, int EPL = 4>
 struct TmemCols {
-    static constexpr int per_chunk = 4 * R * NWE;
+    static constexpr int per_chunk = EPL * R * NWE;
     static constexpr int per_warp = DT * per_chunk;
     static constexpr int need = per_warp * ((W + 3) / 4);       // warps w, w+4, .. share lanes
     static constexpr int alloc = need <= 32 ? 32 : need <= 64 ? 64 : need <= 128 ? 128
@@ -305,35 +320,37 @@ __device__ __forceinline__ void colseed_wait(const ColSeed& cs) {
         } while (v < cs.epoch);
     }
 }
-// sum_{q < n} vec_q[c .. c+3] in q order (columns >= cols read as 0); volatile
-// loads: the vectors may have been written over NVLink by another GPU
-template <typename T>
-__device__ __forceinline__ V4<T> colseed4(const ColSeed& cs, int64_t c, int64_t cols) {
-    T e[4] = {T(0), T(0), T(0), T(0)};
+// sum_{q < n} vec_q[c .. c+N-1] in q order (columns >= cols read as 0);
+// volatile loads: the vectors may have been written over NVLink by another GPU
+template <typename T, int N>
+__device__ __forceinline__ Vec<T, N> colseedv(const ColSeed& cs, int64_t c, int64_t cols) {
+    Vec<T, N> s = zerov<T, N>();
     for (int q = 0; q < cs.n; ++q) {
         const volatile T* v = reinterpret_cast<const volatile T*>(
             reinterpret_cast<const uint8_t*>(cs.base) + int64_t(q) * cs.stride);
 #pragma unroll
-        for (int i = 0; i < 4; ++i)
-            if (c + i < cols) e[i] += v[c + i];
+        for (int i = 0; i < N; ++i)
+            if (c + i < cols) s.e[i] += v[c + i];
     }
-    return V4<T>{e[0], e[1], e[2], e[3]};
+    return s;
 }
 
 template <typename T, int R, int W, int S, int DT, int SUB, int NCW, int NS, int MODE, bool TMA, int MINB,
-          int LBW_ = 0, typename TI = T>
+          int LBW_ = 0, typename TI = T, int TWK = TW>
 __global__ void __launch_bounds__((W + NCW + 1) * 32, MINB)
 sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 const BandParams p)
 {
     constexpr int TH = R * W;
+    constexpr int EPL = TWK / 32;  // elements per lane in a chunk row
+    static_assert(TWK % 32 == 0 && EPL * sizeof(T) >= 16, "a lane moves at least 16 B per chunk row");
     constexpr int CW = W;          // first control warp
     constexpr int PW = W + NCW;    // producer warp
-    constexpr uint32_t TILE_BYTES = uint32_t(TH) * TW * sizeof(TI);
-    using SM = BandSmem<T, R, W, S, DT, SUB, TI>;
+    constexpr uint32_t TILE_BYTES = uint32_t(TH) * TWK * sizeof(TI);
+    using SM = BandSmem<T, R, W, S, DT, SUB, TI, TWK>;
     static_assert(std::is_same<T, TI>::value || MODE == MODE_SAT, "widening input: 1R1W only");
     constexpr int NWE = Words<T>::N;             // 32-bit words per element
-    using TC = TmemCols<R, W, DT, NWE>;
+    using TC = TmemCols<R, W, DT, NWE, EPL>;
     constexpr int XS = SM::XS;
     constexpr bool HOLD = (MODE != MODE_ROW);    // chunks wait for a vertical carry
     // A control warp waits on colr[] of chunk k only after finishing chunk
@@ -398,7 +415,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
     const unsigned long long kbase = p.base_dev ? __ldcg(p.base_dev) : p.base;
 
     const int64_t img_elems = p.rows * p.cols;
-    const int desc_w = p.nc * TW;
+    const int desc_w = p.nc * TWK;
     const int64_t lx_stride = int64_t(p.total_bands) * TH;
     uint32_t g = 0;                              // CTA-local chunk counter (carry / TMEM slots)
     uint32_t gq = 0;                             // CTA-local ring-slot counter (SUB chunks per slot)
@@ -424,26 +441,26 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             if (p.trace != nullptr && warp == 0 && lane == 0)
                 p.trace[(int64_t(fgb) * p.nc + fJ) * 8 + 6] = globaltimer();
         }
-        const V4<T> add = lds4<T>(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane);
+        const Vec<T, EPL> add = ldsv<T, EPL>(xbuf + (size_t(it % XS) * W + warp) * TWK + EPL * lane);
         uint32_t u[TC::per_chunk];
         tmem_wait_st();
         tmem_ld<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
         tmem_wait_ld();
-        const int64_t c = int64_t(fJ) * TW + 4 * lane;
+        const int64_t c = int64_t(fJ) * TWK + EPL * lane;
 #pragma unroll
         for (int r = 0; r < R; ++r) {
-            const uint32_t* q = u + 4 * r * NWE;
-            V4<T> v{from_words<T>(q), from_words<T>(q + NWE), from_words<T>(q + 2 * NWE), from_words<T>(q + 3 * NWE)};
-            add4(v, add);
+            Vec<T, EPL> v;
+#pragma unroll
+            for (int i = 0; i < EPL; ++i) v.e[i] = from_words<T>(u + (EPL * r + i) * NWE);
+            addv(v, add);
             const int64_t row = frow0 + rbase + r;
             if (row < p.rows) {
                 if constexpr (TMA) {
-                    if (c < p.cols) st_global_v4(fout + row * p.cols + c, v);
+                    if (c < p.cols) stgv(fout + row * p.cols + c, v);
                 } else {
-                    const T e[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                    for (int i = 0; i < 4; ++i)
-                        if (c + i < p.cols) fout[row * p.cols + c + i] = e[i];
+                    for (int i = 0; i < EPL; ++i)
+                        if (c + i < p.cols) fout[row * p.cols + c + i] = v.e[i];
                 }
             }
         }
@@ -547,19 +564,18 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 
             // store R rows of 4 values to the output (16-B vectors on the TMA
             // path, where cols % 4 == 0; guarded scalars otherwise)
-            auto store_rows = [&](const V4<T> (&v)[R], int k) {
-                const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
+            auto store_rows = [&](const Vec<T, EPL> (&v)[R], int k) {
+                const int64_t c = int64_t(j0 + k) * TWK + EPL * lane;
 #pragma unroll
                 for (int r = 0; r < R; ++r) {
                     const int64_t row = row0 + rbase + r;
                     if (row < p.rows) {
                         if constexpr (TMA) {
-                            if (c < p.cols) st_global_v4(gout + row * p.cols + c, v[r]);
+                            if (c < p.cols) stgv(gout + row * p.cols + c, v[r]);
                         } else {
-                            const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
 #pragma unroll
-                            for (int i = 0; i < 4; ++i)
-                                if (c + i < p.cols) gout[row * p.cols + c + i] = e[i];
+                            for (int i = 0; i < EPL; ++i)
+                                if (c + i < p.cols) gout[row * p.cols + c + i] = v[r].e[i];
                         }
                     }
                 }
@@ -569,9 +585,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             // park the result in TMEM, warp bottom row into xbuf
             auto local = [&](int k) {
                 const uint32_t it = g + k;
-                V4<T> v[R];
-                V4<T> sd;
-                if (seeded) sd = colseed4<T>(p.cseed, int64_t(j0 + k) * TW + 4 * lane, p.cols);
+                Vec<T, EPL> v[R];
+                Vec<T, EPL> sd;
+                if (seeded) sd = colseedv<T, EPL>(p.cseed, int64_t(j0 + k) * TWK + EPL * lane, p.cols);
                 if constexpr (TMA) {
                     const uint32_t q = gq + uint32_t(k / SUB);     // ring slot of chunk k
                     const int s = q % S;
@@ -582,9 +598,9 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     }
                     {
                         const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems
-                                      + size_t(rbase) * TW + 4 * lane;
+                                      + size_t(rbase) * TWK + EPL * lane;
 #pragma unroll
-                        for (int r = 0; r < R; ++r) v[r] = lds4_in<T, TI>(t + r * TW);
+                        for (int r = 0; r < R; ++r) v[r] = ldsv_in<T, TI, EPL>(t + r * TWK);
                     }
                     if (k % SUB == SUB - 1 || k == nch - 1) {
                         // release the slot to the next TMA write only once the
@@ -594,42 +610,38 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         // (seen as corrupted rows with 4 compute warps)
 #pragma unroll
                         for (int r = 0; r < R; ++r) {
-                            uint32_t w[4 * NWE];
-                            v4_words(v[r], w);
+                            uint32_t w[EPL * NWE];
+                            vec_words(v[r], w);
 #pragma unroll
-                            for (int k = 0; k < 4 * NWE; ++k) asm volatile("" :: "r"(w[k]));
+                            for (int k = 0; k < EPL * NWE; ++k) asm volatile("" :: "r"(w[k]));
                         }
                         fence_proxy_async_smem();
                         mbar_arrive(&empty[s]);
                     }
                 } else {
-                    const int64_t c = int64_t(j0 + k) * TW + 4 * lane;
+                    const int64_t c = int64_t(j0 + k) * TWK + EPL * lane;
 #pragma unroll
                     for (int r = 0; r < R; ++r) {
                         const int64_t row = row0 + rbase + r;
-                        T e[4];
 #pragma unroll
-                        for (int i = 0; i < 4; ++i)
-                            e[i] = (row < p.rows && c + i < p.cols) ? T(gin[row * p.cols + c + i]) : T(0);
-                        v[r] = V4<T>{e[0], e[1], e[2], e[3]};
+                        for (int i = 0; i < EPL; ++i)
+                            v[r].e[i] = (row < p.rows && c + i < p.cols) ? T(gin[row * p.cols + c + i]) : T(0);
                     }
                 }
-                if (seeded) add4(v[0], sd);
-                if constexpr (MODE != MODE_COL) row_scan<T, R>(v, L, lane);
+                if (seeded) addv(v[0], sd);
+                if constexpr (MODE != MODE_COL) row_scan<T, R, EPL>(v, L, lane);
                 if constexpr (!HOLD) {
                     store_rows(v, k);                    // the row pass is final
                 } else {
 #pragma unroll
-                    for (int r = 1; r < R; ++r) add4(v[r], v[r - 1]);
+                    for (int r = 1; r < R; ++r) addv(v[r], v[r - 1]);
                     uint32_t u[TC::per_chunk];
 #pragma unroll
-                    for (int r = 0; r < R; ++r) {
-                        const T e[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+                    for (int r = 0; r < R; ++r)
 #pragma unroll
-                        for (int i = 0; i < 4; ++i) to_words<T>(e[i], u + (4 * r + i) * NWE);
-                    }
+                        for (int i = 0; i < EPL; ++i) to_words<T>(v[r].e[i], u + (EPL * r + i) * NWE);
                     tmem_st<TC::per_chunk>(tm_warp + uint32_t((it % DT) * TC::per_chunk), u);
-                    sts4(xbuf + (size_t(it % XS) * W + warp) * TW + 4 * lane, v[R - 1]);
+                    stsv(xbuf + (size_t(it % XS) * W + warp) * TWK + EPL * lane, v[R - 1]);
                     if (lane == 0) wmeta[it % DT] = make_int2(gb, j0 + k);
                     mbar_arrive(&colr[it % XS]);
                 }
@@ -684,13 +696,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             // lane), so one round trip reads LBW = 16/CPL bands' words in the
             // same 32 registers per lane.
             if constexpr (HOLD) {
-                constexpr int CPL = 4 / NS;
+                constexpr int CPL = EPL / NS;
                 constexpr int G = NCW / NS;
                 constexpr int NW = CPL * NWE;                  // descriptor words per band
                 constexpr int LBW = LBW_ > 0 ? LBW_ : (16 / NW > 0 ? 16 / NW : 1);   // bands per round trip
                 const int cw = warp - CW;
                 const int grp = cw / NS;
-                const int cl = (cw % NS) * (TW / NS) + lane * CPL;   // column within the chunk
+                const int cl = (cw % NS) * (TWK / NS) + lane * CPL;  // column within the chunk
                 const uint32_t tagbase = band_tag(kbase, gb);
                 const bool lookback = (p.top_src == TOP_LOOKBACK);
                 const bool publish = lookback && band + 1 < p.nb;   // the last band is never read
@@ -703,8 +715,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                 for (int k = int((uint32_t(grp) + uint32_t(G) - g % uint32_t(G)) % uint32_t(G)); k < nch; k += G) {
                     const uint32_t it = g + k;
                     const int J = j0 + k;
-                    const int c0 = J * TW + cl;
-                    T* xb = xbuf + size_t(it % XS) * W * TW + cl;
+                    const int c0 = J * TWK + cl;
+                    T* xb = xbuf + size_t(it % XS) * W * TWK + cl;
                     mbar_wait(&colr[it % XS], (it / XS) & 1);
                     if constexpr (kDebug) {
                         if (traced && cw == grp * NS && lane == 0)
@@ -715,7 +727,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                     for (int w2 = 1; w2 < W; ++w2) {
                         T b[CPL];
-                        lds_cols<T, CPL>(xb + w2 * TW, b);
+                        lds_cols<T, CPL>(xb + w2 * TWK, b);
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) agg[i] += b[i];
                     }
@@ -820,8 +832,8 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
 #pragma unroll
                     for (int w2 = 0; w2 < W; ++w2) {
                         T b[CPL];
-                        lds_cols<T, CPL>(xb + w2 * TW, b);
-                        sts_cols<T, CPL>(xb + w2 * TW, top);
+                        lds_cols<T, CPL>(xb + w2 * TWK, b);
+                        sts_cols<T, CPL>(xb + w2 * TWK, top);
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) top[i] += b[i];
                     }
@@ -845,7 +857,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                         mbar_arrive_expect_tx(&full[s], TILE_BYTES * nsub);
                         for (int j = 0; j < nsub; ++j)   // adjacent boxes: SUB*512 B per row
                             tma_load_3d(tiles + size_t(s) * SM::slot_elems + size_t(j) * SM::tile_elems,
-                                        &tm_in, &full[s], (j0 + k0 + j) * TW, row0, img, pol);
+                                        &tm_in, &full[s], (j0 + k0 + j) * TWK, row0, img, pol);
                     }
                 }
             }

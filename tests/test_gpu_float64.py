@@ -76,14 +76,14 @@ def test_shapes_float64(libsat, variant, shape):
     within_order_bound(libsat.sat(dev(a53), variant=variant), oracle.sat(a53), variant)
 
 
-@pytest.mark.parametrize("tile_rows", [16, 32, 64])
+@pytest.mark.parametrize("tile_rows", [16, 32, 64, 128])
 @pytest.mark.parametrize("generic", [False, True])
 @pytest.mark.parametrize("variant", ["1r1w", "2r2w", "2r1w", "1+rr1w"])
 def test_tile_configs_float64(libsat, tile_rows, generic, variant):
     a = make_np(700, 1300, "float64", "unit", seed=tile_rows)
     exact(libsat.sat(dev(a), variant=variant, tile_rows=tile_rows, force_generic=generic),
           oracle.sat(a))
-    if variant in ("1r1w", "2r1w", "1+rr1w") and not generic:
+    if not generic and (variant == "1r1w" or (variant in ("2r1w", "1+rr1w") and tile_rows <= 64)):
         assert libsat.last_tile_rows() == tile_rows
 
 
@@ -152,3 +152,24 @@ def test_float64_16k_full(libsat):
     st = oracle.Stream(n, False)
     for r0 in range(0, n, 1024):
         exact(y[r0:r0 + 1024], st.feed(a[r0:r0 + 1024]))
+
+
+@pytest.mark.parametrize("shape", [(1000, 1100), (128 * 100 + 7, 700), (300, 64 * 33 + 4), (129, 4)],
+                         ids=lambda s: f"{s[0]}x{s[1]}")
+def test_float64_th128_narrow_chunks(libsat, shape):
+    """float64 at TH 128 runs 64-column chunks (two doubles per lane, the int32
+    TH-128 geometry): partial last chunks, many bands, segments, seeds, jitter."""
+    a = make_np(*shape, "float64", "unit", seed=shape[0] % 97)
+    ref = oracle.sat(a)
+    x = dev(a)
+    exact(libsat.sat(x, tile_rows=128), ref)
+    assert libsat.last_tile_rows() == 128
+    exact(libsat.sat(x, tile_rows=128, segments=3), ref)
+    exact(libsat.sat(x, tile_rows=128, jitter=20000), ref)
+    if shape[0] > 300:
+        r0 = 257
+        exact(libsat.sat_seeded(dev(a[r0:]), carry_row=dev(oracle.column_totals(a[:r0]))), ref[r0:])
+    b = make_np(*shape, "float64", "unit", seed=3, batch=2)
+    got = libsat.sat_batched(dev(b), tile_rows=128).cpu().numpy()
+    for i in range(2):
+        exact(got[i], oracle.sat(b[i]))
