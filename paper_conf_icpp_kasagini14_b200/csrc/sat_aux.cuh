@@ -161,7 +161,16 @@ __global__ void sat_carry_rows_kernel(const CarryParams p)
             const int J = J0 + lane;
             const T tot = (J < j1) ? bt[int64_t(J) * TW + TW - 1] : T(0);
             const T inc = warp_inclusive_scan(tot, lane);
-            if (J <= jend) lsum[J] = base + inc - tot;
+            // exclusive prefix: by subtraction only in Z/2^32; floats shift
+            // (inc - tot would turn an Inf total into NaN)
+            T exc;
+            if constexpr (std::is_same<T, uint32_t>::value) {
+                exc = inc - tot;
+            } else {
+                exc = __shfl_up_sync(0xffffffffu, inc, 1);
+                if (lane == 0) exc = T(0);
+            }
+            if (J <= jend) lsum[J] = base + exc;
             base += __shfl_sync(0xffffffffu, inc, 31);
         }
     }

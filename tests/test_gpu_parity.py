@@ -343,6 +343,46 @@ def test_cfg4_65536_properties(libsat):
         with np.errstate(over="ignore"):
             rec = w[1, 1] - w[0, 1] - w[1, 0] + w[0, 0]
         assert rec == np.uint32(int(x[i, j]) & 0xFFFFFFFF)
+    # the LAST 2048 rows, whole, against the oracle streamed from the column
+    # sums of every row above them: these rows are the end of the longest
+    # vertical carry chain (511 bands, 16 segments), which the 2x2 windows
+    # above cannot see (they cancel any per-band carry error).  The column
+    # sums come from torch (int64 accumulation of the input rows, independent
+    # of libsat); the SAT rows from the oracle.
+    r0 = n - 2048
+    acc = torch.zeros(n, dtype=torch.int64, device="cuda")
+    for a in range(0, r0, 4096):
+        acc += x[a:min(r0, a + 4096)].to(torch.int64).sum(dim=0)
+    st = oracle.Stream(n, True)
+    st.colsum[:] = (acc % 2**32).cpu().numpy().astype(np.uint32)
+    for a in range(r0, n, 512):
+        ref = st.feed(x[a:a + 512].cpu().numpy())
+        got = y[a:a + 512].cpu().numpy()
+        assert np.array_equal(got, ref), f"rows {a}..{a + 511}"
+
+
+def test_float_nan_inf_propagate(libsat):
+    """IEEE semantics: a NaN poisons every SAT element at or
+    below-right of it, +Inf likewise (no FTZ / fast-math), for every variant;
+    elements above or left of it stay finite and exact."""
+    for dtype in ("float32", "float64"):
+        a = make_np(600, 700, dtype, "unit", seed=1)
+        a[300, 400] = np.nan
+        a[100, 650] = np.inf
+        for variant in VARIANTS:
+            got = libsat.sat(dev(a), variant=variant).cpu().numpy()
+            assert np.isnan(got[300:, 400:]).all(), variant
+            assert np.isinf(got[100:300, 650:]).all() and (got[100:300, 650:] > 0).all(), variant
+            clean = a.copy()
+            clean[300, 400] = 0
+            clean[100, 650] = 0
+            ref = oracle.sat(clean)
+            ok = np.isfinite(got)
+            assert ok[:100].all() and ok[:300, :400].all()
+            if dtype == "float64":
+                assert np.array_equal(got[:300, :400], ref[:300, :400]), variant
+            else:
+                assert oracle.max_rel_err(got[:300, :400], ref[:300, :400]) <= FTOL, variant
 
 
 def test_debug_trace_records_events(libsat):
