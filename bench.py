@@ -221,6 +221,17 @@ def run_reference(args, cfg_key):
 
 
 # ------------------------------------------------------------------ our arm
+def _coll(fn, t, *a, **k):
+    """A small collective on a CUDA tensor; through host memory when the
+    process group is gloo (multi-process tests sharing one GPU)."""
+    import torch.distributed as dist
+    if dist.get_backend() == "gloo" and t.is_cuda:
+        h = t.cpu()
+        fn(h, *a, **k)
+        t.copy_(h)
+    else:
+        fn(t, *a, **k)
+
 def strip_parity(x, y, dtype, r0, rows_above_gen, check_rows=256):
     """Parity of this rank's strip (first ``check_rows`` rows) against the CPU
     oracle streamed from the column sums of every row above the strip.  Those
@@ -264,6 +275,8 @@ def main():
                     help="write a 2 x L2 buffer between timed steps (auto: when the working set < 4 x L2)")
     ap.add_argument("--last-weight", type=float, default=1.5,
                     help="N>1 row strips: the last rank's share (it skips the totals pass)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="N>1 process group (gloo: host-memory exchange, for multi-process tests on one GPU)")
     ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
                     help="N>1 row strips: NCCL all-gather, or the fused peer exchange (IPC mailboxes)")
     args = ap.parse_args()
@@ -290,10 +303,16 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}")
-    torch.cuda.set_device(local)
+    # --dist-backend gloo lets the N>1 path run as several processes sharing
+    # fewer GPUs (tests on a one-GPU box); the driver's runs use NCCL
+    gpu = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(gpu)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
+        else:
+            dist.init_process_group("gloo")
+    dev = torch.device("cuda", gpu)
     stream = torch.cuda.current_stream()
     tdt = torch.int32 if dtype == "int32" else torch.float32
     dist_name = "u32" if dtype == "int32" else "unit"
@@ -338,7 +357,7 @@ def main():
             launches[0] += libsat.last_launch_count()
     elif sharded:
         from paper_conf_icpp_kasagini14_b200.dist import RowStripSAT
-        op = RowStripSAT(cols, tdt, device=dev)
+        op = RowStripSAT(cols, tdt, device=dev, host_exchange=args.dist_backend != "nccl")
         breakdown = {"totals_ms": [], "gather_ms": [], "sat_ms": []}
         step_events = []
 
@@ -399,7 +418,7 @@ def main():
                           lambda a, b: make_torch(b - a, cols, dtype, dist_name, seed=4001, row0=a,
                                                   device=dev))
         t = torch.tensor([0 if ok else 1], device=dev)
-        dist.all_reduce(t)
+        _coll(dist.all_reduce, t)
         parity = {"ranks_checked": world, "rows_per_rank": 256, "ok": int(t.item()) == 0}
 
     # ---------------- timed region
@@ -422,7 +441,7 @@ def main():
         kern_ms = [a.elapsed_time(b) for a, b in kev]
         return ev0.elapsed_time(ev1), kern_ms
 
-    with ClockSampler(local) as clk:
+    with ClockSampler(gpu) as clk:
         time.sleep(0.3)                     # let the sampler start
         ms_local, kern_ms = timed(flush)
     clocks = clk.summary()
@@ -442,7 +461,7 @@ def main():
                 breakdown["sat_ms"].append(e["totals"].elapsed_time(e["sat"]))
     t = torch.tensor([ms_local, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        _coll(dist.all_reduce, t, op=dist.ReduceOp.MAX)
     ms_total, kern_avg_ms = float(t[0]), float(t[1])
     ms_per_step = ms_total / args.steps
     value = total_elems * args.steps / (ms_total / 1e3)
@@ -468,7 +487,7 @@ def main():
         alg_bytes = 5 * eb * my_elems
     mine = torch.tensor([alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(mine, op=dist.ReduceOp.MIN)    # the slowest rank's band kernel
+        _coll(dist.all_reduce, mine, op=dist.ReduceOp.MIN)    # the slowest rank's band kernel
     achieved = float(mine[0])
     traffic = ncu_traffic(f"{cfg_key}:{variant}:n{world}")
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
@@ -506,8 +525,10 @@ def main():
         vals = torch.tensor([statistics.mean(breakdown["totals_ms"]),
                              statistics.mean(breakdown["gather_ms"]) if breakdown["gather_ms"] else 0.0,
                              statistics.mean(breakdown["sat_ms"])], dtype=torch.float64, device=dev)
-        allv = [torch.zeros_like(vals) for _ in range(world)]
-        dist.all_gather(allv, vals)
+        src = vals.cpu() if args.dist_backend == "gloo" else vals
+        allv = [torch.zeros_like(src) for _ in range(world)]
+        dist.all_gather(allv, src)
+        allv = [a.cpu() for a in allv]
         bd = {"per_rank_ms": [[round(float(v), 4) for v in a.tolist()] for a in allv],
               "columns": ["totals (extra read)", "all-gather wait", "seeded SAT (band kernel)"],
               "rows": [list(partition_rows(rows, world, p, args.last_weight)) for p in range(world)]}
@@ -593,7 +614,7 @@ def run_e2e(args, libsat, x, rows, cols, batch, dtype, world, rank, dev, sharded
     barrier()
     ms = torch.tensor([ev0.elapsed_time(ev1)], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+        _coll(dist.all_reduce, ms, op=dist.ReduceOp.MAX)
     ms = float(ms[0])
     return {"value": total_elems * steps / (ms / 1e3), "unit": "elem/s",
             "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes, "steps": steps,

@@ -60,10 +60,14 @@ class RowStripSAT:
     """This rank's end of the row-strip sharded SAT, with its exchange
     buffers allocated once (``send``: cols, ``gathered``: P x cols)."""
 
-    def __init__(self, cols: int, dtype, device=None, group=None, ops=None, host_exchange: bool = False):
+    def __init__(self, cols: int, dtype, device=None, group=None, ops=None, host_exchange=None):
         """``host_exchange``: all-gather through host memory (gloo process
-        groups, e.g. several processes sharing one GPU in tests)."""
+        groups, e.g. several processes sharing one GPU in tests); default:
+        when the group is gloo and the buffers live on a GPU."""
         self.group = group
+        on_gpu = device is not None and torch.device(device).type == "cuda"
+        if host_exchange is None:
+            host_exchange = on_gpu and dist.get_backend(group) == "gloo"
         self.host_exchange = host_exchange
         self.rank = dist.get_rank(group)
         self.P = dist.get_world_size(group)

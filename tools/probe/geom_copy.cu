@@ -50,7 +50,7 @@ template <int N>
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
 
 // MODE 0: consumers LDS + STG.cs; MODE 1: producer TMA-stores each landed slot (pure DMA)
-template <int H, int C, int S, int W, int MODE>
+template <int H, int C, int S, int W, int MODE, bool STRIP = false>
 __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant__ CUtensorMap tin,
                                                           const __grid_constant__ CUtensorMap tout, uint32_t* out,
                                                           int n, int U, unsigned long long* ticket, int units) {
@@ -75,7 +75,12 @@ __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant_
         const int unit = *s_unit;
         __syncthreads();
         if (unit >= units) break;
-        const int band = unit / upr, k0 = (unit % upr) * U;
+        // band-major: unit = (band, chunk range), chunk k at (cols (k0+k)*C, rows band*H)
+        // strip-major: unit = (row segment, strip), chunk k at (cols strip*C, rows (k0+k)*H)
+        const int spr = n / (H * U);            // row segments per strip (STRIP)
+        const int band = STRIP ? 0 : unit / upr, k0 = STRIP ? (unit / (n / C)) * U : (unit % upr) * U;
+        const int strip = STRIP ? unit % (n / C) : 0;
+        (void)spr;
         if (warp == W) {
             if (lane == 0 && MODE == 0) {
                 for (int k = 0; k < U; ++k) {
@@ -84,7 +89,8 @@ __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant_
                     if (it >= S) mbar_wait(&empty[s], ((it / S) & 1) ^ 1);
                     mbar_expect(&full[s], TILE * 4);
                     for (int b = 0; b < C / 128; ++b)
-                        tma_ld(tiles + size_t(s) * TILE + b * 128 * H, &tin, &full[s], (k0 + k) * C + b * 128, band * H,
+                        tma_ld(tiles + size_t(s) * TILE + b * 128 * H, &tin, &full[s],
+                               STRIP ? strip * C + b * 128 : (k0 + k) * C + b * 128, STRIP ? (k0 + k) * H : band * H,
                                pol);
                 }
             } else if (lane == 0) {
@@ -128,7 +134,10 @@ __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant_
                 for (int i = 0; i < V; ++i) {
                     const int q = (i * W + warp) * 32 + lane;
                     const int b = q / (32 * H), rem = q % (32 * H), r = rem / 32, c4 = rem % 32;
-                    __stcs((uint4*)(out + size_t(band * H + r) * n + (k0 + k) * C + b * 128 + c4 * 4), v[i]);
+                    if (STRIP)
+                        __stcs((uint4*)(out + size_t((k0 + k) * H + r) * n + strip * C + b * 128 + c4 * 4), v[i]);
+                    else
+                        __stcs((uint4*)(out + size_t(band * H + r) * n + (k0 + k) * C + b * 128 + c4 * 4), v[i]);
                 }
             }
         }
@@ -183,7 +192,7 @@ struct Ctx {
     unsigned long long* ticket;
 };
 
-template <int H, int C, int S, int W, int MODE>
+template <int H, int C, int S, int W, int MODE, bool STRIP = false>
 void run(int n, uint32_t* in, uint32_t* out, int U, int occ_force, const char* tag) {
     Ctx c;
     c.n = n; c.in = in; c.out = out; c.U = U;
@@ -195,7 +204,7 @@ void run(int n, uint32_t* in, uint32_t* out, int U, int occ_force, const char* t
         CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     c.smem = int(size_t(S) * H * C * 4 + 2 * S * 8 + 16);
     c.threads = (W + 1) * 32;
-    auto k = band_copy<H, C, S, W, MODE>;
+    auto k = band_copy<H, C, S, W, MODE, STRIP>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, c.smem);
     int occ = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, c.threads, c.smem);
@@ -206,7 +215,7 @@ void run(int n, uint32_t* in, uint32_t* out, int U, int occ_force, const char* t
     auto launch = [](void* p) {
         Ctx& c = *(Ctx*)p;
         cudaMemsetAsync(c.ticket, 0, 8);
-        band_copy<H, C, S, W, MODE><<<c.grid, c.threads, c.smem>>>(c.ti, c.to, c.out, c.n, c.U, c.ticket, c.units);
+        band_copy<H, C, S, W, MODE, STRIP><<<c.grid, c.threads, c.smem>>>(c.ti, c.to, c.out, c.n, c.U, c.ticket, c.units);
     };
     float avg, best = timed(launch, &c, 10, &avg);
     cudaError_t e = cudaGetLastError();
@@ -237,23 +246,13 @@ int main(int argc, char** argv) {
                2.0 * n * n * 4 / best / 1e6, avg, 2.0 * n * n * 4 / avg / 1e6);
     }
     const int nc = n / 128;
-    // the band kernel's geometry: 128 x 128 chunks, whole bands, 3-slot ring, 16 consumers
+    const int nr = n / 128;   // 128-row chunks per strip
     run<128, 128, 3, 16, 0>(n, in, out, nc, 1, "band128");
-    run<128, 128, 3, 16, 1>(n, in, out, nc, 1, "band128");
-    run<128, 128, 3, 16, 0>(n, in, out, nc / 2, 1, "band128h");
-    run<128, 128, 3, 16, 0>(n, in, out, nc / 8, 1, "band128s8");
-    run<128, 128, 3, 16, 1>(n, in, out, nc / 8, 1, "band128s8");
-    run<64, 128, 3, 8, 0>(n, in, out, nc, 2, "band64");
-    run<64, 128, 6, 8, 0>(n, in, out, nc, 1, "band64r6");
-    run<64, 256, 3, 8, 0>(n, in, out, nc / 2, 1, "band64w");
-    run<64, 256, 3, 8, 1>(n, in, out, nc / 2, 1, "band64w");
-    run<64, 256, 3, 8, 0>(n, in, out, nc / 16, 1, "band64ws");
-    run<32, 256, 3, 8, 0>(n, in, out, nc / 2, 2, "band32w");
-    run<32, 512, 3, 8, 0>(n, in, out, nc / 4, 1, "band32ww");
-    run<32, 512, 3, 8, 1>(n, in, out, nc / 4, 1, "band32ww");
-    run<16, 1024, 3, 8, 0>(n, in, out, nc / 8, 1, "band16");
-    run<16, 1024, 3, 8, 1>(n, in, out, nc / 8, 1, "band16");
-    run<128, 128, 3, 16, 1>(n, in, out, nc / 32, 1, "band128s32");
+    run<128, 128, 3, 16, 0, true>(n, in, out, nr, 1, "strip128");
+    run<128, 128, 3, 16, 0, true>(n, in, out, nr / 4, 1, "strip128s4");
+    run<128, 128, 3, 16, 0, true>(n, in, out, nr / 16, 1, "strip128s16");
+    run<64, 128, 3, 8, 0, true>(n, in, out, n / 64, 2, "strip64");
+    run<128, 128, 3, 16, 1, true>(n, in, out, nr, 1, "strip128dma");
     run<64, 128, 4, 4, 1>(n, in, out, nc / 16, 2, "band64d");
     return 0;
 }
