@@ -881,9 +881,15 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             t_r = r_eff;
             if (tA == 0) {
                 // r_eff = 0: both triangles are empty -- plain 1R1W (no empty
-                // Step 1/2 launches, band segments allowed)
+                // Step 1/2 launches, band segments allowed, plain 1R1W's band
+                // height: float64 may take TH 128)
+                Job j1 = j;
+                if (!o.tile_rows && dtype == SAT_FLOAT64) {
+                    j1.th = auto_th(rows, batch, di, SAT_1R1W, dtype);
+                    j1.th = eff_th(j1, MODE_SAT);
+                }
                 BandParams p = base_params();
-                return run_band(j, MODE_SAT, in, out, p);
+                return run_band(j1, MODE_SAT, in, out, p);
             }
             // (A) 2R1W on the top-left triangle; its Step 2 also leaves the
             // row carry into (C) in Lx.
