@@ -594,7 +594,13 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     if (k % SUB == 0) mbar_wait(&full[s], (q / S) & 1);
                     if constexpr (kDebug) {
                         if (traced && warp == 0 && lane == 0)
+                        {
                             p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 0] = globaltimer();
+                            uint32_t smid, nsm;
+                            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+                            asm volatile("mov.u32 %0, %%nsmid;" : "=r"(nsm));
+                            p.trace[(int64_t(gb) * p.nc + j0 + k) * 8 + 7] = (uint64_t(blockIdx.x) << 32) | smid;
+                        }
                     }
                     {
                         const TI* t = tiles + size_t(s) * SM::slot_elems + size_t(k % SUB) * SM::tile_elems

@@ -239,3 +239,14 @@ def test_box_fused_matches_two_pass(libsat):
     big = libsat.box_filter(x, 40, 3).cpu().numpy()
     assert libsat.last_launch_count() >= 2
     assert np.array_equal(big, oracle.box_filter(a, 40, 3))
+
+
+def test_box_huge_radius_clamped(libsat):
+    """a radius of INT_MAX ('the whole image') is clamped on the
+    host; every window covers the whole image, so every output is the image
+    total (mod 2^32)."""
+    a = u8img(300, 500, seed=12, batch=2)
+    y = libsat.box_filter(dev(a), 2**31 - 1, 2**31 - 1).cpu().numpy()
+    for b in range(2):
+        assert (y[b] == np.int64(a[b].astype(np.int64).sum()).astype(np.int32)).all()
+        assert np.array_equal(y[b], oracle.box_filter(a[b].astype(np.int32), 300, 500))

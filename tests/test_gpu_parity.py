@@ -683,3 +683,39 @@ def test_capture_host_call_refused(libsat):
     torch.cuda.synchronize()
     libsat.sat_host(a, o)
     assert np.array_equal(o.numpy(), oracle.sat(a.numpy()))
+
+
+def test_graph_replay_after_workspace_growth(libsat):
+    """capture a small call, grow the stream's workspace
+    with a larger eager call, replay the graph: the graph's buffers were
+    retired (not freed), so the replay is still correct and writes nothing
+    into memory the caller allocated afterwards; sat_release_workspace then
+    frees everything and the stream starts over."""
+    s = torch.cuda.Stream()
+    a = gen(640, 1280, "int32", seed=61)
+    x = dev(a)
+    with torch.cuda.stream(s):
+        y = libsat.sat(x)                    # sizes the workspace for this shape
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.sat(x, out=y)
+    big = gen(4096, 4096, "int32", seed=62)
+    with torch.cuda.stream(s):
+        yb = libsat.sat(dev(big))            # grows the descriptors: old buffers retired
+    s.synchronize()
+    check(yb, oracle.sat(big), "int32")
+    sentinel = torch.full((64 << 20,), 0x5A5A5A5A, dtype=torch.int32, device="cuda")
+    for it in range(3):
+        host = gen(640, 1280, "int32", seed=70 + it)
+        x.copy_(dev(host))
+        with torch.cuda.stream(s):
+            g.replay()
+        s.synchronize()
+        check(y, oracle.sat(host), "int32")
+    assert bool((sentinel == 0x5A5A5A5A).all())
+    libsat.release_workspace(s)
+    with torch.cuda.stream(s):
+        z = libsat.sat(x)
+    s.synchronize()
+    check(z, oracle.sat(x.cpu().numpy()), "int32")
