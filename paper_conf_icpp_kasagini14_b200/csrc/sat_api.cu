@@ -126,6 +126,8 @@ struct Workspace {
     Buf part;                 // column totals partials
     Buf cnt;                  // column totals: per-chunk-column and global arrival counters (self-resetting)
     Buf bticket;              // fused box filter: unit ticket (zeroed per call on the stream)
+    Buf order;                // segment-unit ticket order (int2 per unit), for order_key
+    unsigned long long order_key = 0;
     Buf shard;                // sharded default workspace
     Buf din, dout;            // host e2e device copies
     std::vector<void*> retired;   // buffers a captured graph may still reference (freed by sat_release_workspace)
@@ -589,6 +591,35 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
             p.nseg = (p.nc + p.segc - 1) / p.segc;
             p.total_units = (long long)p.total_bands * p.nseg;
         }
+    }
+    // Skewed ticket order of the segment units: sorted
+    // by band + K * segment with K = 12 x resident CTAs / segments, so the
+    // band above a unit (same segment) runs ~nseg tickets earlier instead of
+    // alongside it, and the same band's previous segment ~K * nseg tickets
+    // earlier (long finished).  65536^2: 5.81-5.87 vs 5.87-5.97 ms,
+    // 49152^2: 3.37-3.41 vs 3.45-3.47 (three rounds each, profiles/r02_skew.txt);
+    // where K exceeds the bands it is the plain segment-major order.
+    constexpr int kSkewMult = 12;
+    p.order = nullptr;
+    if (p.nseg > 1) {
+        const int K = std::max(1, kSkewMult * j.di->sms * ctas_per_sm(j.dtype, j.th) / p.nseg);
+        const unsigned long long key = (unsigned long long)p.total_bands | ((unsigned long long)p.nseg << 32) |
+                                       ((unsigned long long)K << 44);
+        Workspace& w = *j.ws;
+        if (w.order_key != key || !w.order.p) {
+            std::vector<int2> ord;
+            ord.reserve(size_t(p.total_bands) * p.nseg);
+            const long long kmax = (long long)p.total_bands - 1 + (long long)K * (p.nseg - 1);
+            for (long long d = 0; d <= kmax; ++d)
+                for (int sg = 0; sg < p.nseg; ++sg) {
+                    const long long b = d - (long long)K * sg;
+                    if (b >= 0 && b < p.total_bands) ord.push_back(make_int2(sg, int(b)));
+                }
+            SAT_TRY(ensure(w.order, ord.size() * sizeof(int2), false));
+            CUDA_TRY(cudaMemcpy(w.order.p, ord.data(), ord.size() * sizeof(int2), cudaMemcpyHostToDevice));
+            w.order_key = key;
+        }
+        p.order = static_cast<const int2*>(w.order.p);
     }
     p.jitter = j.jitter;
     if (kDebug) {
@@ -1572,7 +1603,7 @@ int sat_release_workspace(void* stream) {
     // the stream's queued work may still use the buffers
     CUDA_TRY(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     for (Buf* b : {&w->desc, &w->lseg, &w->ticket, &w->bt, &w->rs, &w->lx, &w->lsum, &w->topx, &w->lb,
-                   &w->tr, &w->box, &w->part, &w->cnt, &w->bticket, &w->shard, &w->din, &w->dout})
+                   &w->tr, &w->box, &w->part, &w->cnt, &w->bticket, &w->order, &w->shard, &w->din, &w->dout})
         free_buf(*b);
     for (void* p : w->retired) cudaFree(p);
     if (w->cstream_in) cudaStreamDestroy(w->cstream_in);

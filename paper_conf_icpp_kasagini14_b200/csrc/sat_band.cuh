@@ -506,8 +506,14 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
             j0 = min(r1, r0 + sr * p.tile_units);
             j1 = min(r1, j0 + p.tile_units);
         } else if (p.nseg > 1) {
-            seg = int(unit / p.total_bands);
-            gb = int(unit - (long long)seg * p.total_bands);
+            if (p.order != nullptr) {
+                const int2 u = __ldg(p.order + unit);
+                seg = u.x;
+                gb = u.y;
+            } else {
+                seg = int(unit / p.total_bands);
+                gb = int(unit - (long long)seg * p.total_bands);
+            }
             j0 = seg * p.segc;
             j1 = min(p.nc, j0 + p.segc);
         } else {

@@ -84,6 +84,11 @@ struct BandParams {
     int nseg;                  // 1 = whole bands
     int segc;                  // chunks per segment
     uint64_t* Lseg;            // [total_bands][TH] row carry at the end of the band's last segment
+    // Ticket order of the segment units (nullable = segment-major): order[t]
+    // = (segment, band) of ticket t, sorted by band + K * segment: both
+    // predecessors of a unit -- the same segment of the band above and the
+    // previous segment of the same band -- hold earlier tickets.
+    const int2* order;
     unsigned long long* trace; // debug builds (SAT_DEBUG): [total_bands*nc][8] event times (ns), nullable
     unsigned int* diag;        // debug builds: host-mapped progress marks, nullable
 };
