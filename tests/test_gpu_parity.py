@@ -719,3 +719,38 @@ def test_graph_replay_after_workspace_growth(libsat):
         z = libsat.sat(x)
     s.synchronize()
     check(z, oracle.sat(x.cpu().numpy()), "int32")
+
+
+@pytest.mark.slow
+def test_fused_exchange_with_band_segments(libsat):
+    """Strips tall and wide enough for band segments (> one wave of TH-128
+    bands, >= 32 chunks): every band-0 segment unit adds its columns' share of
+    the peers' totals, and only the last one acknowledges (the self-resetting
+    counter), over 4 consecutive calls (both parities) on 2 virtual ranks."""
+    from paper_conf_icpp_kasagini14_b200.dist import partition_rows
+    P, n, m = 2, 2 * 20480, 4096
+    nb = libsat.PeerExchange.mailbox_bytes(m, P, torch.int32)
+    boxes = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(P)]
+    ptrs = [b.data_ptr() for b in boxes]
+    exs = [libsat.PeerExchange(p, P, m, torch.int32, boxes[p], ptrs) for p in range(P)]
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    bounds = [partition_rows(n, P, p) for p in range(P)]
+    for it in range(4):
+        full = make_torch(n, m, "int32", "u32", seed=90 + it, device="cuda")
+        strips = [full[a:b] for a, b in bounds]
+        outs = [torch.empty_like(s) for s in strips]
+        torch.cuda.synchronize()
+        for p in range(P):
+            with torch.cuda.stream(streams[p]):
+                exs[p].sat(strips[p], out=outs[p], stream=streams[p])
+        torch.cuda.synchronize()
+        # rank 1's strip against the oracle streamed from torch column sums of rank 0's rows
+        st = oracle.Stream(m, True)
+        st.colsum[:] = (full[:bounds[1][0]].to(torch.int64).sum(dim=0) % 2**32).cpu().numpy().astype(np.uint32)
+        r0 = bounds[1][0]
+        for a in range(0, bounds[1][1] - r0, 4096):
+            ref = st.feed(full[r0 + a:r0 + a + 4096].cpu().numpy())
+            assert np.array_equal(outs[1][a:a + 4096].cpu().numpy(), ref), (it, a)
+        check(outs[0][:512], oracle.sat(full[:512].cpu().numpy()), "int32")
+    for e in exs:
+        e.close()
