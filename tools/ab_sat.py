@@ -18,7 +18,7 @@ import oracle
 import paper_conf_icpp_kasagini14_b200 as libsat
 from sat_inputs import make_np, make_torch
 
-shapes = [tuple(int(v) for v in s.split("x")) for s in sys.argv[1].split(",")]
+shapes = [tuple(int(v) for v in s.split("x")) for s in sys.argv[1].split(",")]   # n x m, or batch x n x m
 cfgs = [tuple(int(v) for v in c.split(":")) for c in sys.argv[2].split(",")]
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 10
 rounds = int(sys.argv[4]) if len(sys.argv) > 4 else 3
@@ -36,27 +36,34 @@ for c in cfgs:
     print(f"parity th={th} seg={seg}: {ok[c]} (th used {libsat.last_tile_rows()})", flush=True)
 
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
-for (n, m) in shapes:
-    x = make_torch(n, m, dtype, dist, seed=1, device="cuda")
+def call(x, y, c):
+    if x.dim() == 3:
+        return libsat.sat_batched(x, out=y, tile_rows=c[0], segments=c[1])
+    return libsat.sat(x, out=y, tile_rows=c[0], segments=c[1])
+
+
+for shp in shapes:
+    bt, (n, m) = (shp[0], shp[1:]) if len(shp) == 3 else (None, shp)
+    x = make_torch(n, m, dtype, dist, seed=1, device="cuda", batch=bt)
     y = torch.empty_like(x)
     res = {c: [] for c in cfgs}
     for c in cfgs:
         for _ in range(2):
-            libsat.sat(x, out=y, tile_rows=c[0], segments=c[1])
+            call(x, y, c)
     for _ in range(rounds):
         for c in cfgs:
             for _ in range(reps):
                 flush.fill_(1)
                 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 s.record()
-                libsat.sat(x, out=y, tile_rows=c[0], segments=c[1])
+                call(x, y, c)
                 e.record()
                 e.synchronize()
                 res[c].append(s.elapsed_time(e))
     nb = 2 * x.numel() * x.element_size()
     for c in cfgs:
         ms = statistics.median(res[c])
-        print(f"{n}x{m} {dtype} th={c[0]} seg={c[1]} median {ms:.4f} ms min {min(res[c]):.4f} "
+        print(f"{'x'.join(map(str, shp))} {dtype} th={c[0]} seg={c[1]} median {ms:.4f} ms min {min(res[c]):.4f} "
               f"{nb / ms / 1e6:.0f} GB/s frac {nb / ms / 1e6 / 6550.1:.3f} parity={ok[c]}", flush=True)
     del x, y
     torch.cuda.empty_cache()

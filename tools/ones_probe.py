@@ -16,12 +16,11 @@ for rows, cols in cases:
     ii = torch.arange(1, rows + 1, device="cuda", dtype=torch.int64).view(-1, 1)
     jj = torch.arange(1, cols + 1, device="cuda", dtype=torch.int64).view(1, -1)
     for th in (64, 128):
-        for seg in ("1", "4", "16"):
+        for seg in (1, 4, 16):
             for inplace in (False, True):
-                os.environ["SAT_SEG"] = seg
                 x = torch.ones(rows, cols, dtype=torch.int32, device="cuda")
                 try:
-                    y = libsat.sat(x, out=x if inplace else None, tile_rows=th)
+                    y = libsat.sat(x, out=x if inplace else None, tile_rows=th, segments=seg)
                     torch.cuda.synchronize()
                 except Exception as e:
                     print(rows, cols, th, seg, inplace, "ERROR", e, flush=True)

@@ -15,17 +15,20 @@ from sat_inputs import make_torch
 rows, cols, th = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
 out = sys.argv[4]
 seg = int(sys.argv[5]) if len(sys.argv) > 5 else 0
-x = make_torch(rows, cols, "int32", "u32", seed=1, device="cuda")
+batch = int(sys.argv[6]) if len(sys.argv) > 6 else None
+x = make_torch(rows, cols, "int32", "u32", seed=1, device="cuda", batch=batch)
 y = torch.empty_like(x)
+run = (lambda: libsat.sat(x, out=y, tile_rows=th, segments=seg)) if batch is None else \
+    (lambda: libsat.sat_batched(x, out=y, tile_rows=th, segments=seg))
 for _ in range(3):
-    libsat.sat(x, out=y, tile_rows=th, segments=seg)
-nb, nc = (rows + th - 1) // th, (cols + 127) // 128
+    run()
+nb, nc = (batch or 1) * ((rows + th - 1) // th), (cols + 127) // 128
 buf = torch.zeros(nb * nc * 8, dtype=torch.int64, device="cuda")
 torch.cuda.synchronize()
 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 libsat.debug_trace(buf)
 s.record()
-libsat.sat(x, out=y, tile_rows=th, segments=seg)
+run()
 e.record()
 torch.cuda.synchronize()
 print("ms", s.elapsed_time(e), "th", libsat.last_tile_rows(), "grid", libsat.last_grid())
