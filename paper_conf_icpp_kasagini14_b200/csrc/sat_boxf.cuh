@@ -47,7 +47,7 @@ template <int MAXH, int NS, typename TI, typename TS, int NWARP>
 struct BoxSmem {
     static constexpr size_t ring = size_t(NS) * MAXH * TW * sizeof(TI);
     static constexpr size_t ring_al = (ring + 127) / 128 * 128;
-    static constexpr size_t satb = size_t(3) * MAXH * TW * sizeof(TS);
+    static constexpr size_t satb = size_t(3) * (MAXH + 1) * TW * sizeof(TS);   // row 0 of each buffer: zeros
     static constexpr size_t bot = size_t(NWARP) * TW * sizeof(TS);
     static constexpr size_t bars = size_t(NS) * 8 + 16;
     static constexpr size_t total = ring_al + satb + bot + bars;
@@ -63,7 +63,7 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
     using SM = BoxSmem<MAXH, NS, TI, TS, NWARP>;
     extern __shared__ __align__(1024) uint8_t smem[];
     TI* ring = reinterpret_cast<TI*>(smem);
-    TS* satb = reinterpret_cast<TS*>(smem + SM::ring_al);            // [3][MAXH][TW]
+    TS* satb = reinterpret_cast<TS*>(smem + SM::ring_al);            // [3][1 + MAXH][TW]
     TS* bot = reinterpret_cast<TS*>(smem + SM::ring_al + SM::satb);  // [NWARP][TW]
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + SM::ring_al + SM::satb + SM::bot);
     long long* s_unit = reinterpret_cast<long long*>(full + NS);
@@ -73,6 +73,9 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
         fence_mbar_init();
         prefetch_tmap(&tm_in);
     }
+    // row 0 of every chunk buffer holds the SAT row above the halo: zeros
+    for (int i = threadIdx.x; i < 3 * TW; i += blockDim.x)
+        satb[size_t(i / TW) * (MAXH + 1) * TW + (i % TW)] = TS(0);
     __syncthreads();
     asm volatile("griddepcontrol.wait;" ::: "memory");
     const uint64_t pol = policy_evict_first();
@@ -116,11 +119,15 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
                 // prefix down this warp's rows
                 const TI* src = ring + size_t(qk % NS) * MAXH * TW + 4 * lane;
                 const bool cin = k * TW + 4 * lane < bp.cols;
+                // warps whose rows all lie below the halo band (H < MAXH for
+                // small radii) have nothing to do: their rows are never read
+                const bool act = warp * RPW < H;
                 TS v[RPW][4];
                 TS run[4] = {TS(0), TS(0), TS(0), TS(0)};
 #pragma unroll
                 for (int r = 0; r < RPW; ++r) {
                     const int lr = warp * RPW + r;
+                    if (!act) break;
                     TS e[4] = {TS(0), TS(0), TS(0), TS(0)};
                     if (lr < H && cin) {
                         if constexpr (sizeof(TI) == 1) {
@@ -146,14 +153,14 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
                 for (int i = 0; i < 4; ++i) b[i] = run[i];
                 __syncthreads();                        // bottom rows published, ring slot read
                 TS add[4] = {TS(0), TS(0), TS(0), TS(0)};
-                for (int w2 = 0; w2 < warp; ++w2)
+                for (int w2 = 0; act && w2 < warp; ++w2)
 #pragma unroll
                     for (int i = 0; i < 4; ++i) add[i] += bot[w2 * TW + 4 * lane + i];
-                TS* dst = satb + size_t(k % 3) * MAXH * TW + 4 * lane;
+                TS* dst = satb + (size_t(k % 3) * (MAXH + 1) + 1) * TW + 4 * lane;
 #pragma unroll
                 for (int r = 0; r < RPW; ++r) {
                     const int lr = warp * RPW + r;
-                    if (lr < MAXH) {
+                    if (lr < H) {
                         if constexpr (sizeof(TS) == 4) {
                             *reinterpret_cast<uint4*>(dst + size_t(lr) * TW) =
                                 make_uint4(to_bits(v[r][0] + add[0]), to_bits(v[r][1] + add[1]),
@@ -175,31 +182,43 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
                 // corner reads of a warp hit 32 consecutive words (no bank
                 // conflicts; a 4-consecutive-columns-per-lane mapping made
                 // them 4-way)
-                int j2[4], j1[4];
+                // per lane and e: smem offsets of the two corner columns
+                // (buffer of their chunk + column in it), and a mask that
+                // zeroes the left corner terms when j1 - 1 < 0
+                int o2[4], o1[4];
+                TS m1[4];
 #pragma unroll
                 for (int e = 0; e < 4; ++e) {
                     const int j = kc * TW + lane + 32 * e;
-                    j2[e] = min(j + bp.rc, bp.cols - 1);
-                    j1[e] = max(j - bp.rc, 0) - 1;      // -1: column before the image (S = 0)
+                    const int j2 = min(j + bp.rc, bp.cols - 1);
+                    const int j1 = max(j - bp.rc, 0) - 1;      // -1: column before the image (S = 0)
+                    const int jl = max(j1, 0);
+                    o2[e] = ((j2 >> 7) % 3) * (MAXH + 1) * TW + (j2 & (TW - 1));
+                    o1[e] = ((jl >> 7) % 3) * (MAXH + 1) * TW + (jl & (TW - 1));
+                    m1[e] = j1 >= 0 ? TS(1) : TS(0);
+                    if constexpr (std::is_same<TS, uint32_t>::value) m1[e] = j1 >= 0 ? 0xFFFFFFFFu : 0u;
                 }
-                auto sat_at = [&](int lr, int c) -> TS {
-                    if (lr < 0 || c < 0) return TS(0);
-                    return box_ld(satb + (size_t((c >> 7) % 3) * MAXH + lr) * TW + (c & (TW - 1)));
-                };
                 for (int i = r0 + warp; i < r1; i += NWARP) {
-                    const int a2 = min(i + bp.rr, bp.rows - 1) - t0;
-                    const int a1 = max(i - bp.rr, 0) - 1 - t0;
+                    // local SAT rows of the window's last row and of the row
+                    // above its first (+1: row 0 of each buffer is zero)
+                    const int a2 = (min(i + bp.rr, bp.rows - 1) - t0 + 1) * TW;
+                    const int a1 = (max(i - bp.rr, 0) - t0) * TW;
                     TO* prow = gout + int64_t(i) * bp.cols + kc * TW + lane;
+                    int hh = 0;
+                    if constexpr (!std::is_same<TS, uint32_t>::value)
+                        hh = min(i + bp.rr, bp.rows - 1) - max(i - bp.rr, 0) + 1;
 #pragma unroll
                     for (int e = 0; e < 4; ++e) {
-                        TS s = sat_at(a2, j2[e]);
-                        s -= sat_at(a1, j2[e]);
-                        s -= sat_at(a2, j1[e]);
-                        s += sat_at(a1, j1[e]);
-                        if constexpr (!std::is_same<TS, uint32_t>::value) {
+                        const TS right = satb[a2 + o2[e]] - satb[a1 + o2[e]];
+                        const TS left = satb[a2 + o1[e]] - satb[a1 + o1[e]];
+                        TS s;
+                        if constexpr (std::is_same<TS, uint32_t>::value) {
+                            s = right - (left & m1[e]);
+                        } else {
+                            s = right - left * m1[e];
                             if (bp.normalize) {
-                                const int hh = min(i + bp.rr, bp.rows - 1) - max(i - bp.rr, 0) + 1;
-                                const int ww = j2[e] - j1[e];
+                                const int j = kc * TW + lane + 32 * e;
+                                const int ww = min(j + bp.rc, bp.cols - 1) - max(j - bp.rc, 0) + 1;
                                 s = s / TS(int64_t(hh) * int64_t(ww));
                             }
                         }
