@@ -267,6 +267,15 @@ struct BandCfg {
 // per compute thread.  Two CTAs per SM.
 constexpr BandCfg kCfg16{4, 4, 3, 8, 4, 4, 1, 2};
 constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
+// TH 32 when the bands fit in one wave of ONE CTA per SM (4096^2: 128
+// bands): 8 compute warps of 4 rows, a 4 x 32 KB ring, 16 chunks parked (all
+// 512 TMEM columns) and 12 control groups walking one band per round trip.
+// The look-back of a lockstep wave is ~11 hops deep, so its latency (not the
+// bandwidth) sets the chunk rate: 4096^2 int32 45 vs 53-55 us, 3072^2 35 vs
+// 41, 2048^2 25 vs 29 (profiles/r02_small.txt; 8 groups 47, window 2 / 4:
+// 49 / 53, 8 parked chunks 51)
+constexpr BandCfg kCfg32S{4, 8, 4, 16, 2, 12, 1, 1};
+constexpr int kLbw32S = 1;
 // column / row passes (2R2W, 4R4W) at TH 64: two CTAs per SM
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // 1R1W at TH 64 ("wide"): one CTA per SM, 192 KB ring of 64 x 256 slots
@@ -418,8 +427,11 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
         return fail(SAT_ERR_INVALID, "float64: no band configuration for this tile_rows");
     } else {
         switch (th) {
+            case 32:
+                if (p.top_src == TOP_LOOKBACK && p.total_units <= di.sms)
+                    return launch_band_t<T, SAT_CFG(kCfg32S), MODE, TMA, kCfg32S.MINB, kLbw32S>(p, ti, di, st, grid);
+                return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
             case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, di, st, grid);
-            case 32: return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
             case 64: return launch_band_t<T, SAT_CFG(kCfg64W), MODE, TMA, kCfg64W.MINB>(p, ti, di, st, grid);
             case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
         }
@@ -478,19 +490,19 @@ int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dty
             const long long bands = batch * ((rows + th - 1) / th);
             if (bands * 5 >= 4LL * di.sms) return th;
         }
-        return rows * batch >= 1024 ? 32 : 16;
+        return rows * batch >= 512 ? 32 : 16;
     }
     // 1R1W (one CTA per SM for TH 64 and 128; r02 sweep, profiles/r02_ab_th.txt):
     // TH = 128 once its bands fill about two thirds of the SMs (the look-back
     // chain is one hop per band; 16K^2+: 5.3-5.4 TB/s); the wide TH 64 below
     // that while its bands fill 60 % of the SMs (6144^2-10240^2: 9-11 %
-    // faster than TH 32 or 128); then TH 32 from 1536 rows (2048^2-4096^2:
-    // 15-25 % faster than TH 16), else TH 16.
+    // faster than TH 32 or 128); then TH 32 from 512 rows (one wave of
+    // kCfg32S: 768^2-4096^2 10-40 % faster than TH 16), else TH 16.
     if (variant == SAT_1R1W || variant == SAT_1PLUSR_R1W) {   // (1+r): its band C is 1R1W
         const long long b128 = batch * ((rows + 127) / 128), b64 = batch * ((rows + 63) / 64);
         if (b128 * 100 >= 65LL * di.sms) return 128;
         if (b64 * 10 >= 6LL * di.sms) return 64;
-        return rows * batch >= 1536 ? 32 : 16;
+        return rows * batch >= 512 ? 32 : 16;
     }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
     for (int th : {64, 32}) {

@@ -245,6 +245,21 @@ int main(int argc, char** argv) {
         printf("flat       grid=%4d x 512  best %.4f ms %.0f GB/s avg %.4f ms %.0f GB/s\n", f.grid, best,
                2.0 * n * n * 4 / best / 1e6, avg, 2.0 * n * n * 4 / avg / 1e6);
     }
+    if (argc > 2 && argv[2][0] == 's') {
+        // small matrices (one wave of bands, argv[2] = "s"): ring depth / box
+        // geometry at TH 32 and 16, band-major and strip-major
+        run<32, 256, 4, 8, 0>(n, in, out, n / 256, 1, "b32c256s4");
+        run<32, 256, 6, 8, 0>(n, in, out, n / 256, 1, "b32c256s6");
+        run<32, 512, 3, 8, 0>(n, in, out, n / 512, 1, "b32c512s3");
+        run<32, 128, 8, 8, 0>(n, in, out, n / 128, 1, "b32c128s8");
+        run<32, 256, 3, 4, 0>(n, in, out, n / 256, 2, "b32c256s3o2");
+        run<16, 512, 6, 8, 0>(n, in, out, n / 512, 1, "b16c512s6");
+        run<16, 512, 3, 8, 0>(n, in, out, n / 512, 2, "b16c512s3o2");
+        run<32, 256, 4, 8, 0>(n, in, out, n / 1024, 1, "b32c256u4");
+        run<32, 128, 4, 8, 0, true>(n, in, out, n / 256, 1, "strip32u16");
+        run<32, 128, 6, 8, 0, true>(n, in, out, n / 128, 1, "strip32s4");
+        return 0;
+    }
     const int nc = n / 128;
     const int nr = n / 128;   // 128-row chunks per strip
     run<128, 128, 3, 16, 0>(n, in, out, nc, 1, "band128");

@@ -1,6 +1,6 @@
 """Record per-(band, chunk) look-back event times of one 1R1W launch.
 
-python tools/trace_lookback.py rows cols tile_rows out.npz
+python tools/trace_lookback.py rows cols tile_rows out.npz [segments] [batch] [xcfg]
 """
 import os
 import sys
@@ -15,11 +15,22 @@ from sat_inputs import make_torch
 rows, cols, th = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
 out = sys.argv[4]
 seg = int(sys.argv[5]) if len(sys.argv) > 5 else 0
-batch = int(sys.argv[6]) if len(sys.argv) > 6 else None
+batch = (int(sys.argv[6]) or None) if len(sys.argv) > 6 else None
 x = make_torch(rows, cols, "int32", "u32", seed=1, device="cuda", batch=batch)
 y = torch.empty_like(x)
-run = (lambda: libsat.sat(x, out=y, tile_rows=th, segments=seg)) if batch is None else \
-    (lambda: libsat.sat_batched(x, out=y, tile_rows=th, segments=seg))
+xcfg = int(sys.argv[7]) if len(sys.argv) > 7 else 0     # sat_options.reserved[0] (experiments)
+
+
+def run():
+    import ctypes
+    o = libsat.options(tile_rows=th, segments=seg)
+    o.reserved[0] = xcfg
+    if batch is None:
+        libsat._check(libsat._lib.sat_compute_ex(x.data_ptr(), y.data_ptr(), rows, cols, libsat._dtype_code(x), 2,
+                                                 ctypes.byref(o), None))
+    else:
+        libsat._check(libsat._lib.sat_compute_batched(x.data_ptr(), y.data_ptr(), batch, rows, cols,
+                                                      libsat._dtype_code(x), 2, ctypes.byref(o), None))
 for _ in range(3):
     run()
 nb, nc = (batch or 1) * ((rows + th - 1) // th), (cols + 127) // 128
