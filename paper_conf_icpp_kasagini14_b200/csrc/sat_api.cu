@@ -276,6 +276,7 @@ constexpr BandCfg kCfg32{8, 4, 3, 8, 2, 4, 1, 2};
 // 49 / 53, 8 parked chunks 51)
 constexpr BandCfg kCfg32S{4, 8, 4, 16, 2, 12, 1, 1};
 constexpr int kLbw32S = 1;
+
 // column / row passes (2R2W, 4R4W) at TH 64: two CTAs per SM
 constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // 1R1W at TH 64 ("wide"): one CTA per SM, 192 KB ring of 64 x 256 slots
@@ -283,8 +284,11 @@ constexpr BandCfg kCfg64{8, 8, 3, 4, 1, 4, 1, 2};
 // columns).  Between one half and two thirds of a wave of 128-row bands it
 // beats both TH 32 and TH 128: 6144^2 int32 0.084 vs 0.094 ms (TH 32),
 // 8192^2 0.127 vs 0.143, 10240^2 0.179 vs 0.198 (TH 128); the two-CTA TH-64
-// configuration was 20-30 % slower (profiles/r02_ab_th.txt)
-constexpr BandCfg kCfg64W{8, 8, 3, 8, 2, 4, 1, 1};
+// configuration was 20-30 % slower (profiles/r02_ab_th.txt).  8 control
+// groups walking one band per round trip: 6144^2-12288^2 5-7 % faster than 4
+// groups with a window of 4 (profiles/r02_small.txt)
+constexpr BandCfg kCfg64W{8, 8, 3, 8, 2, 8, 1, 1};
+constexpr int kLbw64W = 1;
 // TH = 128: 16 compute warps, one CTA per SM (ring 3 x 64 KB, TMEM 4 chunks =
 // all 512 columns); half the descriptor bytes and look-back hops per element
 constexpr BandCfg kCfg128{8, 16, 3, 4, 1, 3, 1, 1};
@@ -432,7 +436,7 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
                     return launch_band_t<T, SAT_CFG(kCfg32S), MODE, TMA, kCfg32S.MINB, kLbw32S>(p, ti, di, st, grid);
                 return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
             case 16: return launch_band_t<T, SAT_CFG(kCfg16), MODE, TMA, kCfg16.MINB>(p, ti, di, st, grid);
-            case 64: return launch_band_t<T, SAT_CFG(kCfg64W), MODE, TMA, kCfg64W.MINB>(p, ti, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfg64W), MODE, TMA, kCfg64W.MINB, kLbw64W>(p, ti, di, st, grid);
             case 128: return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
         }
         return fail(SAT_ERR_INVALID, "no band configuration for this tile_rows");
