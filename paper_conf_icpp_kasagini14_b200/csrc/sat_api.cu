@@ -307,6 +307,11 @@ constexpr BandCfg kCfgD64{8, 8, 3, 4, 1, 2, 2, 1};   // 224 KB smem, 512 TMEM co
 // warps of 2 columns per lane (4 descriptor words per band, window 2)
 constexpr BandCfg kCfgD128{8, 16, 3, 4, 1, 3, 1, 1};
 constexpr int kTwD128 = 64;
+// float64 1R1W at TH 64 / 128: one band per look-back round trip (18432^2
+// 1.076 vs 1.101 ms at TH 64, 1.002 vs 1.006 at TH 128; more control groups
+// were 2-8 % slower, profiles/r02_float64_th128.txt)
+constexpr int kLbwD = 1;
+
 // uint8 input widened to uint32 sums: the ring holds bytes (TH x 128 B per
 // chunk), so it is 6 slots deep
 constexpr BandCfg kCfgU64{8, 8, 6, 4, 1, 4, 1, 2};
@@ -422,11 +427,11 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
         }
     } else if constexpr (sizeof(T) == 8) {
         switch (th) {
-            case 128: return launch_band_t<T, SAT_CFG(kCfgD128), MODE, TMA, kCfgD128.MINB, kLbw128, T, kTwD128>(
+            case 128: return launch_band_t<T, SAT_CFG(kCfgD128), MODE, TMA, kCfgD128.MINB, kLbwD, T, kTwD128>(
                           p, ti, di, st, grid);
             case 16: return launch_band_t<T, SAT_CFG(kCfgD16), MODE, TMA, kCfgD16.MINB>(p, ti, di, st, grid);
             case 32: return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
-            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
+            case 64: return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB, kLbwD>(p, ti, di, st, grid);
         }
         return fail(SAT_ERR_INVALID, "float64: no band configuration for this tile_rows");
     } else {
