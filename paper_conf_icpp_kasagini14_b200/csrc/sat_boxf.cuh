@@ -53,8 +53,19 @@ struct BoxSmem {
     static constexpr size_t total = ring_al + satb + bot + bars;
 };
 
+// scalar shared load from a 32-bit shared-window address
 template <typename T>
-__device__ __forceinline__ T box_ld(const T* s) { return *s; }
+__device__ __forceinline__ T lds_s(uint32_t a) {
+    if constexpr (sizeof(T) == 4) {
+        uint32_t v;
+        asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a));
+        return from_bits<T>(v);
+    } else {
+        double v;
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+        return T(v);
+    }
+}
 
 template <typename TI, typename TS, typename TO, int TH, int MAXH, int NS, int NWARP>
 __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_constant__ CUtensorMap tm_in,
@@ -182,49 +193,56 @@ __global__ void __launch_bounds__(NWARP * 32, 1) sat_boxf_kernel(const __grid_co
                 // corner reads of a warp hit 32 consecutive words (no bank
                 // conflicts; a 4-consecutive-columns-per-lane mapping made
                 // them 4-way)
-                // per lane and e: smem offsets of the two corner columns
-                // (buffer of their chunk + column in it), and a mask that
-                // zeroes the left corner terms when j1 - 1 < 0
-                int o2[4], o1[4];
+                // per lane and e: shared addresses of the two corner columns
+                // (buffer of their chunk + column in it; 32-bit shared-window
+                // addresses, so a corner read is one IADD + LDS), and a mask
+                // that zeroes the left corner terms when j1 - 1 < 0
+                uint32_t o2[4], o1[4];
                 TS m1[4];
+                const uint32_t sb = smem_u32(satb);
 #pragma unroll
                 for (int e = 0; e < 4; ++e) {
                     const int j = kc * TW + lane + 32 * e;
                     const int j2 = min(j + bp.rc, bp.cols - 1);
                     const int j1 = max(j - bp.rc, 0) - 1;      // -1: column before the image (S = 0)
                     const int jl = max(j1, 0);
-                    o2[e] = ((j2 >> 7) % 3) * (MAXH + 1) * TW + (j2 & (TW - 1));
-                    o1[e] = ((jl >> 7) % 3) * (MAXH + 1) * TW + (jl & (TW - 1));
-                    m1[e] = j1 >= 0 ? TS(1) : TS(0);
+                    o2[e] = sb + uint32_t((((j2 >> 7) % 3) * (MAXH + 1) * TW + (j2 & (TW - 1))) * sizeof(TS));
+                    o1[e] = sb + uint32_t((((jl >> 7) % 3) * (MAXH + 1) * TW + (jl & (TW - 1))) * sizeof(TS));
                     if constexpr (std::is_same<TS, uint32_t>::value) m1[e] = j1 >= 0 ? 0xFFFFFFFFu : 0u;
+                    else m1[e] = j1 >= 0 ? TS(1) : TS(0);
                 }
-                for (int i = r0 + warp; i < r1; i += NWARP) {
-                    // local SAT rows of the window's last row and of the row
-                    // above its first (+1: row 0 of each buffer is zero)
-                    const int a2 = (min(i + bp.rr, bp.rows - 1) - t0 + 1) * TW;
-                    const int a1 = (max(i - bp.rr, 0) - t0) * TW;
-                    TO* prow = gout + int64_t(i) * bp.cols + kc * TW + lane;
-                    int hh = 0;
-                    if constexpr (!std::is_same<TS, uint32_t>::value)
-                        hh = min(i + bp.rr, bp.rows - 1) - max(i - bp.rr, 0) + 1;
+                const bool full_chunk = kc * TW + TW <= bp.cols;
+                const int64_t rstride = int64_t(NWARP) * bp.cols;
+                TO* prow = gout + int64_t(r0 + warp) * bp.cols + kc * TW + lane;
+                for (int i = r0 + warp; i < r1; i += NWARP, prow += rstride) {
+                    // byte offsets of the local SAT rows of the window's last row
+                    // and of the row above its first (+1: row 0 of each buffer is zero)
+                    const uint32_t a2 = uint32_t((min(i + bp.rr, bp.rows - 1) - t0 + 1) * TW * int(sizeof(TS)));
+                    const uint32_t a1 = uint32_t((max(i - bp.rr, 0) - t0) * TW * int(sizeof(TS)));
+                    TS s[4];
 #pragma unroll
                     for (int e = 0; e < 4; ++e) {
-                        const TS right = satb[a2 + o2[e]] - satb[a1 + o2[e]];
-                        const TS left = satb[a2 + o1[e]] - satb[a1 + o1[e]];
-                        TS s;
-                        if constexpr (std::is_same<TS, uint32_t>::value) {
-                            s = right - (left & m1[e]);
-                        } else {
-                            s = right - left * m1[e];
-                            if (bp.normalize) {
+                        const TS right = lds_s<TS>(a2 + o2[e]) - lds_s<TS>(a1 + o2[e]);
+                        const TS left = lds_s<TS>(a2 + o1[e]) - lds_s<TS>(a1 + o1[e]);
+                        if constexpr (std::is_same<TS, uint32_t>::value) s[e] = right - (left & m1[e]);
+                        else s[e] = right - left * m1[e];
+                    }
+                    if constexpr (!std::is_same<TS, uint32_t>::value) {
+                        if (bp.normalize) {
+                            const int hh = min(i + bp.rr, bp.rows - 1) - max(i - bp.rr, 0) + 1;
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
                                 const int j = kc * TW + lane + 32 * e;
                                 const int ww = min(j + bp.rc, bp.cols - 1) - max(j - bp.rc, 0) + 1;
-                                s = s / TS(int64_t(hh) * int64_t(ww));
+                                s[e] = s[e] / TS(int64_t(hh) * int64_t(ww));
                             }
                         }
-                        if (kc * TW + lane + 32 * e < bp.cols) {
-                            if constexpr (std::is_same<TS, uint32_t>::value) __stcs(prow + 32 * e, TO(int32_t(s)));
-                            else __stcs(prow + 32 * e, TO(s));
+                    }
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) {
+                        if (full_chunk || kc * TW + lane + 32 * e < bp.cols) {
+                            if constexpr (std::is_same<TS, uint32_t>::value) __stcs(prow + 32 * e, TO(int32_t(s[e])));
+                            else __stcs(prow + 32 * e, TO(s[e]));
                         }
                     }
                 }
