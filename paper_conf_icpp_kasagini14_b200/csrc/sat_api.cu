@@ -606,6 +606,10 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         // the band's previous segment)
         const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th);
         int want = p.total_bands > slots ? std::min(16, p.nc / 16) : 1;
+        // short bands (batches of images): segments of >= 3 chunks
+        // (32 x 1080x1920 float32: 0.1045 vs 0.1070 ms, 64 images 0.1935 vs
+        // 0.2048 with 5 segments of 3 chunks, profiles/r02_small.txt)
+        if (p.total_bands > slots && want < 2) want = std::min(5, p.nc / 3);
         if (j.segments > 0) want = j.segments;
         if (want > 1 && p.nc > 1) {
             p.segc = (p.nc + want - 1) / want;
