@@ -609,7 +609,10 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         // short bands (batches of images): segments of >= 3 chunks
         // (32 x 1080x1920 float32: 0.1045 vs 0.1070 ms, 64 images 0.1935 vs
         // 0.2048 with 5 segments of 3 chunks, profiles/r02_small.txt)
-        if (p.total_bands > slots && want < 2) want = std::min(5, p.nc / 3);
+        // (not the widening loads: 32 x 1080x1920 uint8 -> int32 0.078 vs
+        // 0.084 ms, float32 -> float64 0.187 vs 0.24-0.25 without / with)
+        if (p.total_bands > slots && want < 2 && j.in_dtype == j.dtype && j.dtype != SAT_FLOAT64)
+            want = std::min(5, p.nc / 3);
         if (j.segments > 0) want = j.segments;
         if (want > 1 && p.nc > 1) {
             p.segc = (p.nc + want - 1) / want;
@@ -1075,7 +1078,7 @@ int sharded_fused_t(const void* in, void* out, int64_t strip_rows, PeerExchange&
 }
 
 // Fused box filter (sat_boxf.cuh): one launch, the SAT stays on chip.
-template <typename TI, typename TS, typename TO, int TH, int MAXH, int NS, int NWARP = 16>
+template <typename TI, typename TS, typename TO, int TH, int MAXH, int NS, int NWARP = 16, int CPS = 1>
 int box_fused_t(const void* in, int in_dtype, void* out, int64_t batch, int64_t rows, int64_t cols, int rr, int rc,
                 int normalize, const DevInfo& di, Workspace& ws, cudaStream_t st) {
     auto kern = sat_boxf_kernel<TI, TS, TO, TH, MAXH, NS, NWARP>;
@@ -1102,7 +1105,7 @@ int box_fused_t(const void* in, int in_dtype, void* out, int64_t batch, int64_t 
     bp.ticket = static_cast<unsigned long long*>(ws.bticket.p);
     bp.base = 0;
     const long long units = (long long)batch * bp.nb;
-    const int grid = int(std::min<long long>(units, di.sms));
+    const int grid = int(std::min<long long>(units, (long long)CPS * di.sms));
     cudaLaunchConfig_t cfg;
     std::memset(&cfg, 0, sizeof(cfg));
     cfg.gridDim = dim3(unsigned(grid));
@@ -1291,15 +1294,30 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
         const bool i32 = in_dtype == SAT_INT32 && cols % 4 == 0 && 2 * rr <= 32;
         const bool f32 = in_dtype == SAT_FLOAT32 && cols % 4 == 0 && 2 * rr <= 16;
         if (al && apart && rc <= 127 && rows <= INT32_MAX && cols <= INT32_MAX && (u8 || i32 || f32)) {
+            // uint8 with 2 rr <= 16: 32-row bands of 8 warps, ~104 KB of shared
+            // memory, two CTAs per SM (one CTA's barrier phases overlap the
+            // other's work)
+            if (u8 && 2 * rr <= 16)
+                return box_fused_t<uint8_t, uint32_t, int32_t, 32, 48, 4, 8, 2>(in, in_dtype, out, batch, rows, cols, rr,
+                                                                                 rc, 0, di, *ws, st);
             if (u8)
                 return box_fused_t<uint8_t, uint32_t, int32_t, 64, 96, 4>(in, in_dtype, out, batch, rows, cols, rr, rc, 0,
                                                                            di, *ws, st);
+            if (i32 && 2 * rr <= 16)
+                return box_fused_t<uint32_t, uint32_t, int32_t, 16, 32, 2, 8, 2>(in, in_dtype, out, batch, rows, cols,
+                                                                                  rr, rc, 0, di, *ws, st);
             if (i32)
                 return box_fused_t<uint32_t, uint32_t, int32_t, 32, 64, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
                                                                             0, di, *ws, st);
+            if (out_dtype == SAT_FLOAT32 && 2 * rr <= 8)
+                return box_fused_t<float, double, float, 16, 24, 2, 8, 2>(in, in_dtype, out, batch, rows, cols, rr,
+                                                                           rc, normalize, di, *ws, st);
             if (out_dtype == SAT_FLOAT32)
                 return box_fused_t<float, double, float, 32, 48, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
                                                                      normalize, di, *ws, st);
+            if (2 * rr <= 8)
+                return box_fused_t<float, double, double, 16, 24, 2, 8, 2>(in, in_dtype, out, batch, rows, cols, rr,
+                                                                            rc, normalize, di, *ws, st);
             return box_fused_t<float, double, double, 32, 48, 2>(in, in_dtype, out, batch, rows, cols, rr, rc,
                                                                   normalize, di, *ws, st);
         }
