@@ -110,7 +110,13 @@ typedef struct sat_options {
     int segments;        /* 1R1W band segments: 0 =
                             automatic, n >= 1 = cut every band into n column
                             segments (tests) */
-    int reserved[3];     /* must be 0 */
+    int lookback_group;  /* look-back over bands: 0 =
+                            automatic, -1 = flat (band by band), n >= 2 =
+                            hierarchical: the last band of every group of n
+                            bands also publishes the group's sums, and a walk
+                            visits its own group band by band, then one word
+                            per group above.  Same results either way. */
+    int reserved[2];     /* must be 0 */
 } sat_options;
 
 /* Fill *opt with defaults (r = 0.25, automatic tile, TMA when eligible). */
@@ -317,6 +323,9 @@ int sat_last_launch_count(void);
 int sat_last_tile_rows(void);
 /* Grid size (persistent CTAs) of the last band-kernel launch on this thread. */
 int sat_last_grid(void);
+/* Look-back group size of the last band-kernel launch on this thread (0 =
+ * flat walk; sat_options.lookback_group). */
+int sat_last_lookback_group(void);
 /* Realised r of the last SAT_1PLUSR_R1W call on this thread. */
 double sat_last_r_effective(void);
 

@@ -32,7 +32,8 @@ SAT_OK = 0
 class SatOptions(ctypes.Structure):
     _fields_ = [("r", ctypes.c_double), ("tile_rows", ctypes.c_int),
                 ("force_generic", ctypes.c_int), ("jitter", ctypes.c_int),
-                ("segments", ctypes.c_int), ("reserved", ctypes.c_int * 3)]
+                ("segments", ctypes.c_int), ("lookback_group", ctypes.c_int),
+                ("reserved", ctypes.c_int * 2)]
 
 
 class SatShardStats(ctypes.Structure):
@@ -77,6 +78,7 @@ _SIGS = {
     "sat_last_launch_count": ([], _I),
     "sat_last_tile_rows": ([], _I),
     "sat_last_grid": ([], _I),
+    "sat_last_lookback_group": ([], _I),
     "sat_last_r_effective": ([], ctypes.c_double),
     "sat_strerror": ([_I], ctypes.c_char_p),
     "sat_last_error": ([], ctypes.c_char_p),
@@ -134,7 +136,7 @@ def _check_dev(*ts):
 
 
 def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
-            jitter: int = 0, segments: int = 0) -> SatOptions:
+            jitter: int = 0, segments: int = 0, lookback_group: int = 0) -> SatOptions:
     o = SatOptions()
     _lib.sat_options_init(ctypes.byref(o))
     o.r = float(r)
@@ -142,11 +144,13 @@ def options(r: float = 0.25, tile_rows: int = 0, force_generic: bool = False,
     o.force_generic = int(bool(force_generic))
     o.jitter = int(jitter)
     o.segments = int(segments)
+    o.lookback_group = int(lookback_group)
     return o
 
 
 def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
-        force_generic: bool = False, jitter: int = 0, segments: int = 0, stream=None):
+        force_generic: bool = False, jitter: int = 0, segments: int = 0, stream=None,
+        lookback_group: int = 0):
     """SAT of a 2-D CUDA tensor (int32 wraps mod 2^32, float32/float64 IEEE).
 
     ``out`` may be ``x`` itself (in place).  ``variant`` in
@@ -160,14 +164,15 @@ def sat(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
     _check_dev(x, out)
     if out.shape != x.shape or out.dtype != x.dtype:
         raise ValueError("out must match x in shape and dtype")
-    o = options(r, tile_rows, force_generic, jitter, segments)
+    o = options(r, tile_rows, force_generic, jitter, segments, lookback_group)
     _check(_lib.sat_compute_ex(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                _dtype_code(x), VARIANTS[variant], ctypes.byref(o), _stream(stream)))
     return out
 
 
 def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: int = 0,
-                force_generic: bool = False, segments: int = 0, stream=None):
+                force_generic: bool = False, segments: int = 0, stream=None,
+                lookback_group: int = 0):
     """SATs of a (batch, rows, cols) CUDA tensor, one launch for the batch."""
     import torch
     if x.dim() != 3:
@@ -175,7 +180,7 @@ def sat_batched(x, variant: str = "1r1w", out=None, r: float = 0.25, tile_rows: 
     if out is None:
         out = torch.empty_like(x)
     _check_dev(x, out)
-    o = options(r, tile_rows, force_generic, 0, segments)
+    o = options(r, tile_rows, force_generic, 0, segments, lookback_group)
     _check(_lib.sat_compute_batched(x.data_ptr(), out.data_ptr(), x.shape[0], x.shape[1],
                                     x.shape[2], _dtype_code(x), VARIANTS[variant],
                                     ctypes.byref(o), _stream(stream)))
@@ -421,6 +426,10 @@ def last_tile_rows() -> int:
 
 def last_grid() -> int:
     return _lib.sat_last_grid()
+
+
+def last_lookback_group() -> int:
+    return _lib.sat_last_lookback_group()
 
 
 def last_r_effective() -> float:

@@ -37,6 +37,7 @@ thread_local std::string t_err;
 thread_local int t_launches = 0;
 thread_local int t_th = 0;
 thread_local int t_grid = 0;
+thread_local int t_hg = 0;
 thread_local double t_r = 0.0;
 thread_local unsigned long long* t_trace = nullptr;
 thread_local bool t_capture = false;   // the current call's stream is being captured
@@ -531,6 +532,7 @@ struct Job {
     bool tma;
     int jitter;
     int segments;     // sat_options.segments: 0 = automatic band segments
+    int hg;           // sat_options.lookback_group: 0 = automatic, -1 = flat, n >= 2 groups of n bands
     const DevInfo* di;
     Workspace* ws;
     cudaStream_t st;
@@ -658,9 +660,33 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         }
     }
     Workspace& ws = *j.ws;
+    // hierarchical look-back: group words live after
+    // the band descriptors in the same buffer (cleared with them)
+    p.hg = 0;
+    p.ngroups = 0;
+    if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW && p.region == REG_ALL) {
+        // automatic: groups of 4 bands for one-wave 1R1W launches of bands
+        // <= 64 rows (the one-wave TH-32 and wide TH-64 configurations, whose
+        // control groups walk one band per round trip): 4096^2 45.1 -> 42.0 us,
+        // 3072^2 34.8 -> 32.8, 5120^2 75.8 -> 72.7, 6144^2 79.9 -> 77.8,
+        // 4096^2 float64 112 -> 107; flat at TH 128 (16384^2 0.408 vs
+        // 0.410-0.419 ms for groups of 4-16) and for many waves (65536^2,
+        // 8192^2, 12288^2: 0.5-2 % slower); profiles/r02_hier.txt
+        int hg = j.hg;
+        if (hg == 0) {
+            const int slots = j.di->sms * ctas_per_sm(j.dtype, j.th);
+            hg = (mode == MODE_SAT && j.th <= 64 && p.total_units <= slots) ? 4 : -1;
+        }
+        if (hg >= 2 && hg < p.nb) {
+            p.hg = hg;
+            p.ngroups = (p.nb + hg - 1) / hg;
+        }
+    }
+    size_t desc_words = 0;
     if (p.top_src == TOP_LOOKBACK && mode != MODE_ROW) {
-        const size_t need = size_t(p.total_bands) * size_t(p.nc) * tw * sizeof(uint64_t) * (esize(j.dtype) / 4);
-        SAT_TRY(ensure(ws.desc, need, true));
+        desc_words = size_t(p.total_bands) * size_t(p.nc) * tw * (esize(j.dtype) / 4);
+        const size_t gwords = size_t(j.batch) * size_t(p.ngroups) * size_t(p.nc) * tw * (esize(j.dtype) / 4);
+        SAT_TRY(ensure(ws.desc, (desc_words + gwords) * sizeof(uint64_t), true));
     }
     SAT_TRY(ensure(ws.ticket, 4 * sizeof(unsigned long long), true));
     if (p.nseg > 1)
@@ -684,6 +710,8 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
         ws.next_base = 0;
     }
     p.desc = static_cast<uint64_t*>(ws.desc.p);
+    p.gdesc = p.hg > 0 ? p.desc + desc_words : nullptr;
+    t_hg = p.hg;
     p.Lseg = static_cast<uint64_t*>(ws.lseg.p);
     p.ticket = static_cast<unsigned long long*>(ws.ticket.p);
     p.base = ws.next_base;
@@ -888,6 +916,8 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
         return fail(SAT_ERR_INVALID, "tile_rows must be 0, 16, 32, 64 or 128");
     if (!(o.r >= 0.0 && o.r <= 1.0)) return fail(SAT_ERR_INVALID, "r must be in [0, 1]");
     if (o.segments < 0) return fail(SAT_ERR_INVALID, "segments must be >= 0");
+    if (o.lookback_group < -1 || o.lookback_group == 1)
+        return fail(SAT_ERR_INVALID, "lookback_group must be -1, 0 or >= 2");
     if (rows == 0 || cols == 0 || batch == 0) return SAT_OK;
     int dev;
     DevInfo di;
@@ -901,6 +931,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     j.tma = !o.force_generic && tma_ok(in, out, cols, in_dtype);
     j.jitter = o.jitter;
     j.segments = o.segments;
+    j.hg = o.lookback_group;
     j.di = &di;
     j.ws = ws;
     j.st = st;
@@ -1659,6 +1690,7 @@ int sat_release_workspace(void* stream) {
 int sat_last_launch_count(void) { return t_launches; }
 int sat_last_tile_rows(void) { return t_th; }
 int sat_last_grid(void) { return t_grid; }
+int sat_last_lookback_group(void) { return t_hg; }
 double sat_last_r_effective(void) { return t_r; }
 
 const char* sat_strerror(int status) {

@@ -766,16 +766,21 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                     } else {
                         // decoupled look-back over bands band-1, band-2, ...,
                         // LBW descriptor rows per round trip: adds the SAT row
-                        // above this band to top
-                        uint32_t pend = (1u << CPL) - 1u;
+                        // above this band to top.  Hierarchical (p.hg > 0,
+                        // DESIGN.md Sec. 4.13): band by band only down to the
+                        // first band g0 of this band's group, then one group
+                        // word per group above (phase 2 below)
+                        constexpr uint32_t kAll = (1u << CPL) - 1u;
+                        uint32_t pend = kAll;
+                        const int g0 = p.hg > 0 ? band - band % p.hg : 0;
                         int kb = band - 1;
                         SpinGuard guard(0x80000000u | uint32_t(J), uint32_t(gb));
-                        while (pend) {
+                        while (pend && kb >= g0) {
                             uint64_t wv[LBW][NW];
 #pragma unroll
                             for (int q = 0; q < LBW; ++q) {
                                 const int b2 = kb - q;
-                                if (b2 >= 0) {
+                                if (b2 >= g0) {
                                     load_words<NW>(p.desc + ((int64_t(gb) - (band - b2)) * desc_w + c0) * NWE, wv[q]);
                                 } else {
 #pragma unroll
@@ -787,6 +792,7 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             for (int q = 0; q < LBW; ++q) {
                                 if (!pend || stalled) break;
                                 const int b2 = kb - q;
+                                if (b2 < g0) break;
                                 if (p.region == REG_C && b2 + J < p.tA) {
                                     // tile (b2, J) belongs to (A): its final SAT row is in `out`
                                     const int64_t row = int64_t(b2 + 1) * TH - 1;
@@ -827,12 +833,78 @@ sat_band_kernel(const __grid_constant__ CUtensorMap tm_in,
                             if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
                             else kb -= LBW;
                         }
+                        if (p.hg > 0 && pend) {
+                            // phase 2: every band g0 .. band-1 was an aggregate
+                            const int grpi = band / p.hg;
+                            const int64_t gimg = int64_t(img) * p.ngroups;
+                            // the group's last band publishes the group aggregate
+                            // (sum of its bands' aggregates) before walking on, so
+                            // the bands below never wait on a chain of inclusives
+                            if (publish && band == g0 + p.hg - 1 && pend == kAll) {
+                                T ga[CPL];
+#pragma unroll
+                                for (int i = 0; i < CPL; ++i) ga[i] = top[i] + agg[i];
+                                publish_words<T, CPL>(p.gdesc + ((gimg + grpi) * desc_w + c0) * NWE, tagbase | 1u, ga);
+                            }
+                            // group 0's word always ends inclusive (its walk meets
+                            // band 0), so the walk stops at kg >= 0
+                            int kg = grpi - 1;
+                            while (pend) {
+                                uint64_t wv[LBW][NW];
+#pragma unroll
+                                for (int q = 0; q < LBW; ++q) {
+                                    const int g2 = kg - q;
+                                    if (g2 >= 0) {
+                                        load_words<NW>(p.gdesc + ((gimg + g2) * desc_w + c0) * NWE, wv[q]);
+                                    } else {
+#pragma unroll
+                                        for (int i = 0; i < NW; ++i) wv[q][i] = 0;
+                                    }
+                                }
+                                bool stalled = false;
+#pragma unroll
+                                for (int q = 0; q < LBW; ++q) {
+                                    if (!pend || stalled) break;
+                                    const int g2 = kg - q;
+                                    const uint32_t tk = band_tag(kbase, gb - band + g2 * p.hg + p.hg - 1);
+                                    bool ready = true;
+#pragma unroll
+                                    for (int i = 0; i < NW; ++i) {
+                                        const uint32_t t = uint32_t(wv[q][i] >> 32);
+                                        ready = ready && ((t & ~3u) == tk) && (t & 3u);
+                                    }
+#pragma unroll
+                                    for (int i = 0; i < CPL; ++i)
+#pragma unroll
+                                        for (int k = 1; k < NWE; ++k)
+                                            ready = ready && (uint32_t(wv[q][i * NWE + k] >> 32) == uint32_t(wv[q][i * NWE] >> 32));
+                                    if (!ready) { stalled = true; kg = g2; break; }
+#pragma unroll
+                                    for (int i = 0; i < CPL; ++i) {
+                                        if ((pend >> i) & 1u) {
+                                            uint32_t w[NWE];
+#pragma unroll
+                                            for (int k = 0; k < NWE; ++k) w[k] = uint32_t(wv[q][i * NWE + k]);
+                                            top[i] += from_words<T>(w);
+                                            if ((uint32_t(wv[q][i * NWE] >> 32) & 3u) == 2u) pend &= ~(1u << i);
+                                        }
+                                    }
+                                    ++hops;
+                                }
+                                if (stalled) { __nanosleep(32); guard.tick(); ++polls; }
+                                else kg -= LBW;
+                            }
+                        }
                     }
                     if (publish) {
                         T inc[CPL];
 #pragma unroll
                         for (int i = 0; i < CPL; ++i) inc[i] = agg[i] + top[i];
                         publish_words<T, CPL>(my, tagbase | 2u, inc);
+                        // the group's last band: its inclusive is the group's
+                        if (p.hg > 0 && (band + 1) % p.hg == 0)
+                            publish_words<T, CPL>(p.gdesc + ((int64_t(img) * p.ngroups + band / p.hg) * desc_w + c0) * NWE,
+                                                  tagbase | 2u, inc);
                     }
                     if constexpr (kDebug) {
                         if (traced && cw == grp * NS && lane == 0)

@@ -89,6 +89,13 @@ struct BandParams {
     // predecessors of a unit -- the same segment of the band above and the
     // previous segment of the same band -- hold earlier tickets.
     const int2* order;
+    // Hierarchical look-back: hg > 0 groups the bands
+    // of an image by hg; the last band of a group also publishes the group's
+    // aggregate / inclusive words in gdesc[img * ngroups + group][column], and
+    // a walk visits its own group band by band, then one word per group above.
+    int hg;                    // 0 = flat look-back
+    int ngroups;               // groups per image = ceil(nb / hg)
+    uint64_t* gdesc;           // [batch * ngroups][nc*TW] group descriptor words
     unsigned long long* trace; // debug builds (SAT_DEBUG): [total_bands*nc][8] event times (ns), nullable
     unsigned int* diag;        // debug builds: host-mapped progress marks, nullable
 };

@@ -6,8 +6,8 @@ rounds to cancel clock drift.
 
 python tools/ab_sat.py "16384x16384,65536x65536" "128:0,64:0" [reps] [rounds] [dtype]
 
-A config is th:seg[:x], x = an experiment selector passed in sat_options.reserved[0]
-(0 in release builds).
+A config is th:seg[:hg], hg = sat_options.lookback_group (0 automatic, -1 flat,
+n >= 2 groups of n bands).
 """
 import ctypes
 import os
@@ -30,9 +30,8 @@ dtype = sys.argv[5] if len(sys.argv) > 5 else "int32"
 dist = "u32" if dtype == "int32" else "unit"
 
 def call(x, y, c):
-    """c = (tile_rows, segments, experiment selector in sat_options.reserved[0])"""
-    o = libsat.options(tile_rows=c[0], segments=c[1])
-    o.reserved[0] = c[2]
+    """c = (tile_rows, segments, lookback_group)"""
+    o = libsat.options(tile_rows=c[0], segments=c[1], lookback_group=c[2])
     if x.dim() == 3:
         libsat._check(libsat._lib.sat_compute_batched(x.data_ptr(), y.data_ptr(), x.shape[0], x.shape[1], x.shape[2],
                                                       libsat._dtype_code(x), 2, ctypes.byref(o), None))
