@@ -317,6 +317,10 @@ int sat_release_workspace(void *stream);
  * 0 restores the default) so the tag-exhaustion paths run. */
 int sat_debug_set_tag_space(uint64_t space);
 
+/* Tests / tuning only: output rows per unit of the column-walk box filter
+ * (DESIGN.md Sec. 4.12); 0 restores the automatic choice. */
+int sat_debug_set_box_rows(int rows);
+
 /* Number of kernels launched by the last successful call on this thread. */
 int sat_last_launch_count(void);
 /* Band height used by the last 1R1W-family call on this thread. */

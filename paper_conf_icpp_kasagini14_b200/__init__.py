@@ -72,6 +72,7 @@ _SIGS = {
     "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
     "sat_release_workspace": ([_P], _I),
     "sat_debug_set_tag_space": ([ctypes.c_uint64], _I),
+    "sat_debug_set_box_rows": ([ctypes.c_int], _I),
     "sat_debug_trace": ([_P], _I),
     "sat_debug_diag_enable": ([], _I),
     "sat_debug_diag_dump": ([], _I),
@@ -409,6 +410,11 @@ def ipc_close(ptr: int) -> None:
 def release_workspace(stream=None) -> None:
     """Free libsat's workspace of ``stream`` (sat_release_workspace)."""
     _check(_lib.sat_release_workspace(_stream(stream)))
+
+
+def set_box_rows(rows: int) -> None:
+    """Tests / tuning only: output rows per column-walk box-filter unit (0 = automatic)."""
+    _check(_lib.sat_debug_set_box_rows(int(rows)))
 
 
 def set_tag_space(space: int) -> None:

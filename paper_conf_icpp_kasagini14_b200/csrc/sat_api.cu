@@ -27,6 +27,7 @@
 #include "sat_paper.cuh"
 #include "sat_box.cuh"
 #include "sat_boxf.cuh"
+#include "sat_boxw.cuh"
 #include "sat_xchg.cuh"
 
 using namespace sat;
@@ -113,6 +114,7 @@ struct Buf {
 // look-back tags are 30 bits (band_tag); sat_debug_set_tag_space (tests only)
 // shrinks the space so the reset paths run
 std::atomic<unsigned long long> g_tag_space{1ull << 30};
+std::atomic<int> g_box_rb{0};        // sat_debug_set_box_rows (0 = automatic)
 unsigned long long tag_space() { return g_tag_space.load(std::memory_order_relaxed); }
 
 struct Workspace {
@@ -1155,6 +1157,71 @@ int box_fused_t(const void* in, int in_dtype, void* out, int64_t batch, int64_t 
     return SAT_OK;
 }
 
+// Column-walk box filter (sat_boxw.cuh): one launch, one warp per unit of
+// 128 columns x rb output rows, the SAT evaluated on the fly.
+template <typename TI, typename TS, typename TO>
+int box_walk_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols, int rr, int rc, int normalize,
+               cudaStream_t st) {
+    constexpr int NWARP = 4;
+    constexpr int PF = sizeof(TI) == 1 ? 8 : 4;   // rows in flight per warp (cp.async ring)
+    auto kern = sat_boxw_kernel<TI, TS, TO, NWARP, PF>;
+    const size_t smem = size_t(NWARP) * boxw_warp_smem<TI, TS, PF>(rr);
+    static KernelSetup setup;
+    int dev = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    if (dev < 0 || dev >= kMaxDev) return fail(SAT_ERR_CUDA, "device ordinal out of range");
+    std::call_once(setup.once[dev], [&] {
+        setup.err[dev] = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    });
+    if (setup.err[dev] != cudaSuccess)
+        return fail(SAT_ERR_CUDA, std::string("box kernel set-up: ") + cudaGetErrorString(setup.err[dev]));
+    if (smem > 200 * 1024) return fail(SAT_ERR_UNSUPPORTED, "box filter: radius too large for the walk kernel");
+    BoxWParams bp;
+    bp.in = in; bp.out = out; bp.rows = int(rows); bp.cols = int(cols); bp.batch = int(batch);
+    bp.rr = rr; bp.rc = rc; bp.normalize = normalize;
+    bp.nc = int((cols + TW - 1) / TW);
+    bp.rb = g_box_rb.load(std::memory_order_relaxed);
+    if (bp.rb <= 0) {
+        // one wave: as many row blocks per strip as the resident warps allow
+        // (units = batch x strips x row blocks <= warp slots), so every warp
+        // runs from the start and the 2 rr-row warm-up is paid as few times
+        // as possible; blocks of >= 32 rows.  32 x 1080x1920 uint8 r = 4:
+        // 0.119 ms (6 blocks of 180 rows) vs 0.125 (64-row blocks, two
+        // waves) and 0.141 (120-row blocks, 1.04 waves); tools/box_rows.py
+        int per_sm = 0;
+        CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NWARP * 32, smem));
+        int sms = 0;
+        CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        const long long slots = (long long)std::max(per_sm, 1) * NWARP * sms;
+        const long long strips = batch * (long long)bp.nc;
+        const long long nrb = std::max(1LL, slots / strips);
+        bp.rb = int(std::max<long long>(32, (rows + nrb - 1) / nrb));
+    }
+    bp.nrb = int((rows + bp.rb - 1) / bp.rb);
+    bp.units = (long long)batch * bp.nrb * bp.nc;
+    const uintptr_t ia = reinterpret_cast<uintptr_t>(in);
+    bp.vec = 1;
+    if (!(sizeof(TI) == 1 ? (cols % 8 == 0 && (ia & 7) == 0) : (cols % 4 == 0 && (ia & 15) == 0)))
+        return fail(SAT_ERR_INVALID, "box walk: misaligned rows");
+    const long long grid = (bp.units + NWARP - 1) / NWARP;
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(unsigned(grid));
+    cfg.blockDim = dim3(NWARP * 32);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, kern, bp));
+    CUDA_TRY(cudaGetLastError());
+    t_launches = 1;
+    t_grid = int(std::min<long long>(grid, INT32_MAX));
+    return SAT_OK;
+}
+
 }  // namespace
 
 // ====================================================================== C ABI
@@ -1315,6 +1382,18 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
+    // Column walk (one launch, one warp per 128-column strip of a row block,
+    // sat_boxw.cuh) when out does not alias in, rc <= 63 and the D ring fits:
+    // 32 x 1080x1920 uint8 r = 4: see DESIGN.md Sec. 4.12
+    const bool walk_al = in_dtype == SAT_UINT8 ? (cols % 8 == 0 && (reinterpret_cast<uintptr_t>(in) & 7) == 0)
+                                               : (cols % 4 == 0 && (reinterpret_cast<uintptr_t>(in) & 15) == 0);
+    if (walk_al && in != out && rc <= 63 && rr <= 16 && rows <= INT32_MAX && cols <= INT32_MAX &&
+        batch * rows <= INT32_MAX) {
+        if (in_dtype == SAT_UINT8 && rr <= 8)
+            return box_walk_t<uint8_t, uint32_t, int32_t>(in, out, batch, rows, cols, rr, rc, 0, st);
+        if (in_dtype == SAT_INT32 && rr <= 8)
+            return box_walk_t<uint32_t, uint32_t, int32_t>(in, out, batch, rows, cols, rr, rc, 0, st);
+    }
     // Fused (one launch, the SAT never leaves the chip, sat_boxf.cuh) when the
     // input is TMA-addressable, out does not alias it (a band's halo rows are
     // another band's output rows), the halo fits the band buffer and rc < 128.
@@ -1653,6 +1732,12 @@ int sat_debug_diag_dump(void) {
 int sat_debug_trace(void* dev_buf) {
     if (!kDebug) return fail(SAT_ERR_UNSUPPORTED, "event traces need a debug build (SAT_DEBUG=1)");
     t_trace = static_cast<unsigned long long*>(dev_buf);
+    return SAT_OK;
+}
+
+int sat_debug_set_box_rows(int rows) {
+    if (rows < 0 || rows > (1 << 20)) return fail(SAT_ERR_INVALID, "box rows must be in [0, 2^20]");
+    g_box_rb.store(rows, std::memory_order_relaxed);
     return SAT_OK;
 }
 

@@ -250,3 +250,24 @@ def test_box_huge_radius_clamped(libsat):
     for b in range(2):
         assert (y[b] == np.int64(a[b].astype(np.int64).sum()).astype(np.int32)).all()
         assert np.array_equal(y[b], oracle.box_filter(a[b].astype(np.int32), 300, 500))
+
+
+@pytest.mark.parametrize("rb", [1, 5, 17, 64, 200])
+def test_box_walk_row_blocks(libsat, rb):
+    """Column-walk box filter with forced rows per unit:
+    every unit re-runs the 2 rr-row warm-up of its window, so unit borders
+    anywhere (1 row, ragged, taller than the image) give the same sums."""
+    try:
+        libsat.set_box_rows(rb)
+        a = u8img(301, 520, seed=rb, batch=2)
+        for rr, rc in ((0, 0), (4, 4), (8, 63), (3, 17)):
+            y = libsat.box_filter(dev(a), rr, rc).cpu().numpy()
+            assert libsat.last_launch_count() == 1
+            for b in range(2):
+                assert np.array_equal(y[b], oracle.box_filter(a[b].astype(np.int32), rr, rc)), (rr, rc, b)
+        ai = make_np(150, 264, "int32", "u32", seed=rb, batch=2)
+        y = libsat.box_filter(dev(ai), 6, 40).cpu().numpy()
+        for b in range(2):
+            assert np.array_equal(y[b], oracle.box_filter(ai[b], 6, 40))
+    finally:
+        libsat.set_box_rows(0)

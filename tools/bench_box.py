@@ -65,12 +65,16 @@ def main():
         ("widen u8->i32 1R1W", lambda: libsat.sat_widening(u8, torch.int32, out=i32), 5 * px, px),
         ("widen f32->f64 1R1W", lambda: libsat.sat_widening(f32, torch.float64, out=f64), 12 * px, px),
         ("sat i32 1R1W (same images)", lambda: libsat.sat_batched(i32, out=box), 8 * px, px),
-        (f"box filter u8 r={r} fused (1 B in x (1 + 2r/32) + 4 B out)", lambda: libsat.box_filter(u8, r, r, out=box),
-         int((1 + 2 * r / 32) * px) + 4 * px, px),
-        (f"box filter f32->f32 r={r} fused (float64 SAT on chip)", lambda: libsat.box_filter(f32, r, r, out=f32o),
+        # column walk (sat_boxw.cuh, rc <= 63): input (1 + 2r/64) x eb_in (row-block warm-up), 4 B out
+        (f"box filter u8 r={r} walk (1 B in x (1 + 2r/64) + 4 B out)", lambda: libsat.box_filter(u8, r, r, out=box),
+         int((1 + 2 * r / 64) * px) + 4 * px, px),
+        (f"box filter f32->f32 r={r} fused band (float64 SAT on chip)", lambda: libsat.box_filter(f32, r, r, out=f32o),
          int(4 * (1 + 2 * r / 16) * px) + 4 * px, px),
-        (f"box filter int32 r={r} fused (4 B in x (1 + 2r/16) + 4 B out)", lambda: libsat.box_filter(i32, r, r, out=box),
-         int(4 * (1 + 2 * r / 16) * px) + 4 * px, px),
+        (f"box filter int32 r={r} walk (4 B in x (1 + 2r/64) + 4 B out)", lambda: libsat.box_filter(i32, r, r, out=box),
+         int(4 * (1 + 2 * r / 64) * px) + 4 * px, px),
+        # band kernel with the SAT on chip (sat_boxf.cuh) for 64 <= rc < 128
+        (f"box filter u8 rr={r} rc=100 fused band (1 B in x (1 + 2r/32) + 4 B out)",
+         lambda: libsat.box_filter(u8, r, 100, out=box), int((1 + 2 * r / 32) * px) + 4 * px, px),
         ("rect sums (1M queries)", lambda: libsat.rect_sums(i32, rects, out=qout), None, 1 << 20),
     ]
     for name, fn, nbytes, units in cases:
