@@ -118,3 +118,38 @@ def test_automatic_choice(libsat):
     a = gen(3000, 2000, "int32", seed=9)
     check(libsat.sat(dev(a), lookback_group=-1), oracle.sat(a), "int32")
     assert libsat.last_lookback_group() == 0
+
+
+def test_group_words_across_tag_resets(libsat):
+    """With a tiny tag space the descriptors (group words included: they live
+    in the same buffer) are cleared whenever the tags run out; group words of
+    earlier calls must never be taken for this call's."""
+    libsat.set_tag_space(300000)
+    try:
+        for k in range(30):
+            shape = (1500 + 61 * k, 700 + 13 * k)
+            a = gen(*shape, "int32", seed=300 + k)
+            check(libsat.sat(dev(a), tile_rows=32, lookback_group=2 + k % 4), oracle.sat(a), "int32")
+    finally:
+        libsat.set_tag_space(0)
+
+
+def test_graph_replay_hierarchical(libsat):
+    """A captured one-wave launch (automatic groups of 4) replayed on fresh
+    inputs, with the device-side ticket base."""
+    n, m = 4096, 4096
+    x = dev(gen(n, m, "float32", seed=1))
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        y = libsat.sat(x)
+    s.synchronize()
+    assert libsat.last_lookback_group() == 4
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        libsat.sat(x, out=y)
+    for it in range(3):
+        host = gen(n, m, "float32", seed=50 + it)
+        x.copy_(dev(host))
+        g.replay()
+        torch.cuda.synchronize()
+        check(y, oracle.sat(host), "float32")
