@@ -1200,7 +1200,6 @@ int box_walk_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t c
     bp.nrb = int((rows + bp.rb - 1) / bp.rb);
     bp.units = (long long)batch * bp.nrb * bp.nc;
     const uintptr_t ia = reinterpret_cast<uintptr_t>(in);
-    bp.vec = 1;
     if (!(sizeof(TI) == 1 ? (cols % 8 == 0 && (ia & 7) == 0) : (cols % 4 == 0 && (ia & 15) == 0)))
         return fail(SAT_ERR_INVALID, "box walk: misaligned rows");
     const long long grid = (bp.units + NWARP - 1) / NWARP;

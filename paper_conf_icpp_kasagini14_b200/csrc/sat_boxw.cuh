@@ -46,7 +46,6 @@ struct BoxWParams {
     int nrb;               // row blocks per image
     int nc;                // 128-column strips per image
     long long units;       // batch * nrb * nc
-    int vec;               // rows are 8-B (uint8) / 16-B aligned (host-checked; always 1)
 };
 
 // shared bytes per warp: raw-row ring (PF rows x 256 span columns of TI) +
@@ -139,7 +138,8 @@ __global__ void __launch_bounds__(NWARP * 32) sat_boxw_kernel(const BoxWParams b
     const int c0 = c * 128;
     const int s0 = c0 - 64 + 8 * lane;
     // lane groups are whole 4/8-column groups inside or outside the image
-    // (host: cols % 8 == 0 for uint8, % 4 == 0 for 4-byte types)
+    // (host: cols % 8 == 0 and 8-B aligned rows for uint8, cols % 4 == 0 and
+    // 16-B aligned rows for 4-byte types)
     const bool ok0 = s0 >= 0 && s0 + (sizeof(TI) == 1 ? 8 : 4) <= bp.cols;
     const bool ok1 = s0 + 4 >= 0 && s0 + 8 <= bp.cols;
     const TI* src = reinterpret_cast<const TI*>(bp.in) + (int64_t(img) * bp.rows + kstart) * bp.cols
