@@ -12,6 +12,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <vector>
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t c) {
@@ -49,6 +50,14 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 template <int N>
 __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory"); }
 
+// optional per-unit trace (argv[2] == "t"): [unit][2] = start / end globaltimer
+__device__ unsigned long long* d_tr = nullptr;
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
 // MODE 0: consumers LDS + STG.cs; MODE 1: producer TMA-stores each landed slot (pure DMA)
 template <int H, int C, int S, int W, int MODE, bool STRIP = false>
 __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant__ CUtensorMap tin,
@@ -75,6 +84,11 @@ __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant_
         const int unit = *s_unit;
         __syncthreads();
         if (unit >= units) break;
+        if (d_tr && threadIdx.x == 0) {
+            unsigned int smid;
+            asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+            d_tr[2 * unit] = (gtimer() & 0xFFFFFFFFFFFFull) | (uint64_t(smid) << 56);
+        }
         // band-major: unit = (band, chunk range), chunk k at (cols (k0+k)*C, rows band*H)
         // strip-major: unit = (row segment, strip), chunk k at (cols strip*C, rows (k0+k)*H)
         const int spr = n / (H * U);            // row segments per strip (STRIP)
@@ -141,6 +155,7 @@ __global__ void __launch_bounds__((W + 1) * 32) band_copy(const __grid_constant_
                 }
             }
         }
+        if (d_tr && MODE == 0 && warp == 0 && lane == 0) d_tr[2 * unit + 1] = gtimer();
         g += U;
     }
     if (MODE == 1 && warp == W && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
@@ -244,6 +259,24 @@ int main(int argc, char** argv) {
         float avg, best = timed(launch, &f, 10, &avg);
         printf("flat       grid=%4d x 512  best %.4f ms %.0f GB/s avg %.4f ms %.0f GB/s\n", f.grid, best,
                2.0 * n * n * 4 / best / 1e6, avg, 2.0 * n * n * 4 / avg / 1e6);
+    }
+    if (argc > 2 && argv[2][0] == 't') {
+        // per-band start / end times of the band-kernel geometry copy (one
+        // wave of whole 128-row bands): do lower bands finish later?
+        unsigned long long* tr;
+        const int units = n / 128;
+        cudaMalloc(&tr, size_t(units) * 16);
+        cudaMemcpyToSymbol(d_tr, &tr, sizeof(tr));
+        run<128, 128, 3, 16, 0>(n, in, out, n / 128, 1, "band128t");
+        std::vector<unsigned long long> h(size_t(units) * 2);
+        cudaMemcpy(h.data(), tr, h.size() * 8, cudaMemcpyDeviceToHost);
+        unsigned long long t0 = ~0ull;
+        const unsigned long long M = 0xFFFFFFFFFFFFull;
+        for (int u = 0; u < units; ++u) t0 = std::min(t0, h[2 * u] & M);
+        printf("band smid end_us (last timed launch)\n");
+        for (int u = 0; u < units; ++u)
+            printf("T %d %d %.1f\n", u, int(h[2 * u] >> 56), ((h[2 * u + 1] & M) - t0) / 1e3);
+        return 0;
     }
     if (argc > 2 && argv[2][0] == 's') {
         // small matrices (one wave of bands, argv[2] = "s"): ring depth / box
