@@ -1,6 +1,6 @@
 """Record per-(band, chunk) look-back event times of one 1R1W launch.
 
-python tools/trace_lookback.py rows cols tile_rows out.npz [segments] [batch] [xcfg]
+python tools/trace_lookback.py rows cols tile_rows out.npz [segments] [batch] [lookback_group]
 """
 import os
 import sys
@@ -18,13 +18,12 @@ seg = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 batch = (int(sys.argv[6]) or None) if len(sys.argv) > 6 else None
 x = make_torch(rows, cols, "int32", "u32", seed=1, device="cuda", batch=batch)
 y = torch.empty_like(x)
-xcfg = int(sys.argv[7]) if len(sys.argv) > 7 else 0     # sat_options.reserved[0] (experiments)
+hg = int(sys.argv[7]) if len(sys.argv) > 7 else 0       # sat_options.lookback_group
 
 
 def run():
     import ctypes
-    o = libsat.options(tile_rows=th, segments=seg)
-    o.reserved[0] = xcfg
+    o = libsat.options(tile_rows=th, segments=seg, lookback_group=hg)
     if batch is None:
         libsat._check(libsat._lib.sat_compute_ex(x.data_ptr(), y.data_ptr(), rows, cols, libsat._dtype_code(x), 2,
                                                  ctypes.byref(o), None))
