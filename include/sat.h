@@ -168,14 +168,22 @@ int sat_compute_widening(const void *in, int in_dtype, void *out, int dtype,
 
 /* Box filter (the SAT's use, "the sum of any rectangular area
  * in O(1)"): out[b][i][j] = sum of in[b][k][l] over
- * |k - i| <= rr, |l - j| <= rc, clipped to the image.  Computed as a widening
- * 1R1W SAT into a library workspace (uint32 sums for SAT_UINT8/SAT_INT32
- * input, float64 sums for SAT_FLOAT32/SAT_FLOAT64 input) followed by one
- * kernel doing four SAT reads per output element.  out_dtype: SAT_INT32 for
+ * |k - i| <= rr, |l - j| <= rc, clipped to the image; the four-corner SAT
+ * formula with uint32 sums for SAT_UINT8/SAT_INT32 input and float64 sums for
+ * SAT_FLOAT32/SAT_FLOAT64 input.  One launch, the SAT never in HBM, when out
+ * does not alias in: integer input with rr <= 8, rc <= 63
+ * and 8-B (uint8, cols % 8 == 0) / 16-B (int32, cols % 4 == 0) aligned rows
+ * takes the column-walk kernel (row prefix sums differenced, a running
+ * vertical window sum); other TMA-addressable cases with rc <= 127 and
+ * 2 rr <= 32 (uint8/int32) or 16 (float32) the band kernel with the local SAT
+ * in shared memory.  Otherwise (in place, larger radii, float64 input,
+ * unaligned rows) a widening 1R1W SAT goes to a library workspace and a second
+ * kernel does four SAT reads per output element.  out_dtype: SAT_INT32 for
  * integer input (sums mod 2^32), SAT_FLOAT32 or SAT_FLOAT64 for float input.
  * normalize != 0 divides by the clipped window's element count (box mean;
- * float input only).  rr, rc >= 0; batch <= 65535.  Bytes moved per pixel:
- * in + 2 x sum (SAT write + read) + out. */
+ * float input only).  rr, rc >= 0 (radii beyond the image are clamped);
+ * batch <= 65535.  Bytes moved per pixel: in x (1 + halo rows) + out for the
+ * one-launch paths, in + 2 x sum + out for the two-pass path. */
 int sat_box_filter(const void *in, int in_dtype, void *out, int out_dtype,
                    int64_t batch, int64_t rows, int64_t cols, int rr, int rc,
                    int normalize, void *stream);
