@@ -277,8 +277,10 @@ def main():
                     help="N>1 row strips: the last rank's share (it skips the totals pass)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N>1 process group (gloo: host-memory exchange, for multi-process tests on one GPU)")
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
-                    help="N>1 row strips: NCCL all-gather, or the fused peer exchange (IPC mailboxes)")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "libsat-nccl", "fused"],
+                    help="N>1 row strips: NCCL all-gather via torch.distributed (with the step breakdown), "
+                         "the C-ABI call with libsat's own NCCL communicator (sat_compute_sharded_nccl), "
+                         "or the fused peer exchange (IPC mailboxes)")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
@@ -352,6 +354,20 @@ def main():
             if ev:
                 ev[0].record(stream)
             xchg.sat(x, out=y)
+            if ev:
+                ev[1].record(stream)
+            launches[0] += libsat.last_launch_count()
+    elif sharded and args.exchange == "libsat-nccl":
+        # one C-ABI call per step: column totals, ncclAllGather on libsat's
+        # communicator, seeded SAT (the events bracket the whole call)
+        uid = [libsat.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        ncomm = libsat.NcclComm(uid[0], rank, world)
+
+        def step(ev=None):
+            if ev:
+                ev[0].record(stream)
+            libsat.sat_sharded_nccl(x, ncomm, variant=variant, out=y)
             if ev:
                 ev[1].record(stream)
             launches[0] += libsat.last_launch_count()

@@ -288,6 +288,33 @@ int sat_compute_sharded(const void *in_strip, void *out_strip, int64_t strip_row
                         void *stream, sat_shard_stats *stats);
 size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype);
 
+/* As sat_compute_sharded with a variant: SAT_1R1W (the seeded band kernel) or
+ * SAT_2R2W (the seed enters the column pass's first row; 2 x the strip bytes
+ * in stats).  Other variants: SAT_ERR_UNSUPPORTED (their carry passes take no
+ * seed). */
+int sat_compute_sharded_ex(const void *in_strip, void *out_strip, int64_t strip_rows,
+                           int64_t cols, int dtype, int variant, int rank, int nranks,
+                           sat_allgather_fn allgather, void *comm_ctx, void *workspace,
+                           void *stream, sat_shard_stats *stats);
+
+/* In-library NCCL for the sharded mode (north star (3): the all-gather of the
+ * strips' column totals over NVLink / NVSwitch).  libnccl.so.2 is loaded on
+ * first use (dlopen; a copy already in the process, e.g. PyTorch's, is
+ * shared); without it these return SAT_ERR_UNSUPPORTED.
+ * sat_nccl_unique_id: 128 bytes for rank 0 to share out of band.
+ * sat_nccl_comm_create: this process's rank of nranks on the current device
+ *   (collective: every rank calls it with the same id); *comm is an opaque
+ *   ncclComm_t, freed by sat_nccl_comm_destroy.
+ * sat_compute_sharded_nccl: sat_compute_sharded_ex with rank / nranks taken
+ *   from the communicator and the all-gather done by ncclAllGather on
+ *   `stream` (NCCL errors: SAT_ERR_COMM). */
+int sat_nccl_unique_id(void *id128);
+int sat_nccl_comm_create(void **comm, const void *id128, int rank, int nranks);
+int sat_nccl_comm_destroy(void *comm);
+int sat_compute_sharded_nccl(const void *in_strip, void *out_strip, int64_t strip_rows,
+                             int64_t cols, int dtype, int variant, void *comm,
+                             void *workspace, void *stream, sat_shard_stats *stats);
+
 /* End to end from HOST memory: copies in_host (rows*cols elements) to the
  * device, computes the SAT with `variant`, copies it back to out_host, and
  * synchronises `stream` before returning.  Pinned host buffers overlap the

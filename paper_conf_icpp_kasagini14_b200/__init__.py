@@ -69,6 +69,12 @@ _SIGS = {
     "sat_compute_sharded": ([_P, _P, _I64, _I64, _I, _I, _I, ALLGATHER_FN, _P, _P, _P,
                              ctypes.POINTER(SatShardStats)], _I),
     "sat_sharded_workspace_bytes": ([_I64, _I, _I], ctypes.c_size_t),
+    "sat_compute_sharded_ex": ([_P, _P, _I64, _I64, _I, _I, _I, _I, ALLGATHER_FN, _P, _P, _P,
+                                ctypes.POINTER(SatShardStats)], _I),
+    "sat_nccl_unique_id": ([_P], _I),
+    "sat_nccl_comm_create": ([ctypes.POINTER(ctypes.c_void_p), _P, _I, _I], _I),
+    "sat_nccl_comm_destroy": ([_P], _I),
+    "sat_compute_sharded_nccl": ([_P, _P, _I64, _I64, _I, _I, _P, _P, _P, ctypes.POINTER(SatShardStats)], _I),
     "sat_compute_host": ([_P, _P, _I64, _I64, _I, _I, _P], _I),
     "sat_release_workspace": ([_P], _I),
     "sat_debug_set_tag_space": ([ctypes.c_uint64], _I),
@@ -304,8 +310,10 @@ def sat_host(x_host, out_host=None, variant: str = "1r1w", stream=None):
     return out_host
 
 
-def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=None):
-    """Row-strip sharded SAT through the single C-ABI call.
+def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=None,
+                    variant: str = "1r1w"):
+    """Row-strip sharded SAT through the single C-ABI call
+    (sat_compute_sharded_ex; variant "1r1w" or "2r2w").
 
     ``allgather(send, recv)`` receives torch views of the library's send
     (cols) and receive (nranks x cols) buffers and must fill ``recv``.
@@ -334,12 +342,55 @@ def sat_sharded_abi(strip, rank: int, nranks: int, allgather, out=None, stream=N
             return 1
     cfun = ALLGATHER_FN(cb)
     stats = SatShardStats()
-    st = _lib.sat_compute_sharded(strip.data_ptr(), out.data_ptr(), strip.shape[0], cols,
-                                  _dtype_code(strip), int(rank), int(nranks), cfun, None,
-                                  ws.data_ptr(), _stream(stream), ctypes.byref(stats))
+    st = _lib.sat_compute_sharded_ex(strip.data_ptr(), out.data_ptr(), strip.shape[0], cols,
+                                     _dtype_code(strip), VARIANTS[variant], int(rank), int(nranks), cfun,
+                                     None, ws.data_ptr(), _stream(stream), ctypes.byref(stats))
     if err:
         raise err[0]
     _check(st)
+    return out, {f: getattr(stats, f) for f, _ in SatShardStats._fields_}
+
+
+def nccl_unique_id() -> bytes:
+    """128-byte NCCL id for sat_nccl_comm_create (rank 0 makes it, every rank gets it)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.sat_nccl_unique_id(buf))
+    return buf.raw
+
+
+class NcclComm:
+    """libsat's own NCCL communicator (sat_nccl_comm_create) on the current device."""
+
+    def __init__(self, uid: bytes, rank: int, nranks: int):
+        if len(uid) != 128:
+            raise ValueError("NCCL unique id is 128 bytes")
+        h = ctypes.c_void_p()
+        _check(_lib.sat_nccl_comm_create(ctypes.byref(h), ctypes.c_char_p(uid), int(rank), int(nranks)))
+        self.handle, self.rank, self.nranks = h, rank, nranks
+
+    def close(self):
+        if self.handle:
+            _check(_lib.sat_nccl_comm_destroy(self.handle))
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def sat_sharded_nccl(strip, comm: "NcclComm", variant: str = "1r1w", out=None, stream=None):
+    """Row-strip sharded SAT with the all-gather inside libsat (ncclAllGather,
+    sat_compute_sharded_nccl).  Returns (out, stats dict)."""
+    import torch
+    if out is None:
+        out = torch.empty_like(strip)
+    _check_dev(strip, out)
+    stats = SatShardStats()
+    _check(_lib.sat_compute_sharded_nccl(strip.data_ptr(), out.data_ptr(), strip.shape[0], strip.shape[1],
+                                         _dtype_code(strip), VARIANTS[variant], comm.handle, None,
+                                         _stream(stream), ctypes.byref(stats)))
     return out, {f: getattr(stats, f) for f, _ in SatShardStats._fields_}
 
 

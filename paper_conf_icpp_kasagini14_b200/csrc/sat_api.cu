@@ -26,6 +26,9 @@
 #include "sat_band.cuh"
 #include "sat_paper.cuh"
 #include "sat_box.cuh"
+#include <dlfcn.h>
+#include <nccl.h>
+
 #include "sat_boxf.cuh"
 #include "sat_boxw.cuh"
 #include "sat_xchg.cuh"
@@ -911,6 +914,11 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
     const bool seeded = satrow != nullptr || (cs && cs->n > 0);
     if (in_dtype != dtype && (variant != SAT_1R1W || seeded))
         return fail(SAT_ERR_UNSUPPORTED, "widening input: unseeded 1R1W only");
+    // column-sum seeds: 1R1W (band 0's first row) and 2R2W (the column pass's
+    // first row: the column prefix carries it down, the row pass across);
+    // the SAT-row seed: 1R1W only
+    if ((satrow != nullptr && variant != SAT_1R1W) || (cs && cs->n > 0 && variant != SAT_1R1W && variant != SAT_2R2W))
+        return fail(SAT_ERR_UNSUPPORTED, "seeded (sharded) SAT: variant must be 1R1W or 2R2W");
     sat_options o;
     sat_options_init(&o);
     if (opt) o = *opt;
@@ -955,7 +963,9 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             // row-wise prefix-sums (rows independent)
             Job j1 = j;
             j1.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
-            SAT_TRY(run_band(j1, MODE_COL, in, out, base_params()));
+            BandParams pc = base_params();
+            if (cs && cs->n > 0) pc.cseed = *cs;
+            SAT_TRY(run_band(j1, MODE_COL, in, out, pc));
             Job j2 = j1;
             j2.tma = !o.force_generic && tma_ok(out, out, cols);
             return run_band(j2, MODE_ROW, out, out, base_params());
@@ -1536,9 +1546,18 @@ size_t sat_sharded_workspace_bytes(int64_t cols, int nranks, int dtype) {
 int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_rows, int64_t cols,
                         int dtype, int rank, int nranks, sat_allgather_fn allgather,
                         void* comm_ctx, void* workspace, void* stream, sat_shard_stats* stats) {
+    return sat_compute_sharded_ex(in_strip, out_strip, strip_rows, cols, dtype, SAT_1R1W, rank, nranks, allgather,
+                                  comm_ctx, workspace, stream, stats);
+}
+
+int sat_compute_sharded_ex(const void* in_strip, void* out_strip, int64_t strip_rows, int64_t cols,
+                           int dtype, int variant, int rank, int nranks, sat_allgather_fn allgather,
+                           void* comm_ctx, void* workspace, void* stream, sat_shard_stats* stats) {
     t_launches = 0;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAT_ERR_INVALID, "bad rank / nranks");
+    if (variant != SAT_1R1W && variant != SAT_2R2W)
+        return fail(SAT_ERR_UNSUPPORTED, "sharded SAT: variant must be SAT_1R1W or SAT_2R2W");
     SAT_TRY(validate(in_strip, out_strip, 1, strip_rows, cols, dtype));
     if (nranks > 1 && !allgather) return fail(SAT_ERR_INVALID, "allgather callback required");
     if (stats) std::memset(stats, 0, sizeof(*stats));
@@ -1578,15 +1597,15 @@ int sat_compute_sharded(const void* in_strip, void* out_strip, int64_t strip_row
         cs.stride = int64_t(cols) * int64_t(eb);
         cs.n = rank;
     }
-    // 4. seeded local 1R1W
+    // 4. seeded local SAT (1R1W, or 2R2W whose column pass takes the seed)
     if (strip_rows > 0) {
-        SAT_TRY(compute_core(in_strip, out_strip, 1, strip_rows, cols, dtype, SAT_1R1W, nullptr,
+        SAT_TRY(compute_core(in_strip, out_strip, 1, strip_rows, cols, dtype, variant, nullptr,
                              nullptr, &cs, st));
         launches += t_launches;
     }
     t_launches = launches;
     if (stats) {
-        const int64_t b = strip_rows * cols * int64_t(eb);
+        const int64_t b = strip_rows * cols * int64_t(eb) * (variant == SAT_2R2W ? 2 : 1);
         stats->strip_bytes_read = b;
         stats->strip_bytes_written = b;
         stats->extra_bytes_read = (nranks > 1 && rank < nranks - 1) ? b : 0;
@@ -1684,6 +1703,105 @@ int sat_compute_host(const void* in_host, void* out_host, int64_t rows, int64_t 
     t_launches = launches;
     return SAT_OK;
 }
+
+// ------------------------------------------------------------------ in-library NCCL
+// The sharded mode's all-gather over NVLink/NVSwitch through an NCCL
+// communicator owned by the caller's handle.  libnccl.so.2 is loaded on first
+// use (dlopen): a process that already loaded NCCL (e.g. through PyTorch)
+// shares that copy, and libsat has no link-time NCCL dependency.
+namespace {
+struct NcclApi {
+    ncclResult_t (*get_unique_id)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*comm_init_rank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*all_gather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*comm_destroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*comm_count)(const ncclComm_t, int*) = nullptr;
+    ncclResult_t (*comm_user_rank)(const ncclComm_t, int*) = nullptr;
+    const char* (*error_string)(ncclResult_t) = nullptr;
+    std::string err;
+};
+NcclApi& nccl_api() {
+    static NcclApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) { api.err = std::string("dlopen libnccl.so.2: ") + (dlerror() ? dlerror() : "?"); return; }
+        auto sym = [&](const char* n) {
+            void* f = dlsym(h, n);
+            if (!f && api.err.empty()) api.err = std::string("libnccl: missing ") + n;
+            return f;
+        };
+        api.get_unique_id = reinterpret_cast<decltype(api.get_unique_id)>(sym("ncclGetUniqueId"));
+        api.comm_init_rank = reinterpret_cast<decltype(api.comm_init_rank)>(sym("ncclCommInitRank"));
+        api.all_gather = reinterpret_cast<decltype(api.all_gather)>(sym("ncclAllGather"));
+        api.comm_destroy = reinterpret_cast<decltype(api.comm_destroy)>(sym("ncclCommDestroy"));
+        api.comm_count = reinterpret_cast<decltype(api.comm_count)>(sym("ncclCommCount"));
+        api.comm_user_rank = reinterpret_cast<decltype(api.comm_user_rank)>(sym("ncclCommUserRank"));
+        api.error_string = reinterpret_cast<decltype(api.error_string)>(sym("ncclGetErrorString"));
+    });
+    return api;
+}
+#define NCCL_TRY(x)                                                                              \
+    do {                                                                                         \
+        const ncclResult_t r_ = (x);                                                             \
+        if (r_ != ncclSuccess)                                                                   \
+            return fail(SAT_ERR_COMM, std::string("NCCL: ") + nccl_api().error_string(r_));      \
+    } while (0)
+int nccl_allgather_cb(void* ctx, const void* send, void* recv, size_t bytes, void* stream) {
+    return nccl_api().all_gather(send, recv, bytes, ncclUint8, static_cast<ncclComm_t>(ctx),
+                                 static_cast<cudaStream_t>(stream)) == ncclSuccess ? 0 : 1;
+}
+}  // namespace
+
+extern "C" {
+
+int sat_nccl_unique_id(void* id128) {
+    if (!id128) return fail(SAT_ERR_INVALID, "null id buffer");
+    NcclApi& a = nccl_api();
+    if (!a.err.empty()) return fail(SAT_ERR_UNSUPPORTED, a.err);
+    ncclUniqueId id;
+    NCCL_TRY(a.get_unique_id(&id));
+    static_assert(sizeof(id) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(id128, &id, sizeof(id));
+    return SAT_OK;
+}
+
+int sat_nccl_comm_create(void** comm, const void* id128, int rank, int nranks) {
+    if (!comm || !id128) return fail(SAT_ERR_INVALID, "null pointer");
+    *comm = nullptr;
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(SAT_ERR_INVALID, "bad rank / nranks");
+    NcclApi& a = nccl_api();
+    if (!a.err.empty()) return fail(SAT_ERR_UNSUPPORTED, a.err);
+    ncclUniqueId id;
+    std::memcpy(&id, id128, sizeof(id));
+    ncclComm_t c = nullptr;
+    NCCL_TRY(a.comm_init_rank(&c, nranks, id, rank));
+    *comm = c;
+    return SAT_OK;
+}
+
+int sat_nccl_comm_destroy(void* comm) {
+    if (!comm) return SAT_OK;
+    NcclApi& a = nccl_api();
+    if (!a.err.empty()) return fail(SAT_ERR_UNSUPPORTED, a.err);
+    NCCL_TRY(a.comm_destroy(static_cast<ncclComm_t>(comm)));
+    return SAT_OK;
+}
+
+int sat_compute_sharded_nccl(const void* in_strip, void* out_strip, int64_t strip_rows, int64_t cols, int dtype,
+                             int variant, void* comm, void* workspace, void* stream, sat_shard_stats* stats) {
+    if (!comm) return fail(SAT_ERR_INVALID, "null NCCL communicator");
+    NcclApi& a = nccl_api();
+    if (!a.err.empty()) return fail(SAT_ERR_UNSUPPORTED, a.err);
+    int rank = 0, nranks = 0;
+    NCCL_TRY(a.comm_user_rank(static_cast<ncclComm_t>(comm), &rank));
+    NCCL_TRY(a.comm_count(static_cast<ncclComm_t>(comm), &nranks));
+    return sat_compute_sharded_ex(in_strip, out_strip, strip_rows, cols, dtype, variant, rank, nranks,
+                                  nccl_allgather_cb, comm, workspace, stream, stats);
+}
+
+}  // extern "C"
 
 static unsigned int* g_diag_host = nullptr;
 static const size_t kDiagWords = size_t(4096) * 32 * 4 * 2;

@@ -105,3 +105,19 @@ def test_validation_new_entry_points_without_gpu():
     assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 5, ctypes.byref(o), None) == -1
     assert L.sat_compute_ex(4096, 1 << 20, 4, 4, 0, 6, ctypes.byref(o), None) == -1
     assert b"variant" in L.sat_last_error()
+
+
+def test_nccl_unique_id_and_argument_checks():
+    """In-library NCCL (sat_nccl_*): libnccl.so.2 is dlopen-ed on first use;
+    the unique id needs no GPU; bad arguments fail before any NCCL call."""
+    a, b = libsat.nccl_unique_id(), libsat.nccl_unique_id()
+    assert len(a) == 128 and len(b) == 128 and a != b
+    h = ctypes.c_void_p()
+    assert L.sat_nccl_comm_create(ctypes.byref(h), a, 2, 2) == -1       # rank >= nranks
+    assert L.sat_nccl_comm_create(ctypes.byref(h), None, 0, 1) == -1    # null id
+    assert L.sat_nccl_comm_destroy(None) == 0
+    stats = libsat.SatShardStats()
+    assert L.sat_compute_sharded_nccl(8, 8, 4, 4, 0, 2, None, None, None, ctypes.byref(stats)) == -1
+    # sharded variants: 1R1W and 2R2W take the seed; the others are refused
+    assert L.sat_compute_sharded_ex(8, 8, 4, 4, 0, 1, 0, 1, libsat.ALLGATHER_FN(0), None, None, None,
+                                    None) == -2

@@ -232,6 +232,51 @@ def test_seeded_gathered_is_the_rank_exscan(libsat):
             check(got, ref[r0:], dtype)
 
 
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("variant", ["1r1w", "2r2w"])
+def test_sharded_abi_variants(libsat, P, variant):
+    """sat_compute_sharded_ex: the 2R2W strip takes the carry row in its column
+    pass; same strips as the unsharded SAT."""
+    from paper_conf_icpp_kasagini14_b200.dist import partition_rows
+    n, m = 1500, 1000
+    for dtype in ("int32", "float32"):
+        full = gen(n, m, dtype, seed=P + 11)
+        ref = oracle.sat(full)
+        bounds = [partition_rows(n, P, p) for p in range(P)]
+        strips = [dev(full[r0:r1]) for r0, r1 in bounds]
+        totals = [libsat.column_totals(s) for s in strips]
+        totals[-1] = torch.zeros_like(totals[-1])
+        outs = []
+        for p in range(P):
+            def ag(send, recv, p=p):
+                torch.cuda.synchronize()
+                recv.copy_(torch.stack(totals))
+            o, st = libsat.sat_sharded_abi(strips[p], p, P, ag, variant=variant)
+            outs.append(o.cpu().numpy())
+            rows = bounds[p][1] - bounds[p][0]
+            assert st["strip_bytes_read"] == rows * m * 4 * (2 if variant == "2r2w" else 1)
+        check(np.concatenate(outs), ref, dtype)
+
+
+@pytest.mark.parametrize("variant", ["1r1w", "2r2w"])
+def test_sharded_nccl_single_rank(libsat, variant):
+    """In-library NCCL communicator (sat_nccl_comm_create, sat_compute_sharded_nccl)
+    with one rank: libnccl loaded, communicator created on the device, rank and
+    size read back from it, the strip computed.  NCCL refuses two ranks on one
+    device, and a one-rank strip needs no gather, so ncclAllGather itself only
+    runs with >= 2 GPUs (bench.py --exchange libsat-nccl); the gather callback
+    path it plugs into is the one the virtual-rank tests above exercise."""
+    comm = libsat.NcclComm(libsat.nccl_unique_id(), 0, 1)
+    try:
+        for dtype in ("int32", "float32"):
+            a = gen(1000, 1300, dtype, seed=21)
+            y, st = libsat.sat_sharded_nccl(dev(a), comm, variant=variant)
+            check(y, oracle.sat(a), dtype)
+            assert st["extra_bytes_read"] == 0 and st["allgather_bytes"] == 0
+    finally:
+        comm.close()
+
+
 @pytest.mark.parametrize("P", [1, 2, 3, 8])
 def test_sharded_abi_single_process(libsat, P):
     """sat_compute_sharded with a fake all-gather: P ranks simulated one after
