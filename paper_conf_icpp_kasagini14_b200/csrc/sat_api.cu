@@ -1174,8 +1174,12 @@ int box_walk_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t c
                cudaStream_t st) {
     constexpr int NWARP = 4;
     constexpr int PF = sizeof(TI) == 1 ? 8 : 4;   // rows in flight per warp (cp.async ring)
-    auto kern = sat_boxw_kernel<TI, TS, TO, NWARP, PF>;
-    const size_t smem = size_t(NWARP) * boxw_warp_smem<TI, TS, PF>(rr);
+    // float input (float64 sums): two outputs per lane, so the float64 D ring
+    // and P buffer stay small enough for ~24 warps per SM
+    constexpr int OPL = sizeof(TS) == 8 ? 2 : 4;
+    constexpr int SWC = 32 * OPL;                 // output columns per unit
+    auto kern = sat_boxw_kernel<TI, TS, TO, NWARP, PF, OPL>;
+    const size_t smem = size_t(NWARP) * boxw_warp_smem<TI, TS, PF, OPL>(rr);
     static KernelSetup setup;
     int dev = 0;
     CUDA_TRY(cudaGetDevice(&dev));
@@ -1189,7 +1193,7 @@ int box_walk_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t c
     BoxWParams bp;
     bp.in = in; bp.out = out; bp.rows = int(rows); bp.cols = int(cols); bp.batch = int(batch);
     bp.rr = rr; bp.rc = rc; bp.normalize = normalize;
-    bp.nc = int((cols + TW - 1) / TW);
+    bp.nc = int((cols + SWC - 1) / SWC);
     bp.rb = g_box_rb.load(std::memory_order_relaxed);
     if (bp.rb <= 0) {
         // one wave: as many row blocks per strip as the resident warps allow
@@ -1391,9 +1395,11 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
     SAT_TRY(get_dev(dev, di));
     Workspace* ws;
     SAT_TRY(get_ws(dev, st, ws));
-    // Column walk (one launch, one warp per 128-column strip of a row block,
-    // sat_boxw.cuh) when out does not alias in, rc <= 63 and the D ring fits:
-    // 32 x 1080x1920 uint8 r = 4: see DESIGN.md Sec. 4.12
+    // Column walk (one launch, one warp per 128-column strip of a row block --
+    // 64 columns for float input, sat_boxw.cuh) when out does not alias in,
+    // rc <= 63 and rr <= 8 (uint8 / int32 / float32): 32 x 1080x1920 r = 4
+    // uint8 0.127 ms, int32 0.150, float32 0.272 (band kernel: 0.182 / 0.186 /
+    // 0.305), DESIGN.md Sec. 4.12
     const bool walk_al = in_dtype == SAT_UINT8 ? (cols % 8 == 0 && (reinterpret_cast<uintptr_t>(in) & 7) == 0)
                                                : (cols % 4 == 0 && (reinterpret_cast<uintptr_t>(in) & 15) == 0);
     if (walk_al && in != out && rc <= 63 && rr <= 16 && rows <= INT32_MAX && cols <= INT32_MAX &&
@@ -1402,6 +1408,10 @@ int sat_box_filter(const void* in, int in_dtype, void* out, int out_dtype, int64
             return box_walk_t<uint8_t, uint32_t, int32_t>(in, out, batch, rows, cols, rr, rc, 0, st);
         if (in_dtype == SAT_INT32 && rr <= 8)
             return box_walk_t<uint32_t, uint32_t, int32_t>(in, out, batch, rows, cols, rr, rc, 0, st);
+        if (in_dtype == SAT_FLOAT32 && rr <= 8)
+            return out_dtype == SAT_FLOAT32
+                       ? box_walk_t<float, double, float>(in, out, batch, rows, cols, rr, rc, normalize, st)
+                       : box_walk_t<float, double, double>(in, out, batch, rows, cols, rr, rc, normalize, st);
     }
     // Fused (one launch, the SAT never leaves the chip, sat_boxf.cuh) when the
     // input is TMA-addressable, out does not alias it (a band's halo rows are

@@ -48,32 +48,60 @@ struct BoxWParams {
     long long units;       // batch * nrb * nc
 };
 
-// shared bytes per warp: raw-row ring (PF rows x 256 span columns of TI) +
-// the P buffer (256 entries) + the D ring (2rr + 1 rows of 128)
-template <typename TI, typename TS, int PF>
+// A unit is SW = 32 * OPL output columns: lane L owns outputs c0 + L + 32e
+// (e < OPL) and the span positions 8L' .. of the SW + 128 columns around them
+// (a 64-column halo each side), EPS = OPL + 4 elements per lane.
+template <int OPL>
+struct BoxWGeom {
+    static constexpr int SW = 32 * OPL;          // output columns per unit
+    static constexpr int SPAN = SW + 128;        // loaded columns
+    static constexpr int EPS = SPAN / 32;        // span elements per lane
+};
+
+// shared bytes per warp: raw-row ring (PF rows of the span, TI) + the P buffer
+// (SPAN entries) + the D ring (2rr + 1 rows of SW)
+template <typename TI, typename TS, int PF, int OPL = 4>
 SAT_HD size_t boxw_warp_smem(int rr) {
-    return size_t(PF) * 256 * sizeof(TI) + (size_t(256) + size_t(2 * rr + 1) * 128) * sizeof(TS);
+    using G = BoxWGeom<OPL>;
+    return size_t(PF) * G::SPAN * sizeof(TI) + (size_t(G::SPAN) + size_t(2 * rr + 1) * G::SW) * sizeof(TS);
 }
 
-// Asynchronous copy of the lane's 8 span elements (8 or 32 bytes) into the
-// warp's raw-row ring; a lane group outside the image copies nothing and its
-// bytes are zero-filled (src-size 0), which is the window clipping.
-template <typename TI>
-__device__ __forceinline__ void boxw_cp(uint32_t dst, const TI* src, bool ok0, bool ok1) {
+// Asynchronous copy of the lane's EPS span elements into the warp's raw-row
+// ring in pieces of 8 B (uint8: one piece of 8; 4-byte types with EPS = 8:
+// two 16-B pieces; EPS = 6: three 8-B pieces); a piece outside the image
+// copies nothing and is zero-filled (src-size 0), which is the window
+// clipping.  ok = bit mask of the pieces inside the image.
+// row = column 0 of the row; a piece outside the image reads from `row`
+// itself (a valid address, no bytes taken)
+template <typename TI, int EPS>
+__device__ __forceinline__ void boxw_cp(uint32_t dst, const TI* row, int s0, uint32_t ok) {
     if constexpr (sizeof(TI) == 1) {
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" :: "r"(dst), "l"(src), "r"(ok0 ? 8 : 0) : "memory");
+        static_assert(EPS == 8, "uint8: 8 span elements per lane");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" :: "r"(dst), "l"(row + ((ok & 1u) ? s0 : 0)),
+                     "r"((ok & 1u) ? 8 : 0) : "memory");
+    } else if constexpr (EPS == 8) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            const bool in = (ok >> q) & 1u;
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst + 16 * q),
+                         "l"(row + (in ? s0 + 4 * q : 0)), "r"(in ? 16 : 0) : "memory");
+        }
     } else {
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst), "l"(src), "r"(ok0 ? 16 : 0) : "memory");
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(dst + 16), "l"(src + 4), "r"(ok1 ? 16 : 0)
-                     : "memory");
+        static_assert(EPS % 2 == 0, "8-B pieces");
+#pragma unroll
+        for (int q = 0; q < EPS / 2; ++q) {
+            const bool in = (ok >> q) & 1u;
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" :: "r"(dst + 8 * q),
+                         "l"(row + (in ? s0 + 2 * q : 0)), "r"(in ? 8 : 0) : "memory");
+        }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
 }
 template <int N>
 __device__ __forceinline__ void boxw_cp_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
 
-template <typename TI, typename TS>
-__device__ __forceinline__ void boxw_widen(uint32_t raddr, TS (&e)[8]) {
+template <typename TI, typename TS, int EPS>
+__device__ __forceinline__ void boxw_widen(uint32_t raddr, TS (&e)[EPS]) {
     if constexpr (sizeof(TI) == 1) {
         uint32_t a, b;
         asm volatile("ld.shared.v2.b32 {%0, %1}, [%2];" : "=r"(a), "=r"(b) : "r"(raddr));
@@ -83,12 +111,12 @@ __device__ __forceinline__ void boxw_widen(uint32_t raddr, TS (&e)[8]) {
             e[4 + t] = TS(__byte_perm(b, 0u, 0x4440u + t));
         }
     } else {
-        uint32_t w[8];
-        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "r"(raddr));
-        asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
-                     : "r"(raddr + 16));
+        uint32_t w[EPS];
 #pragma unroll
-        for (int t = 0; t < 8; ++t) {
+        for (int q = 0; q < EPS / 2; ++q)
+            asm volatile("ld.shared.v2.b32 {%0, %1}, [%2];" : "=r"(w[2 * q]), "=r"(w[2 * q + 1]) : "r"(raddr + 8 * q));
+#pragma unroll
+        for (int t = 0; t < EPS; ++t) {
             if constexpr (std::is_same<TI, float>::value) e[t] = TS(__uint_as_float(w[t]));
             else e[t] = TS(w[t]);
         }
@@ -113,18 +141,20 @@ __device__ __forceinline__ void boxw_sts(uint32_t a, TS v) {
     else asm volatile("st.shared.f64 [%0], %1;" :: "r"(a), "d"(v));
 }
 
-template <typename TI, typename TS, typename TO, int NWARP, int PF>
+template <typename TI, typename TS, typename TO, int NWARP, int PF, int OPL = 4>
 __global__ void __launch_bounds__(NWARP * 32) sat_boxw_kernel(const BoxWParams bp) {
+    using G = BoxWGeom<OPL>;
+    constexpr int SW = G::SW, SPAN = G::SPAN, EPS = G::EPS;
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int ring_rows = 2 * bp.rr + 1;
-    // per-warp shared layout: raw ring [PF][256] TI | P [256] TS | D ring [2rr+1][128] TS
-    const uint32_t wbase = smem_u32(smem) + uint32_t(warp * boxw_warp_smem<TI, TS, PF>(bp.rr));
-    const uint32_t raw0 = wbase + uint32_t(8 * lane * sizeof(TI));          // lane's slot in raw row 0
-    constexpr uint32_t RAW_ROW = 256 * sizeof(TI);
+    // per-warp shared layout: raw ring [PF][SPAN] TI | P [SPAN] TS | D ring [2rr+1][SW] TS
+    const uint32_t wbase = smem_u32(smem) + uint32_t(warp * boxw_warp_smem<TI, TS, PF, OPL>(bp.rr));
+    const uint32_t raw0 = wbase + uint32_t(EPS * lane * sizeof(TI));        // lane's slot in raw row 0
+    constexpr uint32_t RAW_ROW = SPAN * sizeof(TI);
     const uint32_t pb = wbase + PF * RAW_ROW;
-    const uint32_t ring0 = pb + 256 * sizeof(TS) + lane * sizeof(TS);
-    const uint32_t ring_end = ring0 + uint32_t(ring_rows) * 128 * sizeof(TS);
+    const uint32_t ring0 = pb + SPAN * sizeof(TS) + lane * sizeof(TS);
+    const uint32_t ring_end = ring0 + uint32_t(ring_rows) * SW * sizeof(TS);
     asm volatile("griddepcontrol.wait;" ::: "memory");
     const long long unit = (long long)blockIdx.x * NWARP + warp;
     if (unit >= bp.units) return;
@@ -135,23 +165,25 @@ __global__ void __launch_bounds__(NWARP * 32) sat_boxw_kernel(const BoxWParams b
     const int i0 = rbk * bp.rb, i1 = min(bp.rows, i0 + bp.rb);
     const int kstart = max(0, i0 - bp.rr), kend = i1 - 1 + bp.rr;   // inclusive
     const int klast = min(kend, bp.rows - 1);                        // last row that exists
-    const int c0 = c * 128;
-    const int s0 = c0 - 64 + 8 * lane;
-    // lane groups are whole 4/8-column groups inside or outside the image
-    // (host: cols % 8 == 0 and 8-B aligned rows for uint8, cols % 4 == 0 and
-    // 16-B aligned rows for 4-byte types)
-    const bool ok0 = s0 >= 0 && s0 + (sizeof(TI) == 1 ? 8 : 4) <= bp.cols;
-    const bool ok1 = s0 + 4 >= 0 && s0 + 8 <= bp.cols;
-    const TI* src = reinterpret_cast<const TI*>(bp.in) + (int64_t(img) * bp.rows + kstart) * bp.cols
-                    + (ok0 || ok1 ? s0 : 0);
+    const int c0 = c * SW;
+    const int s0 = c0 - 64 + EPS * lane;
+    // copy pieces (8 B for uint8, 16 B at EPS 8, 8 B at EPS 6) lie wholly
+    // inside or outside the image: host requires cols % 8 == 0 for uint8,
+    // % 4 == 0 for 4-byte types
+    constexpr int PIECE = sizeof(TI) == 1 ? 8 : (EPS == 8 ? 4 : 2);   // elements per piece
+    uint32_t ok = 0;
+#pragma unroll
+    for (int q = 0; q < EPS / PIECE; ++q)
+        if (s0 + PIECE * q >= 0 && s0 + PIECE * (q + 1) <= bp.cols) ok |= 1u << q;
+    const TI* src = reinterpret_cast<const TI*>(bp.in) + (int64_t(img) * bp.rows + kstart) * bp.cols;  // row kstart
     TO* dst = reinterpret_cast<TO*>(bp.out) + (int64_t(img) * bp.rows + i0) * bp.cols + c0 + lane;
     // shared addresses of the window's corner columns in P (span index =
     // column - (c0 - 64)); clipping is done by the zero fill
-    uint32_t ar[4], al[4];
-    bool jin[4];
-    int ww[4];
+    uint32_t ar[OPL], al[OPL];
+    bool jin[OPL];
+    int ww[OPL];
 #pragma unroll
-    for (int e = 0; e < 4; ++e) {
+    for (int e = 0; e < OPL; ++e) {
         const int x = 64 + lane + 32 * e;
         ar[e] = pb + uint32_t((x + bp.rc) * sizeof(TS));
         al[e] = pb + uint32_t((x - bp.rc - 1) * sizeof(TS));
@@ -162,75 +194,80 @@ __global__ void __launch_bounds__(NWARP * 32) sat_boxw_kernel(const BoxWParams b
     // prologue: rows kstart .. kstart + PF - 1 in flight (empty groups past klast)
 #pragma unroll
     for (int u = 0; u < PF; ++u) {
-        if (kstart + u <= klast) boxw_cp<TI>(raw0 + u * RAW_ROW, src + int64_t(u) * bp.cols, ok0, ok1);
+        if (kstart + u <= klast) boxw_cp<TI, EPS>(raw0 + u * RAW_ROW, src + int64_t(u) * bp.cols, s0, ok);
         else asm volatile("cp.async.commit_group;" ::: "memory");
     }
     const TI* nxt = src + int64_t(PF) * bp.cols;                  // row k + PF
-    TS V[4] = {TS(0), TS(0), TS(0), TS(0)};
+    TS V[OPL];
+#pragma unroll
+    for (int e = 0; e < OPL; ++e) V[e] = TS(0);
     uint32_t rs = ring0;                                          // ring slot of row k
     int q = 0;                                                    // raw ring slot of row k
     for (int k = kstart; k <= kend; ++k) {
-        TS D[4] = {TS(0), TS(0), TS(0), TS(0)};
+        TS D[OPL];
+#pragma unroll
+        for (int e = 0; e < OPL; ++e) D[e] = TS(0);
         if (k <= klast) {
             boxw_cp_wait<PF - 1>();                               // row k landed (this lane's copies)
-            TS e8[8];
-            boxw_widen<TI, TS>(raw0 + q * RAW_ROW, e8);
+            TS e8[EPS];
+            boxw_widen<TI, TS, EPS>(raw0 + q * RAW_ROW, e8);
             // refill the slot with row k + PF (an empty group keeps the count);
             // a lane reads and refills only its own bytes of the slot
-            if (k + PF <= klast) boxw_cp<TI>(raw0 + q * RAW_ROW, nxt, ok0, ok1);
+            if (k + PF <= klast) boxw_cp<TI, EPS>(raw0 + q * RAW_ROW, nxt, s0, ok);
             else asm volatile("cp.async.commit_group;" ::: "memory");
             nxt += bp.cols;
 #pragma unroll
-            for (int t = 1; t < 8; ++t) e8[t] += e8[t - 1];
-            const TS inc = warp_inclusive_scan(e8[7], lane);
+            for (int t = 1; t < EPS; ++t) e8[t] += e8[t - 1];
+            const TS inc = warp_inclusive_scan(e8[EPS - 1], lane);
             TS exc;
             if constexpr (std::is_same<TS, uint32_t>::value) {
-                exc = inc - e8[7];
+                exc = inc - e8[EPS - 1];
             } else {
                 exc = __shfl_up_sync(0xffffffffu, inc, 1);
                 if (lane == 0) exc = TS(0);
             }
-            const uint32_t pw = pb + uint32_t(8 * lane * sizeof(TS));
+            const uint32_t pw = pb + uint32_t(EPS * lane * sizeof(TS));
             if constexpr (sizeof(TS) == 4) {
+                static_assert(EPS == 8, "uint32 sums: 8 span elements per lane");
                 asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" :: "r"(pw), "r"(e8[0] + exc), "r"(e8[1] + exc),
                              "r"(e8[2] + exc), "r"(e8[3] + exc) : "memory");
                 asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" :: "r"(pw + 16), "r"(e8[4] + exc),
                              "r"(e8[5] + exc), "r"(e8[6] + exc), "r"(e8[7] + exc) : "memory");
             } else {
 #pragma unroll
-                for (int t = 0; t < 8; t += 2)
+                for (int t = 0; t < EPS; t += 2)
                     asm volatile("st.shared.v2.f64 [%0], {%1, %2};" :: "r"(pw + 8 * t), "d"(e8[t] + exc),
                                  "d"(e8[t + 1] + exc) : "memory");
             }
             __syncwarp();
 #pragma unroll
-            for (int e = 0; e < 4; ++e) D[e] = boxw_lds<TS>(ar[e]) - boxw_lds<TS>(al[e]);
+            for (int e = 0; e < OPL; ++e) D[e] = boxw_lds<TS>(ar[e]) - boxw_lds<TS>(al[e]);
             __syncwarp();                                         // P reads done before the next row's writes
             if (++q == PF) q = 0;
         }
         // vertical window: V(k - rr) = sum of D over rows k - 2rr .. k
         if (k - kstart >= ring_rows) {
 #pragma unroll
-            for (int e = 0; e < 4; ++e) V[e] -= boxw_lds<TS>(rs + 32 * e * sizeof(TS));
+            for (int e = 0; e < OPL; ++e) V[e] -= boxw_lds<TS>(rs + 32 * e * sizeof(TS));
         }
 #pragma unroll
-        for (int e = 0; e < 4; ++e) {
+        for (int e = 0; e < OPL; ++e) {
             boxw_sts<TS>(rs + 32 * e * sizeof(TS), D[e]);
             V[e] += D[e];
         }
-        rs += 128 * sizeof(TS);
+        rs += SW * sizeof(TS);
         if (rs == ring_end) rs = ring0;
         const int i = k - bp.rr;
         if (i >= i0) {
             if constexpr (std::is_same<TS, uint32_t>::value) {
 #pragma unroll
-                for (int e = 0; e < 4; ++e)
+                for (int e = 0; e < OPL; ++e)
                     if (jin[e]) __stcs(dst + 32 * e, TO(int32_t(V[e])));
             } else {
                 int hh = 1;
                 if (bp.normalize) hh = min(i + bp.rr, bp.rows - 1) - max(i - bp.rr, 0) + 1;
 #pragma unroll
-                for (int e = 0; e < 4; ++e) {
+                for (int e = 0; e < OPL; ++e) {
                     TS sv = V[e];
                     if (bp.normalize) sv = sv / TS(int64_t(hh) * int64_t(ww[e]));
                     if (jin[e]) __stcs(dst + 32 * e, TO(sv));

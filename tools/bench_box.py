@@ -68,8 +68,8 @@ def main():
         # column walk (sat_boxw.cuh, rc <= 63): input (1 + 2r/64) x eb_in (row-block warm-up), 4 B out
         (f"box filter u8 r={r} walk (1 B in x (1 + 2r/64) + 4 B out)", lambda: libsat.box_filter(u8, r, r, out=box),
          int((1 + 2 * r / 64) * px) + 4 * px, px),
-        (f"box filter f32->f32 r={r} fused band (float64 SAT on chip)", lambda: libsat.box_filter(f32, r, r, out=f32o),
-         int(4 * (1 + 2 * r / 16) * px) + 4 * px, px),
+        (f"box filter f32->f32 r={r} walk (float64 sums)", lambda: libsat.box_filter(f32, r, r, out=f32o),
+         int(4 * (1 + 2 * r / 64) * px) + 4 * px, px),
         (f"box filter int32 r={r} walk (4 B in x (1 + 2r/64) + 4 B out)", lambda: libsat.box_filter(i32, r, r, out=box),
          int(4 * (1 + 2 * r / 64) * px) + 4 * px, px),
         # band kernel with the SAT on chip (sat_boxf.cuh) for 64 <= rc < 128
