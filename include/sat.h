@@ -171,10 +171,10 @@ int sat_compute_widening(const void *in, int in_dtype, void *out, int dtype,
  * |k - i| <= rr, |l - j| <= rc, clipped to the image; the four-corner SAT
  * formula with uint32 sums for SAT_UINT8/SAT_INT32 input and float64 sums for
  * SAT_FLOAT32/SAT_FLOAT64 input.  One launch, the SAT never in HBM, when out
- * does not alias in: integer input with rr <= 8, rc <= 63
- * and 8-B (uint8, cols % 8 == 0) / 16-B (int32, cols % 4 == 0) aligned rows
- * takes the column-walk kernel (row prefix sums differenced, a running
- * vertical window sum); other TMA-addressable cases with rc <= 127 and
+ * does not alias in: uint8 / int32 / float32 input with
+ * rr <= 8, rc <= 63 and 8-B (uint8, cols % 8 == 0) / 16-B (4-byte types,
+ * cols % 4 == 0) aligned rows takes the column-walk kernel (row prefix sums
+ * differenced, a running vertical window sum); other TMA-addressable cases with rc <= 127 and
  * 2 rr <= 32 (uint8/int32) or 16 (float32) the band kernel with the local SAT
  * in shared memory.  Otherwise (in place, larger radii, float64 input,
  * unaligned rows) a widening 1R1W SAT goes to a library workspace and a second
