@@ -1,5 +1,5 @@
 // sat_boxw.cuh -- the box filter as a SAT evaluated on the fly, one warp per
-// strip of 128 output columns walking down the rows (
+// strip of output columns walking down the rows (
 // the sum of any rectangle in O(1) from the SAT).
 //
 // out[i][j] = S[i2][j2] - S[i1-1][j2] - S[i2][j1-1] + S[i1-1][j1-1]
@@ -12,24 +12,27 @@
 // add/subtract per pixel -- no SAT in HBM, no SAT tile in shared memory, no
 // barrier between warps (every warp owns its own units).
 //
-// Unit = (image, 128-column strip c, block of RB output rows).  Per input row
-// k of [i0 - rr, i1 - 1 + rr]:
-//   * lane L loads columns c*128 - 64 + 8L .. +7 (the strip plus a 64-column
-//     halo each side; rc <= 63), out-of-image columns read as 0, so the
-//     prefix P over the 256-column span is flat outside the image and the
-//     clipping of the window comes for free;
-//   * P: 8-element serial scan per lane + warp shuffle scan, written to the
-//     warp's 256-entry shared buffer (P is offset by the span's start, which
-//     cancels in D);
-//   * D for the lane's output columns j = c*128 + L + 32e (e = 0..3:
+// Unit = (image, strip c of SW = 32 OPL output columns, block of RB output
+// rows): OPL = 4 (128 columns) for uint32 sums, 2 (64 columns) for float64
+// sums, whose shared buffers are twice as wide.  Per input row k of
+// [i0 - rr, i1 - 1 + rr]:
+//   * lane L holds columns c*SW - 64 + EPS*L .. +EPS-1 (EPS = OPL + 4: the
+//     strip plus a 64-column halo each side; rc <= 63), copied by cp.async
+//     into a per-warp ring PF rows deep; pieces outside the image are
+//     zero-filled, so the prefix P over the span is flat outside the image and
+//     the clipping of the window comes for free;
+//   * P: EPS-element serial scan per lane + warp shuffle scan, written to the
+//     warp's shared P buffer (P is offset by the span's start, which cancels
+//     in D);
+//   * D for the lane's output columns j = c*SW + L + 32e (e < OPL:
 //     consecutive lanes, consecutive words: conflict-free reads);
 //   * V += D - D(k - 2rr - 1), the old D from a per-warp shared ring of
 //     2rr + 1 rows; output row k - rr once the window is complete, stored as
-//     four coalesced 128-B warp stores.
-// Rows are loaded PF iterations ahead into registers (software pipeline).
-// The first 2rr rows of a unit are a warm-up (input re-read from L2); input
-// traffic ~ (1 + 2rr/RB)(1 + 128/128 halo, L2 hits) x eb_in per pixel, output
-// eb_out per pixel.  DESIGN.md Sec. 4.12.
+//     OPL coalesced warp stores.
+// The first 2rr rows of a unit are a warm-up (input re-read from L2); units
+// are sized by the host to fill one wave of resident warps.  Input traffic
+// ~ (1 + 2rr/RB) x eb_in per pixel from HBM (halo columns and warm-up rows
+// hit L2), output eb_out per pixel.  DESIGN.md Sec. 4.12.
 #pragma once
 #include "sat_common.h"
 #include "sat_device.cuh"
@@ -44,7 +47,7 @@ struct BoxWParams {
     int normalize;         // float only
     int rb;                // output rows per unit
     int nrb;               // row blocks per image
-    int nc;                // 128-column strips per image
+    int nc;                // SW-column strips per image
     long long units;       // batch * nrb * nc
 };
 

@@ -32,3 +32,4 @@ timeout 600 ncu --set full --clock-control none -k regex:sat_boxw -s 2 -c 1 -o $
 ncu -i $O/prof_boxw.ncu-rep --page details > $O/prof_boxw_details.txt 2>/dev/null
 ncu -i $O/prof_boxw.ncu-rep --page raw --csv > $O/prof_boxw_raw.csv 2>/dev/null
 rm -f $O/prof_boxw.ncu-rep
+timeout 400 python tools/fuzz.py --seconds 240 --seed 11 > $O/fuzz11.log 2>&1
