@@ -1736,7 +1736,11 @@ NcclApi& nccl_api() {
     std::call_once(once, [] {
         void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
         if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
-        if (!h) { api.err = std::string("dlopen libnccl.so.2: ") + (dlerror() ? dlerror() : "?"); return; }
+        if (!h) {
+            const char* e = dlerror();          // read once: a second call returns NULL
+            api.err = std::string("dlopen libnccl.so.2: ") + (e ? e : "unknown error");
+            return;
+        }
         auto sym = [&](const char* n) {
             void* f = dlsym(h, n);
             if (!f && api.err.empty()) api.err = std::string("libnccl: missing ") + n;
