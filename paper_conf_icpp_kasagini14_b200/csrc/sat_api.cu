@@ -1173,7 +1173,10 @@ template <typename TI, typename TS, typename TO>
 int box_walk_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t cols, int rr, int rc, int normalize,
                cudaStream_t st) {
     constexpr int NWARP = 4;
-    constexpr int PF = sizeof(TI) == 1 ? 8 : 4;   // rows in flight per warp (cp.async ring)
+    // rows in flight per warp (cp.async ring); 4 also for uint8 rows (8 B per
+    // lane): the smaller ring buys occupancy -- uint8 r = 8 0.148 -> 0.125 ms,
+    // r = 4 0.127 / 0.129 (tools/bench_box.py)
+    constexpr int PF = 4;
     // float input (float64 sums): two outputs per lane, so the float64 D ring
     // and P buffer stay small enough for ~24 warps per SM
     constexpr int OPL = sizeof(TS) == 8 ? 2 : 4;
