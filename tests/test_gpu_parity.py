@@ -799,3 +799,14 @@ def test_fused_exchange_with_band_segments(libsat):
         check(outs[0][:512], oracle.sat(full[:512].cpu().numpy()), "int32")
     for e in exs:
         e.close()
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_2r2w_th128_column_pass(libsat, dtype):
+    """2R2W's column pass takes the TH-128 band configuration where plain 1R1W
+    does (forced, and automatic at 16384 rows); the row pass stays at TH 64."""
+    a = gen(3000, 2500, dtype, seed=31)
+    check(libsat.sat(dev(a), variant="2r2w", tile_rows=128), oracle.sat(a), dtype)
+    b = gen(16384, 1100, dtype, seed=32)
+    check(libsat.sat(dev(b), variant="2r2w"), oracle.sat(b), dtype)
+    check(libsat.sat(dev(b), variant="2r2w", jitter=20000), oracle.sat(b), dtype)
