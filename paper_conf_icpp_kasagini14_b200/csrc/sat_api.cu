@@ -871,7 +871,15 @@ int transpose_t(const void* in, void* out, int64_t batch, int64_t rows, int64_t 
 int run_4r4w(const Job& j, const sat_options& o) {
     Workspace& ws = *j.ws;
     SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * esize(j.dtype), false));
-    SAT_TRY(run_band(j, MODE_COL, j.in, j.out, base_params()));
+    // column passes at TH 128 where plain 1R1W takes it (as in 2R2W)
+    auto col_th = [&](int64_t rows, int th) {
+        if (!o.tile_rows && j.dtype != SAT_FLOAT64 && auto_th(rows, j.batch, *j.di, SAT_1R1W, j.dtype) == 128)
+            return 128;
+        return th;
+    };
+    Job j1 = j;
+    j1.th = col_th(j.rows, j.th);
+    SAT_TRY(run_band(j1, MODE_COL, j.in, j.out, base_params()));
     auto tp = [&](const void* a, void* b, int64_t r, int64_t c) {
         return SAT_DISPATCH(j.dtype, T, transpose_t<T>(a, b, j.batch, r, c, j.st));
     };
@@ -881,7 +889,7 @@ int run_4r4w(const Job& j, const sat_options& o) {
     jt.cols = j.rows;
     jt.in = ws.tr.p;
     jt.out = ws.tr.p;
-    jt.th = o.tile_rows ? o.tile_rows : auto_th(jt.rows, jt.batch, *j.di, SAT_4R4W, j.dtype);
+    jt.th = col_th(jt.rows, o.tile_rows ? o.tile_rows : auto_th(jt.rows, jt.batch, *j.di, SAT_4R4W, j.dtype));
     jt.tma = !o.force_generic && tma_ok(ws.tr.p, ws.tr.p, jt.cols);
     SAT_TRY(run_band(jt, MODE_COL, ws.tr.p, ws.tr.p, base_params()));
     return tp(ws.tr.p, j.out, jt.rows, jt.cols);
