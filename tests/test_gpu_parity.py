@@ -810,3 +810,11 @@ def test_2r2w_th128_column_pass(libsat, dtype):
     b = gen(16384, 1100, dtype, seed=32)
     check(libsat.sat(dev(b), variant="2r2w"), oracle.sat(b), dtype)
     check(libsat.sat(dev(b), variant="2r2w", jitter=20000), oracle.sat(b), dtype)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_2r1w_auto_th128(libsat, dtype):
+    """2R1W takes TH 128 automatically where plain 1R1W does (16384 rows)."""
+    a = gen(16384, 1000, dtype, seed=33)
+    check(libsat.sat(dev(a), variant="2r1w"), oracle.sat(a), dtype)
+    assert libsat.last_tile_rows() == 128
