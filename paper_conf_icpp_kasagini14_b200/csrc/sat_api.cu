@@ -408,7 +408,7 @@ int band_th(int mode, int dtype, bool tma, int th) {
         if (mode == MODE_SAT && dtype != SAT_FLOAT64 && th >= 128) return 128;
         return 32;
     }
-    if (mode == MODE_COL && dtype != SAT_FLOAT64 && th >= 128) return 128;
+    if (mode != MODE_SAT && dtype != SAT_FLOAT64 && th >= 128) return 128;
     if (mode != MODE_SAT) return th >= 64 ? 64 : 32;
     if (dtype == SAT_FLOAT64) return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
     return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
@@ -429,8 +429,7 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
             if (th == 64) return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
             return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
         } else {
-            if constexpr (MODE == MODE_COL)
-                if (th == 128) return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
+            if (th == 128) return launch_band_t<T, SAT_CFG(kCfg128), MODE, TMA, kCfg128.MINB, kLbw128>(p, ti, di, st, grid);
             if (th == 64) return launch_band_t<T, SAT_CFG(kCfg64), MODE, TMA, kCfg64.MINB>(p, ti, di, st, grid);
             return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
         }
@@ -977,10 +976,9 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             // row-wise prefix-sums (rows independent)
             Job j1 = j;
             j1.th = o.tile_rows ? o.tile_rows : auto_th(rows, batch, di, variant, dtype);
-            // the column pass (a 1R1W-style look-back) takes the TH-128
-            // configuration where plain 1R1W does: 16384^2 int32 0.851 ->
-            // 0.797 ms, 18432^2 1.049 -> 0.995, 65536^2 12.37 -> 12.20; the
-            // row pass keeps TH 64 (band_th)
+            // both passes take the TH-128 configuration where plain 1R1W
+            // does: 16384^2 int32 0.851 -> 0.797 ms (column pass) -> 0.759
+            // (and the row pass), 18432^2 1.049 -> 0.987
             if (!o.tile_rows && dtype != SAT_FLOAT64 && auto_th(rows, batch, di, SAT_1R1W, dtype) == 128)
                 j1.th = 128;
             BandParams pc = base_params();
