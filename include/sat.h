@@ -161,7 +161,8 @@ int sat_compute_batched(const void *in, void *out, int64_t batch, int64_t rows,
  * SAT_1R1W.  batch x rows x cols, back to back.  in == out is invalid for a
  * widening pair.  TMA path needs 16-B aligned pointers and cols % 16 == 0
  * (uint8) or cols % 4 == 0; otherwise the generic path runs.  tile_rows: 64 or
- * 128 for uint8 input, 16/32/64 for float32 -> float64. */
+ * 128 for uint8 input, 16/32/64/128 for float32 -> float64 (128: 64-column
+ * chunks, as plain float64). */
 int sat_compute_widening(const void *in, int in_dtype, void *out, int dtype,
                          int64_t batch, int64_t rows, int64_t cols,
                          const sat_options *opt, void *stream);

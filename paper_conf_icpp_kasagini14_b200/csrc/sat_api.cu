@@ -469,6 +469,9 @@ int launch_band_widen(int th, const BandParams& p, const CUtensorMap& ti, const 
         if constexpr (TMA) {
             if (th == 16) return launch_band_t<T, SAT_CFG(kCfgD16), MODE_SAT, TMA, kCfgD16.MINB, 0, TI>(p, ti, di, st, grid);
             if (th == 64) return launch_band_t<T, SAT_CFG(kCfgD64), MODE_SAT, TMA, kCfgD64.MINB, 0, TI>(p, ti, di, st, grid);
+            if (th == 128)
+                return launch_band_t<T, SAT_CFG(kCfgD128), MODE_SAT, TMA, kCfgD128.MINB, kLbwD, TI, kTwD128>(
+                    p, ti, di, st, grid);
         }
         return launch_band_t<T, SAT_CFG(kCfgD32), MODE_SAT, TMA, kCfgD32.MINB, 0, TI>(p, ti, di, st, grid);
     }
@@ -572,7 +575,8 @@ __global__ void sat_epoch_kernel(unsigned long long* tk, unsigned long long wors
 // The band height a launch actually uses (the instantiated configurations).
 int eff_th(const Job& j, int mode) {
     if (j.in_dtype == SAT_UINT8) return (j.tma && j.th >= 128) ? 128 : 64;
-    if (j.in_dtype != j.dtype) return j.tma ? (j.th >= 64 ? 64 : j.th >= 32 ? 32 : 16) : 32;
+    // float32 -> float64: TH 128 with 64-column chunks like plain float64
+    if (j.in_dtype != j.dtype) return j.tma ? (j.th >= 128 ? 128 : j.th >= 64 ? 64 : j.th >= 32 ? 32 : 16) : 32;
     return band_th(mode, j.dtype, j.tma, j.th);
 }
 
@@ -597,8 +601,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     p.cols = j.cols;
     p.batch = int(j.batch);
     // chunk width: 64 columns for float64 at TH 128 (kCfgD128), else 128
-    const int tw = (mode == MODE_SAT && j.tma && j.dtype == SAT_FLOAT64 && j.in_dtype == j.dtype && j.th == 128)
-                       ? kTwD128 : TW;
+    const int tw = (mode == MODE_SAT && j.tma && j.dtype == SAT_FLOAT64 && j.th == 128) ? kTwD128 : TW;
     p.nb = int((j.rows + j.th - 1) / j.th);
     p.nc = int((j.cols + tw - 1) / tw);
     p.total_bands = int(j.batch * p.nb);
