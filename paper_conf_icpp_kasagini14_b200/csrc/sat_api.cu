@@ -408,7 +408,7 @@ int band_th(int mode, int dtype, bool tma, int th) {
         if (mode == MODE_SAT && dtype != SAT_FLOAT64 && th >= 128) return 128;
         return 32;
     }
-    if (mode != MODE_SAT && dtype != SAT_FLOAT64 && th >= 128) return 128;
+    if (mode != MODE_SAT && th >= 128) return 128;          // float64: 64-column chunks
     if (mode != MODE_SAT) return th >= 64 ? 64 : 32;
     if (dtype == SAT_FLOAT64) return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
     return th >= 128 ? 128 : th >= 64 ? 64 : th >= 32 ? 32 : 16;
@@ -426,6 +426,8 @@ int launch_band_th(int th, const BandParams& p, const CUtensorMap& ti, const Dev
             return launch_band_t<T, SAT_CFG(kCfg32), MODE, TMA, kCfg32.MINB>(p, ti, di, st, grid);
     } else if constexpr (MODE != MODE_SAT) {
         if constexpr (sizeof(T) == 8) {
+            if (th == 128)
+                return launch_band_t<T, SAT_CFG(kCfgD128), MODE, TMA, kCfgD128.MINB, kLbwD, T, kTwD128>(p, ti, di, st, grid);
             if (th == 64) return launch_band_t<T, SAT_CFG(kCfgD64), MODE, TMA, kCfgD64.MINB>(p, ti, di, st, grid);
             return launch_band_t<T, SAT_CFG(kCfgD32), MODE, TMA, kCfgD32.MINB>(p, ti, di, st, grid);
         } else {
@@ -601,7 +603,7 @@ int run_band(const Job& j0, int mode, const void* in, void* out, BandParams p) {
     p.cols = j.cols;
     p.batch = int(j.batch);
     // chunk width: 64 columns for float64 at TH 128 (kCfgD128), else 128
-    const int tw = (mode == MODE_SAT && j.tma && j.dtype == SAT_FLOAT64 && j.th == 128) ? kTwD128 : TW;
+    const int tw = (j.tma && j.dtype == SAT_FLOAT64 && j.th == 128) ? kTwD128 : TW;
     p.nb = int((j.rows + j.th - 1) / j.th);
     p.nc = int((j.cols + tw - 1) / tw);
     p.total_bands = int(j.batch * p.nb);
@@ -882,8 +884,7 @@ int run_4r4w(const Job& j, const sat_options& o) {
     SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * esize(j.dtype), false));
     // column passes at TH 128 where plain 1R1W takes it (as in 2R2W)
     auto col_th = [&](int64_t rows, int th) {
-        if (!o.tile_rows && j.dtype != SAT_FLOAT64 && auto_th(rows, j.batch, *j.di, SAT_1R1W, j.dtype) == 128)
-            return 128;
+        if (!o.tile_rows && auto_th(rows, j.batch, *j.di, SAT_1R1W, j.dtype) == 128) return 128;
         return th;
     };
     Job j1 = j;
@@ -986,8 +987,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             // both passes take the TH-128 configuration where plain 1R1W
             // does: 16384^2 int32 0.851 -> 0.797 ms (column pass) -> 0.759
             // (and the row pass), 18432^2 1.049 -> 0.987
-            if (!o.tile_rows && dtype != SAT_FLOAT64 && auto_th(rows, batch, di, SAT_1R1W, dtype) == 128)
-                j1.th = 128;
+            if (!o.tile_rows && auto_th(rows, batch, di, SAT_1R1W, dtype) == 128) j1.th = 128;
             BandParams pc = base_params();
             if (cs && cs->n > 0) pc.cseed = *cs;
             SAT_TRY(run_band(j1, MODE_COL, in, out, pc));
