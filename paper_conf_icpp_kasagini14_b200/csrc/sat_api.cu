@@ -526,9 +526,15 @@ int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dty
         if (b64 * 10 >= 6LL * di.sms) return 64;
         return rows * batch >= 512 ? 32 : 16;
     }
-    // 2R1W: TH 128 where plain 1R1W takes it (its Step-3 band kernel is the
-    // 1R1W one with external carries): 16384^2 int32 0.596 -> 0.569 ms
-    if (variant == SAT_2R1W && batch * ((rows + 127) / 128) * 100 >= 65LL * di.sms) return 128;
+    // 2R1W (its Step-3 band kernel is the 1R1W one with external carries,
+    // no look-back chain, so tall bands pay off earlier): TH 128 from 64
+    // bands of 128 rows, else TH 64 from 32 bands of 64 rows (int32 sweep:
+    // 16384^2 0.596 -> 0.569 ms, 12288^2 428 -> 331 us, 8192^2 208 -> 165,
+    // 6144^2 204 -> 120, 4096^2 93 -> 77, 2048^2 46 -> 44; 1024^2 keeps 16)
+    if (variant == SAT_2R1W) {
+        if (batch * ((rows + 127) / 128) >= 64) return 128;
+        if (batch * ((rows + 63) / 64) >= 32) return 64;
+    }
     const long long slots = 2LL * di.sms;          // 2 CTAs/SM for TH = 32/64
     for (int th : {64, 32}) {
         const long long bands = batch * ((rows + th - 1) / th);
