@@ -543,6 +543,13 @@ int auto_th(int64_t rows, int64_t batch, const DevInfo& di, int variant, int dty
     return 16;
 }
 
+// The 2R2W / 4R4W column and row passes take TH 128 from ~0.6 bands of 128
+// rows per SM (int32 sweep: 12288^2 2R2W 530 -> 456 us, 4R4W 1031 -> 919;
+// at 8192^2, 64 bands, 2R2W is 8 % slower at TH 128)
+bool pass_th128(int64_t rows, int64_t batch, const DevInfo& di) {
+    return batch * ((rows + 127) / 128) * 10 >= 6LL * di.sms;
+}
+
 struct Job {
     const void* in;
     void* out;
@@ -890,7 +897,7 @@ int run_4r4w(const Job& j, const sat_options& o) {
     SAT_TRY(ensure(ws.tr, size_t(j.batch) * j.rows * j.cols * esize(j.dtype), false));
     // column passes at TH 128 where plain 1R1W takes it (as in 2R2W)
     auto col_th = [&](int64_t rows, int th) {
-        if (!o.tile_rows && auto_th(rows, j.batch, *j.di, SAT_1R1W, j.dtype) == 128) return 128;
+        if (!o.tile_rows && pass_th128(rows, j.batch, *j.di)) return 128;
         return th;
     };
     Job j1 = j;
@@ -993,7 +1000,7 @@ int compute_core(const void* in, void* out, int64_t batch, int64_t rows, int64_t
             // both passes take the TH-128 configuration where plain 1R1W
             // does: 16384^2 int32 0.851 -> 0.797 ms (column pass) -> 0.759
             // (and the row pass), 18432^2 1.049 -> 0.987
-            if (!o.tile_rows && auto_th(rows, batch, di, SAT_1R1W, dtype) == 128) j1.th = 128;
+            if (!o.tile_rows && pass_th128(rows, batch, di)) j1.th = 128;
             BandParams pc = base_params();
             if (cs && cs->n > 0) pc.cseed = *cs;
             SAT_TRY(run_band(j1, MODE_COL, in, out, pc));
